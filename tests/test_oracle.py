@@ -1,0 +1,282 @@
+"""Pins for the CPU oracle (`-m "not gpu"`): the oracle is checked against things other than itself.
+
+Each test names what fixes the expected value: the paper's text (Fig. 2), the mathematics
+(dense brute force, identities, stencil closed forms), or an independent implementation
+(pure-Python Alg. 1, ESC, scipy on all-positive inputs).
+"""
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle import pyref
+import workloads as W
+from tests import closed_forms as CF
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _dense_pattern(M):
+    P = np.zeros((M.nrows, M.ncols), dtype=np.int64)
+    for i in range(M.nrows):
+        P[i, M.col[M.row_ptr[i]:M.row_ptr[i + 1]]] = 1
+    return P
+
+
+def _as_dense(C, shape):
+    D = np.zeros(shape)
+    for i in range(shape[0]):
+        for p in range(C["row_ptr"][i], C["row_ptr"][i + 1]):
+            D[i, C["col"][p]] = C["val"][p]
+    return D
+
+
+def _parse_golden(path):
+    rows = {}
+    for line in open(path):
+        line = line.strip()
+        if not line or line.startswith("#"):
+            continue
+        key, rest = line.split(" ", 1)
+        if key.endswith(".shape"):
+            rows[key] = tuple(int(x) for x in rest.split())
+        else:
+            idx, ents = rest.split(":", 1)
+            rows[(key, int(idx))] = ents.strip()
+    return rows
+
+
+# --------------------------------------------------------------------------------- paper pins
+
+def test_fig2_worked_example():
+    """PAPER.md §II-B L74/L78 (Fig. 2): C row 0 has exactly columns {0, 3}; C00 combines two products."""
+    g = _parse_golden(os.path.join(GOLDEN, "fig2_row0.txt"))
+    A, B = W.fig2_instance()
+    # the instance in workloads matches the golden file
+    ents = [e.split(":") for e in g[("A.row", 0)].split()]
+    assert [int(c) for c, _ in ents] == list(A.col) and [float(v) for _, v in ents] == list(A.val)
+    C = oracle.spgemm(A, B)
+    exp = [e.split(":") for e in g[("C.row", 0)].split()]
+    assert list(C["col"]) == [int(c) for c, _ in exp] == [0, 3]
+    assert list(C["val"]) == [float(v) for _, v in exp]
+    assert int(oracle.products(A, B)[0]) == int(g[("C.products_row", 0)])
+
+
+def test_csr_offsets_semantics():
+    """PAPER.md §II-A: row_offsets[r] is the start of row r in col_ids/data (0-based)."""
+    A = W.random_csr(6, 6, 0.5, seed=3)
+    D = A.dense()
+    for r in range(6):
+        for p in range(A.row_ptr[r], A.row_ptr[r + 1]):
+            assert D[r, A.col[p]] == A.val[p]
+
+
+# --------------------------------------------------------------------------------- brute force
+
+@pytest.mark.parametrize("seed", range(12))
+def test_dense_brute_force_small_integers(seed):
+    """Structure = boolean product of the patterns; values = dense product (exact for small ints)."""
+    rng = np.random.default_rng(seed)
+    m, k, n = rng.integers(0, 40, size=3)
+    A = W.random_csr(m, k, rng.uniform(0, 0.6), seed=seed, values="ones", empty_rows=0.2)
+    B = W.random_csr(k, n, rng.uniform(0, 0.6), seed=seed + 100, values="ones", empty_rows=0.2)
+    A.val = rng.integers(-4, 5, size=A.nnz).astype(np.float64)  # includes explicit zeros
+    B.val = rng.integers(-4, 5, size=B.nnz).astype(np.float64)
+    C = oracle.spgemm(A, B)
+    pat = (_dense_pattern(A) @ _dense_pattern(B)) > 0
+    # structure, row by row, sorted
+    for i in range(m):
+        assert list(C["col"][C["row_ptr"][i]:C["row_ptr"][i + 1]]) == list(np.nonzero(pat[i])[0])
+    D = A.dense() @ B.dense()
+    assert np.array_equal(_as_dense(C, (m, n)), D)
+    # products per row = sum over A_ik of nnz(B_k*)
+    pa, pb = _dense_pattern(A), _dense_pattern(B)
+    assert np.array_equal(oracle.products(A, B), pa @ pb.sum(axis=1))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_dense_brute_force_reals_within_bound(seed):
+    rng = np.random.default_rng(seed)
+    m, k, n = rng.integers(1, 64, size=3)
+    A = W.random_csr(m, k, 0.3, seed=seed)
+    B = W.random_csr(k, n, 0.3, seed=seed + 7)
+    C = oracle.spgemm(A, B)
+    D = A.dense() @ B.dense()
+    absD = np.abs(A.dense()) @ np.abs(B.dense())
+    got = _as_dense(C, (m, n))
+    assert np.all(np.abs(got - D) <= 1e-13 * absD + 0.0)
+    # tolerance = 1e-12 * sum |a*b| (checked against the dense |A||B| product)
+    for i in range(m):
+        for p in range(C["row_ptr"][i], C["row_ptr"][i + 1]):
+            j = C["col"][p]
+            assert abs(C["tol"][p] - 1e-12 * absD[i, j]) <= 1e-26 + 1e-15 * C["tol"][p]
+            assert abs(C["ref"][p] - D[i, j]) <= 1e-14 * absD[i, j]
+    # fp64 Alg.1 value within the bound of the extended reference
+    assert oracle.compare(C["row_ptr"], C["col"], C["val"], C)["ok"]
+
+
+# --------------------------------------------------------------------------------- identities
+
+def test_identity_right_and_left_bit_exact():
+    A = W.random_csr(50, 37, 0.2, seed=5, empty_rows=0.1)
+    C = oracle.spgemm(A, W.identity(37))
+    assert np.array_equal(C["row_ptr"], A.row_ptr) and np.array_equal(C["col"], A.col)
+    assert np.array_equal(C["val"], A.val)
+    C = oracle.spgemm(W.identity(50), A)
+    assert np.array_equal(C["row_ptr"], A.row_ptr) and np.array_equal(C["col"], A.col)
+    assert np.array_equal(C["val"], A.val)
+
+
+def test_permutations():
+    """(P A Q)[i, j] = A[p(i), q^-1(j)] -- a transposed operand or wrong index fails this."""
+    rng = np.random.default_rng(1)
+    A = W.random_csr(30, 40, 0.2, seed=9)
+    p, q = rng.permutation(30), rng.permutation(40)
+    PA = oracle.spgemm(W.permutation(p), A)
+    PAQ = oracle.spgemm(type(A)(30, 40, PA["row_ptr"], PA["col"], PA["val"]), W.permutation(q))
+    D = A.dense()
+    expect = np.zeros_like(D)
+    expect[:, q] = D[p, :]
+    assert np.array_equal(_as_dense(PAQ, (30, 40)), expect)
+
+
+def test_sum_identity_and_freivalds():
+    A = W.random_csr_sparse(3000, 2500, 6.0, seed=2)
+    B = W.random_csr_sparse(2500, 2800, 5.0, seed=3)
+    C = oracle.spgemm(A, B)
+    colsumA = np.bincount(A.col, weights=A.val, minlength=A.ncols)
+    rowsumB = np.add.reduceat(B.val, B.row_ptr[:-1]) * (np.diff(B.row_ptr) > 0)
+    total = float(np.dot(colsumA, rowsumB))
+    assert abs(C["val"].sum() - total) <= 1e-9 * (np.abs(A.val).sum() * np.abs(B.val).max())
+    rng = np.random.default_rng(0)
+    x = rng.choice([-1.0, 1.0], size=B.ncols)
+    SA, SB = A.to_scipy(), B.to_scipy()
+    Cs = type(A)(A.nrows, B.ncols, C["row_ptr"], C["col"], C["val"]).to_scipy()
+    lhs = Cs @ x
+    rhs = SA @ (SB @ x)
+    bound = abs(SA) @ (abs(SB) @ np.abs(x))
+    assert np.all(np.abs(lhs - rhs) <= 1e-12 * bound + 1e-300)
+
+
+def test_scipy_all_positive():
+    """scipy's csr product drops exact-zero sums; with positive values none occur (R1)."""
+    A = W.random_csr_sparse(800, 700, 8.0, seed=11, values="positive")
+    B = W.random_csr_sparse(700, 900, 8.0, seed=12, values="positive")
+    C = oracle.spgemm(A, B)
+    S = (A.to_scipy() @ B.to_scipy()).tocsr()
+    S.sort_indices()
+    assert np.array_equal(C["row_ptr"], S.indptr) and np.array_equal(C["col"], S.indices)
+    assert np.all(np.abs(C["val"] - S.data) <= C["tol"])
+
+
+def test_structural_cancellation_kept():
+    """Alg. 1 L42-44 inserts on first touch whatever the value: an exact-zero sum stays stored."""
+    A = W.CSR(1, 2, np.array([0, 2], np.int64), np.array([0, 1], np.int32), np.array([1.0, 1.0]))
+    B = W.CSR(2, 3, np.array([0, 2, 3], np.int64), np.array([0, 2, 2], np.int32), np.array([1.0, 5.0, -5.0]))
+    C = oracle.spgemm(A, B)
+    assert list(C["col"]) == [0, 2] and list(C["val"]) == [1.0, 0.0]
+    assert C["tol"][1] > 0 and oracle.compare(C["row_ptr"], C["col"], C["val"], C)["ok"]
+    # explicit zero in A still generates structure
+    A0 = W.CSR(1, 1, np.array([0, 1], np.int64), np.array([0], np.int32), np.array([0.0]))
+    B0 = W.CSR(1, 2, np.array([0, 2], np.int64), np.array([0, 1], np.int32), np.array([3.0, 4.0]))
+    C0 = oracle.spgemm(A0, B0)
+    assert list(C0["col"]) == [0, 1] and list(C0["val"]) == [0.0, 0.0] and list(C0["tol"]) == [0.0, 0.0]
+
+
+@pytest.mark.parametrize("shape", [(0, 5, 4), (5, 0, 4), (5, 4, 0), (0, 0, 0), (3, 3, 3)])
+def test_degenerate_shapes(shape):
+    m, k, n = shape
+    A = W.random_csr(m, k, 0.0 if shape == (3, 3, 3) else 0.5, seed=1)
+    B = W.random_csr(k, n, 0.5, seed=2)
+    C = oracle.spgemm(A, B)
+    assert len(C["row_ptr"]) == m + 1 and C["row_ptr"][-1] == 0 and len(C["col"]) == 0
+
+
+def test_shape_mismatch_rejected():
+    with pytest.raises(ValueError):
+        oracle.spgemm(W.random_csr(3, 4, 0.5, 1), W.random_csr(5, 3, 0.5, 2))
+
+
+# --------------------------------------------------------------------------------- independent impls
+
+@pytest.mark.parametrize("seed", range(5))
+def test_python_alg1_and_esc_bit_exact(seed):
+    A = W.random_csr_sparse(120, 90, 4.0, seed=seed)
+    B = W.random_csr_sparse(90, 110, 4.0, seed=seed + 50)
+    C = oracle.spgemm(A, B)
+    rp, col, val = pyref.gustavson(A, B)
+    assert list(C["row_ptr"]) == rp and list(C["col"]) == col and list(C["val"]) == val
+    E = oracle.spgemm(A, B, method="esc")
+    assert np.array_equal(E["col"], C["col"]) and np.array_equal(E["val"], C["val"])
+
+
+def test_thread_count_and_row_selection_invariance():
+    A = W.rmat(10, 8, seed=4)
+    C1 = oracle.spgemm(A, A, threads=1)
+    C4 = oracle.spgemm(A, A, threads=4)
+    for k in ("row_ptr", "col", "val", "ref", "tol"):
+        assert np.array_equal(C1[k], C4[k])
+    rows = np.array([5, 0, 5, A.nrows - 1, 17])
+    S = oracle.spgemm(A, A, rows=rows)
+    for t, r in enumerate(rows):
+        a, b = C1["row_ptr"][r], C1["row_ptr"][r + 1]
+        c, d = S["row_ptr"][t], S["row_ptr"][t + 1]
+        assert np.array_equal(S["col"][c:d], C1["col"][a:b]) and np.array_equal(S["val"][c:d], C1["val"][a:b])
+
+
+# --------------------------------------------------------------------------------- stencil closed forms
+
+def test_c1_closed_form_full():
+    """BASELINE config 0 in full: C1 = A^2 for the 64x64 5-point Laplacian (closed form, exact)."""
+    A = W.stencil_2d5(64)
+    assert A.nnz == 20224
+    C = oracle.spgemm(A, A)
+    assert int(oracle.products(A, A).sum()) == CF.c1_products_total(64) == 100104
+    assert C["row_ptr"][-1] == CF.c1_pattern_count(64) == 51972
+    i = np.repeat(np.arange(A.nrows), np.diff(C["row_ptr"]))
+    j = C["col"].astype(np.int64)
+    assert np.all((np.abs(i % 64 - j % 64) + np.abs(i // 64 - j // 64)) <= 2)
+    assert np.array_equal(C["val"], CF.c1_entry(64, i, j))
+    assert C["val"].sum() == 264.0
+
+
+@pytest.mark.parametrize("n", [5, 8, 12])
+def test_c2_closed_form_small(n):
+    """BASELINE config 1 at small n: C = 729 I - 54 S + K^2 (x) K^2 (x) K^2 entrywise."""
+    A = W.stencil_3d27(n)
+    C = oracle.spgemm(A, A)
+    rows = np.arange(A.nrows)
+    assert np.array_equal(oracle.products(A, A), CF.c2_row_products(n, rows))
+    assert np.array_equal(np.diff(C["row_ptr"]), CF.c2_row_nnz(n, rows))
+    for r in (0, 1, n + 1, A.nrows // 2, A.nrows - 1):
+        assert np.array_equal(C["col"][C["row_ptr"][r]:C["row_ptr"][r + 1]], CF.c2_row_cols(n, r))
+    i = np.repeat(rows, np.diff(C["row_ptr"]))
+    assert np.array_equal(C["val"], CF.c2_entry(n, i, C["col"].astype(np.int64)))
+    assert C["val"].sum() == CF.c2_sum(n)
+    p, z = CF.c2_totals(n)
+    assert p == int(oracle.products(A, A).sum()) and z == int(C["row_ptr"][-1])
+
+
+def test_c2_full_size_totals_formula():
+    """The n = 128 figures quoted in SURVEY §8.0 follow from the per-axis closed forms."""
+    p, z = CF.c2_totals(128)
+    assert p == 1142 ** 3 == 1489355288 and z == 634 ** 3 == 254840104
+    assert CF.c2_sum(128) == 8058824.0
+    A = W.stencil_3d27(128)
+    assert A.nnz == 382 ** 3 == 55742968
+    # products of the full matrix by an O(nnz) count independent of the oracle:
+    nnz_row = np.diff(A.row_ptr)
+    colcount = np.bincount(A.col, minlength=A.ncols)
+    assert int(np.dot(colcount, nnz_row)) == p
+
+
+def test_sampled_rows_full_c2():
+    """Oracle rows of the full 128^3 problem agree with the closed form (the GPU full-size pin)."""
+    A = W.stencil_3d27(128)
+    rng = np.random.default_rng(0)
+    rows = np.concatenate([[0, 127, 128 * 128 - 1, A.nrows - 1], rng.integers(0, A.nrows, 200)])
+    S = oracle.spgemm(A, A, rows=rows)
+    assert np.array_equal(np.diff(S["row_ptr"]), CF.c2_row_nnz(128, rows))
+    i = np.repeat(rows, np.diff(S["row_ptr"]))
+    assert np.array_equal(S["val"], CF.c2_entry(128, i, S["col"].astype(np.int64)))
