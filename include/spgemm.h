@@ -1,0 +1,182 @@
+/*
+ * include/spgemm.h -- C ABI of the B200-native out-of-core chunked SpGEMM  C = A x B  (CSR).
+ *
+ * Method: Xia, Jiang, Agrawal, Ramnath, "Scaling Sparse Matrix Multiplication on CPU-GPU Nodes",
+ * IPDPS'21.  Row panels of A times column panels of B give independent chunks of C
+ * (Alg. 3, §III-A); each chunk is computed in-core on the GPU by a two-phase hash
+ * SpGEMM -- per-row product count ("row analysis", §III-B), symbolic hash pass giving nnz
+ * per row (L126, §II-B), exclusive scan (L126), numeric hash accumulate + per-row sort
+ * (§II-B, §III-B) -- into buffers preallocated in one device arena with no allocation
+ * during compute (§IV-B), and every finished chunk streams to host memory over
+ * asynchronous D2H copies overlapped with the next chunk's compute (two+ streams, two+ device
+ * buffers, pinned host memory: §IV-B).
+ *
+ * All entry points are extern "C", take plain pointers and sizes, and return spgemm_status.
+ * No PyTorch type appears here; the Python binding passes device pointers it allocated with
+ * torch and a cudaStream_t as `void *`.
+ *
+ * Data layout (reading R3): CSR with int64 row_ptr [nrows+1] (row_ptr[0] == 0 for host
+ * inputs; any base for device inputs, see spgemm_csr), int32 col_idx sorted strictly increasing in
+ * every row (§II-A), fp64 values (§V-B "double").  Output C uses the same layout; its
+ * rows are sorted by column (§II-B), and entries are STRUCTURAL: a sum that cancels to 0.0 is
+ * stored (Alg. 1 L42-44; reading R1).  Values are the fp64 sums of the products in some order;
+ * each satisfies |c - c_exact| <= 1e-12 * sum_k |a_ik * b_kj| (BASELINE.json north_star).
+ *
+ * Errors: every call returns a status; on error a thread-local message is available from
+ * spgemm_last_error(), out-parameters are left untouched (plan_out is set to NULL), and the
+ * library has released whatever the failed call allocated.  No call aborts the process.
+ *
+ * Threading: a plan is used by one host thread at a time; distinct plans are independent.
+ */
+#ifndef SPGEMM_B200_H
+#define SPGEMM_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SPGEMM_ABI_VERSION 1
+
+typedef enum {
+    SPGEMM_OK = 0,
+    SPGEMM_ERR_INVALID_ARGUMENT = 1, /* NULL pointer, bad option, or (validate=1) malformed CSR   */
+    SPGEMM_ERR_SHAPE = 2,            /* A.ncols != B.nrows, or row range outside A                 */
+    SPGEMM_ERR_INDEX_OVERFLOW = 3,   /* B.ncols > INT32_MAX (col_idx is int32)                     */
+    SPGEMM_ERR_BUDGET = 4,           /* device budget cannot hold B + row arrays + one C row       */
+    SPGEMM_ERR_HOST_ALLOC = 5,       /* pinned host allocation failed                              */
+    SPGEMM_ERR_CUDA = 6,             /* a CUDA runtime call or kernel failed                        */
+    SPGEMM_ERR_STATE = 7,            /* call on a plan that failed earlier                           */
+    SPGEMM_ERR_CAPACITY = 8,         /* caller's output capacity smaller than nnz(C)                 */
+    SPGEMM_ERR_CALLBACK = 9          /* the chunk sink returned non-zero                             */
+} spgemm_status;
+
+typedef enum { SPGEMM_HOST = 0, SPGEMM_DEVICE = 1 } spgemm_where;
+
+/* Input CSR matrix (borrowed: must stay valid and unmodified until spgemm_free of every plan
+ * built from it).  where == SPGEMM_HOST: row_ptr[0] must be 0.  where == SPGEMM_DEVICE: pointers
+ * are device pointers on opts.device (e.g. B after an NCCL broadcast); row_ptr may carry any
+ * base, i.e. row r occupies col_idx[row_ptr[r]] .. col_idx[row_ptr[r+1]-1]. */
+typedef struct {
+    int64_t nrows, ncols, nnz;
+    const int64_t *row_ptr; /* [nrows+1], non-decreasing                                         */
+    const int32_t *col_idx; /* [nnz], strictly increasing in each row, 0 <= c < ncols <= INT32_MAX */
+    const double *values;   /* [nnz]                                                             */
+    int32_t where;          /* spgemm_where                                                       */
+    int32_t reserved;
+} spgemm_csr;
+
+/* Output CSR view (plan-owned memory for spgemm_execute). */
+typedef struct {
+    int64_t nrows, ncols, nnz;
+    int64_t *row_ptr; /* [nrows+1], row_ptr[0] == opts.row_ptr_base                               */
+    int32_t *col_idx; /* [nnz]                                                                    */
+    double *values;   /* [nnz]                                                                    */
+} spgemm_csr_out;
+
+typedef struct {
+    int32_t device;        /* CUDA ordinal; -1 = the calling thread's current device                */
+    int32_t validate;      /* 1 = check both inputs on the device (sortedness, bounds, row_ptr)     */
+    int32_t ring;          /* device C chunk buffers, >= 1 (1 = synchronous ablation); default 2    */
+    int32_t profile;       /* 1 = time every kernel class with CUDA events (spgemm_stats)           */
+    int64_t row_begin;     /* rows [row_begin, row_end) of A are this plan's row panel (multi-GPU  */
+    int64_t row_end;       /*   deal, §III-A); default 0 and -1 = all rows                     */
+    void *workspace;       /* caller-owned device buffer of device_budget_bytes used as the arena   */
+                           /*   (e.g. from torch's allocator); NULL = the library cudaMallocs it     */
+    void *stream;          /* cudaStream_t for kernels; NULL = a library-created stream             */
+    int64_t chunk_nnz;     /* > 0: cap every output chunk at this many nonzeros (test hook), else   */
+                           /*   chunks are sized from the ring buffers left in the budget           */
+    int64_t row_ptr_base;  /* added to every C row_ptr value delivered to the host (rank slices)    */
+    int64_t min_chunks;    /* split C into at least this many chunks for D2H overlap; 0 = auto      */
+} spgemm_opts;
+
+typedef struct spgemm_plan_s *spgemm_plan_t;
+
+/* Fill *opts with defaults (device -1, validate 0, ring 2, rows all, library arena and stream). */
+void spgemm_opts_default(spgemm_opts *opts);
+
+/* Plan = steps S0-S5 + S10 of DESIGN.md: adopt or H2D-copy the inputs into the arena (one
+ * allocation of device_budget_bytes; 0 = 90 % of free device memory), count products per row,
+ * symbolic hash pass (nnz per row), exclusive scan to C row offsets, and cut the output into
+ * chunks that fit the ring buffers left in the budget.  Synchronises the plan's stream.
+ * Returns SPGEMM_ERR_BUDGET if B + the row arrays + one ring slot holding the longest C row do
+ * not fit.  *plan_out receives the plan (NULL on error). */
+spgemm_status spgemm_plan(const spgemm_csr *A, const spgemm_csr *B, size_t device_budget_bytes,
+                          const spgemm_opts *opts, spgemm_plan_t *plan_out);
+
+typedef struct {
+    int64_t nrows, ncols;       /* shape of this plan's C slice                                   */
+    int64_t nnz;                /* nnz of the slice                                               */
+    int64_t products;           /* sum of intermediate products (1 multiply-add each; reading R4)  */
+    int64_t max_row_nnz, max_row_products;
+    int32_t num_chunks, ring;
+    int64_t chunk_capacity;     /* nonzeros per ring buffer                                       */
+    int64_t arena_bytes, arena_used, ring_bytes;
+    int64_t rows_warp, rows_block, rows_global; /* rows per accumulator tier in the symbolic pass   */
+} spgemm_info;
+
+spgemm_status spgemm_plan_info(spgemm_plan_t plan, spgemm_info *info);
+
+/* Chunk table: chunk c covers C rows [rows[c], rows[c+1]) and nonzeros [offs[c], offs[c+1])
+ * (offsets relative to the slice).  Arrays of num_chunks+1 entries, caller-allocated. */
+spgemm_status spgemm_plan_chunks(spgemm_plan_t plan, int64_t *rows, int64_t *offs);
+
+/* Execute = steps S6-S8: numeric hash accumulate + sort per chunk into a ring buffer, each
+ * chunk D2H-copied into host memory while the next is computed.  Synchronises before return.
+ * spgemm_execute_into writes into caller memory: row_ptr [nrows+1] (may be NULL), col_idx and
+ * values [nnz]; page-locked memory (cudaHostAlloc / torch pin_memory) gives asynchronous copies,
+ * pageable memory is correct but slow.  Repeatable on the same plan. */
+spgemm_status spgemm_execute_into(spgemm_plan_t plan, int64_t *row_ptr, int32_t *col_idx, double *values);
+
+/* Same, into plan-owned pinned host memory allocated on the first call (kept until free). */
+spgemm_status spgemm_execute(spgemm_plan_t plan, spgemm_csr_out *C_out);
+
+/* Sink mode for C larger than host memory: every chunk is copied into a pinned staging ring and
+ * handed to cb (on the calling thread) while the GPU computes the next chunks.  row_ptr holds
+ * rows+1 offsets relative to the start of the chunk; the pointers are valid only during the call.
+ * A non-zero return from cb stops execution with SPGEMM_ERR_CALLBACK. */
+typedef int (*spgemm_chunk_cb)(void *user, int64_t row0, int64_t row1, const int64_t *row_ptr,
+                               const int32_t *col_idx, const double *values, int64_t nnz);
+spgemm_status spgemm_execute_stream(spgemm_plan_t plan, spgemm_chunk_cb cb, void *user);
+
+/* Change the base added to C row_ptr values (multi-GPU: global offset of this rank's slice,
+ * known after the ranks exchange their nnz).  Applies to the next execute. */
+spgemm_status spgemm_set_row_ptr_base(spgemm_plan_t plan, int64_t base);
+
+/* One-shot C = A x B on device-resident or host inputs into caller host buffers with capacity
+ * nnz_capacity; plan + execute in one call.  *nnz_out receives nnz(C) (also on CAPACITY error). */
+spgemm_status spgemm_multiply(const spgemm_csr *A, const spgemm_csr *B, size_t device_budget_bytes,
+                              const spgemm_opts *opts, int64_t *row_ptr, int32_t *col_idx, double *values,
+                              int64_t nnz_capacity, int64_t *nnz_out);
+
+/* Per-kernel-class device time of the last plan/execute when opts.profile = 1 (CUDA events on
+ * the launching stream).  name: "count", "symbolic", "scan", "numeric", "d2h", ... */
+typedef struct {
+    char name[24];
+    int32_t launches;
+    double ms;    /* total device ms over the launches */
+    double bytes; /* algorithmic bytes moved by those launches */
+} spgemm_kernel_stat;
+
+/* Fills up to max entries; returns the number of classes in *n. */
+spgemm_status spgemm_stats(spgemm_plan_t plan, spgemm_kernel_stat *stats, int32_t max, int32_t *n);
+
+/* NULL-safe; frees the arena (if library-owned), streams, events and plan-owned host memory. */
+void spgemm_free(spgemm_plan_t plan);
+
+/* Process-wide number of CUDA kernels this library has launched (all plans, all devices). */
+int64_t spgemm_kernel_launches(void);
+
+/* Release the library's cached pinned staging memory. */
+void spgemm_release_cache(void);
+
+const char *spgemm_status_string(spgemm_status s);
+const char *spgemm_last_error(void);
+int32_t spgemm_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SPGEMM_B200_H */

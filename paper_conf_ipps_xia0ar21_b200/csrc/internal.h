@@ -1,0 +1,121 @@
+// internal.h -- launch interface between the host pipeline (api.cu) and the sm_100a kernels
+// (kernels.cu).  Not part of the public ABI (include/spgemm.h).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace spg {
+
+// Device view of a CSR operand.  rp is indexed by local row (0..nrows); its values index col/val
+// directly, so a device input with an arbitrary base, or a row panel of A, needs no copy.
+struct DevCSR {
+    const int64_t *rp;
+    const int32_t *col;
+    const double *val;
+    int64_t nrows, ncols;
+};
+
+// Accumulator tiers.  A row is handled by
+//   W: one warp, shared-memory hash table of TW_* slots   (bound <= CAPW_*)
+//   B: one CTA,  shared-memory hash table of TB_* slots   (bound <= CAPB_*)
+//   G: one CTA,  dense bitmap (+ fp64 array) over all columns in arena scratch (any bound)
+// where bound = min(products, ncols) in the symbolic pass and the exact nnz in the numeric pass.
+constexpr int WARPS_W = 8;                 // warps per CTA in the W kernels
+constexpr int TW_SYM = 1024, CAPW_SYM = 768;
+constexpr int TW_NUM = 512, CAPW_NUM = 384;
+constexpr int THREADS_B = 512;
+constexpr int TB_SYM = 32768, CAPB_SYM = 24576;
+constexpr int TB_NUM = 16384, CAPB_NUM = 12288;
+constexpr int THREADS_G = 512;
+constexpr int ROW_BATCH = 16;              // rows a warp claims per atomic in the W kernels
+
+// Per-pass control block in the arena (zeroed with cudaMemsetAsync before each pass).
+struct Ctl {
+    unsigned long long row_ctr;   // W kernels: next row batch
+    unsigned int nB, nG;          // long-row list lengths
+    unsigned int err;             // bit 0: numeric count mismatch; bit 1: invalid input; bit 2: table overflow
+    unsigned int pad;
+    unsigned long long sum_u;     // count pass: sum of products
+    unsigned long long max_u;     // count pass: max products in a row
+    unsigned long long max_bound; // count pass: max min(products, ncols)
+    unsigned long long max_nnz;   // symbolic pass: max nnz in a row
+    unsigned long long rows_w, rows_b, rows_g;
+    unsigned long long pad2[6];
+};
+
+// --- launchers (all asynchronous on `s`) ---------------------------------------------------
+
+// S2: u[i] = sum_{k in A_i} nnz(B_k)  for i in [0, A.nrows)
+void launch_count(const DevCSR &A, const DevCSR &B, int64_t *u, Ctl *ctl, cudaStream_t s);
+
+// Validation of a CSR operand (rows strictly increasing, 0 <= col < ncols, rp non-decreasing).
+void launch_validate(const DevCSR &M, Ctl *ctl, cudaStream_t s);
+
+// rp[i] -= sub for i in [0, n)
+void launch_rebase(int64_t *rp, int64_t n, int64_t sub, cudaStream_t s);
+
+struct SymArgs {
+    DevCSR A, B;
+    const int64_t *u;
+    int64_t *crp;        // out: crp[i] = nnz_i (i < nrows), then scanned in place
+    int32_t *listB, *listG;
+    Ctl *ctl;
+    uint32_t *gscratch;  // G tier: per-CTA bitmap of ceil(ncols/32) words, zero on entry and exit
+    int64_t gstride;     // words per CTA slot
+    int gblocks;         // CTAs in the G kernel
+    int group;           // lanes per A entry in the W kernel (4, 8, 16, 32)
+};
+// S3+S4: symbolic pass over all rows (tiering + the three tiers).  ev: NULL or 4 events recorded
+// before W, between W/B, between B/G and after G (per-kernel timing on the launching stream).
+void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);
+
+// S5: in-place exclusive scan of crp[0..n] (n+1 entries, crp[n] must be 0 on entry), plus base.
+// tmp: >= 2 * ceil((n+1)/SCAN_TILE) + 64 int64 of scratch.
+constexpr int SCAN_TILE = 4096;
+void launch_scan(int64_t *crp, int64_t n, int64_t base, int64_t *tmp, cudaStream_t s);
+
+// chunk ids: bounds[c] = first row whose offset - crp[0] >= c * cap_prime (empty ids repeat);
+// bounds has nids+1 entries with bounds[nids] = n.
+void launch_cut(const int64_t *crp, int64_t n, int64_t cap_prime, int64_t *bounds, int64_t nids, cudaStream_t s);
+
+// crp[i] += delta for i in [0, n]
+void launch_add(int64_t *crp, int64_t n, int64_t delta, cudaStream_t s);
+
+struct NumArgs {
+    DevCSR A, B;
+    const int64_t *crp;  // scanned offsets (any base)
+    int64_t r0, r1;      // chunk rows
+    int32_t *out_col;    // ring slot: nnz of the chunk
+    double *out_val;
+    int32_t *listB, *listG;
+    Ctl *ctl;
+    uint32_t *gbits;     // G tier scratch: per CTA gstride_bits words of bitmap ...
+    double *gvals;       // ... and gstride_vals doubles, all zero on entry and exit
+    int64_t gstride_bits, gstride_vals;
+    int gblocks;
+    int group;
+};
+// S6+S7: numeric pass over chunk rows [r0, r1); ev as in launch_symbolic
+void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);
+
+// out[i] = crp[idx[i]]
+void launch_gather(const int64_t *crp, const int64_t *idx, int64_t n, int64_t *out, cudaStream_t s);
+
+// lanes per A entry for the W kernels from B's average row length
+int choose_group(const DevCSR &B, int64_t nnzB);
+
+// occupancy-derived grid sizes (queried once per device)
+struct Grids {
+    int count_blocks, symw_blocks, numw_blocks, symb_blocks, numb_blocks;
+};
+const Grids &grids(int device, int num_sms);
+
+// process-wide count of kernels launched by the library
+long long kernel_launches();
+
+size_t symw_smem();
+size_t numw_smem();
+size_t symb_smem();
+size_t numb_smem();
+
+}  // namespace spg

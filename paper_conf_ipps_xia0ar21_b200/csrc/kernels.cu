@@ -1,0 +1,841 @@
+// kernels.cu -- sm_100a kernels of the out-of-core chunked SpGEMM hot path.
+//
+// Steps (DESIGN.md §8 rows; PAPER.md anchors):
+//   S2 count     k_count        products per row ("row analysis", §III-B; Alg. 1 line-4 trip count)
+//   S3 tiering   inside k_sym_w / k_num_w: rows too long for a warp are appended to the CTA (B) or
+//                dense-global (G) list on the device -- the paper's host-side row grouping after a
+//                D2H (§III-B, §IV-B) is replaced by device-side lists, no transfer.
+//   S4 symbolic  k_sym_w / k_sym_b / k_sym_g   (hash set of column ids -> nnz per row, §II-B)
+//   S5 scan      k_scan_{reduce,top,apply}     (row offsets of C, §III-B)
+//   S6 numeric   k_num_w / k_num_b / k_num_g   (hash / dense accumulation, §II-B, §III-B)
+//   S7 sort      in the numeric kernels: in-place compaction + bitonic sort by column (§II-B)
+//
+// No tensor cores: this is not a dense contraction.  Hash tables live in shared memory (W, B
+// tiers); the G tier is a dense bitmap + fp64 array over all columns in arena scratch (the
+// "dense accumulation" of §II-B L107 / §III-B, used here for the longest rows).
+#include <climits>
+#include <cstdio>
+
+#include <atomic>
+
+#include "internal.h"
+
+namespace spg {
+
+static std::atomic<long long> g_launches{0};
+long long kernel_launches() { return g_launches.load(); }
+#define LAUNCHED(n) g_launches.fetch_add((n), std::memory_order_relaxed)
+
+#define FULLMASK 0xffffffffu
+constexpr int32_t EMPTY = -1;
+
+__device__ __forceinline__ uint32_t hslot(int32_t c, int lg) {
+    return ((uint32_t)c * 0x9E3779B1u) >> (32 - lg);
+}
+
+// log2 of the table size for a row with `bound` distinct keys: load factor <= 3/4, >= 32 slots
+__device__ __forceinline__ int table_log2(int64_t bound, int maxlg) {
+    int64_t need = bound + bound / 3 + 1;
+    int lg = 5;
+    while (lg < maxlg && (int64_t(1) << lg) < need) ++lg;
+    return lg;
+}
+
+// symbolic insert: returns 1 if `c` was not yet in the table
+__device__ __forceinline__ int sym_insert(int32_t *keys, int32_t c, int lg) {
+    const uint32_t mask = (1u << lg) - 1;
+    uint32_t h = hslot(c, lg);
+    volatile int32_t *vk = keys;
+    while (true) {
+        int32_t k = vk[h];
+        if (k == c) return 0;
+        if (k == EMPTY) {
+            int32_t old = atomicCAS(&keys[h], EMPTY, c);
+            if (old == EMPTY) return 1;
+            if (old == c) return 0;
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+// numeric insert-or-add (Alg. 1 lines 6-10 with a hash map instead of a list)
+__device__ __forceinline__ void num_insert(int32_t *keys, double *vals, int32_t c, double v, int lg) {
+    const uint32_t mask = (1u << lg) - 1;
+    uint32_t h = hslot(c, lg);
+    volatile int32_t *vk = keys;
+    while (true) {
+        int32_t k = vk[h];
+        if (k == c) break;
+        if (k == EMPTY) {
+            int32_t old = atomicCAS(&keys[h], EMPTY, c);
+            if (old == EMPTY || old == c) break;
+        }
+        h = (h + 1) & mask;
+    }
+    atomicAdd(&vals[h], v);
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(FULLMASK, v, d);
+    return v;
+}
+
+// exclusive block scan of one int64 per thread; s has >= 33 entries; returns exclusive prefix,
+// *total = block sum.  All threads must call.
+template <int NT>
+__device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t *s, int64_t *total) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int64_t x = v;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        int64_t t = __shfl_up_sync(FULLMASK, x, d);
+        if (lane >= d) x += t;
+    }
+    if (lane == 31) s[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+        int64_t w = lane < NT / 32 ? s[lane] : 0;
+        int64_t y = w;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+            int64_t t = __shfl_up_sync(FULLMASK, y, d);
+            if (lane >= d) y += t;
+        }
+        if (lane < NT / 32) s[lane] = y - w;
+        if (lane == 31) s[32] = y;
+    }
+    __syncthreads();
+    int64_t r = x - v + s[wid];
+    *total = s[32];
+    __syncthreads();
+    return r;
+}
+
+// ------------------------------------------------------------------------------------------ S2
+
+__global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__restrict__ u, Ctl *ctl) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+    unsigned long long lsum = 0, lmax = 0, lmaxb = 0;
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < A.nrows; i += nw) {
+        const int64_t s = A.rp[i], e = A.rp[i + 1];
+        int64_t acc = 0;
+        for (int64_t p = s + lane; p < e; p += 32) {
+            const int32_t k = __ldg(&A.col[p]);
+            acc += __ldg(&B.rp[k + 1]) - __ldg(&B.rp[k]);
+        }
+        acc = warp_sum(acc);
+        if (lane == 0) {
+            u[i] = acc;
+            lsum += acc;
+            lmax = max(lmax, (unsigned long long)acc);
+            lmaxb = max(lmaxb, (unsigned long long)min(acc, B.ncols));
+        }
+    }
+    if (lane == 0 && lsum) {
+        atomicAdd(&ctl->sum_u, lsum);
+        atomicMax(&ctl->max_u, lmax);
+        atomicMax(&ctl->max_bound, lmaxb);
+    }
+}
+
+// --------------------------------------------------------------------------------- validation
+
+__global__ void k_validate(DevCSR M, Ctl *ctl) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < M.nrows; i += nw) {
+        const int64_t s = M.rp[i], e = M.rp[i + 1];
+        bool bad = e < s;
+        if (!bad)
+            for (int64_t p = s + lane; p < e; p += 32) {
+                const int32_t c = M.col[p];
+                if (c < 0 || c >= M.ncols || (p > s && M.col[p - 1] >= c)) bad = true;
+            }
+        if (__any_sync(FULLMASK, bad) && lane == 0) atomicOr(&ctl->err, 2u);
+    }
+}
+
+__global__ void k_rebase(int64_t *rp, int64_t n, int64_t sub) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        rp[i] -= sub;
+}
+
+__global__ void k_add(int64_t *rp, int64_t n, int64_t d) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        rp[i] += d;
+}
+
+// ------------------------------------------------------------------------ tier classification
+
+__device__ __forceinline__ void push_long(int64_t i, int64_t bound, int64_t capB, int32_t *listB, int32_t *listG,
+                                          Ctl *ctl) {
+    if (bound <= capB) {
+        unsigned idx = atomicAdd(&ctl->nB, 1u);
+        listB[idx] = (int32_t)i;
+    } else {
+        unsigned idx = atomicAdd(&ctl->nG, 1u);
+        listG[idx] = (int32_t)i;
+    }
+}
+
+// ----------------------------------------------------------------------------- S4 symbolic, W
+//
+// One warp per row; rows are claimed ROW_BATCH at a time from a global counter (dynamic load
+// balance for skewed rows).  Lanes form 32/G groups of G: each group takes one A entry A_ik and
+// its lanes stride over B_k* (coalesced col loads).  Keys go to the warp's shared-memory table.
+
+template <int G>
+__global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
+    extern __shared__ int32_t smem_i[];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int32_t *keys = smem_i + wid * TW_SYM;
+    const int64_t R = a.A.nrows, ncols = a.B.ncols;
+    unsigned long long lmax = 0, nw = 0, nlong = 0;
+    constexpr int MAXLG = 10;  // log2(TW_SYM)
+    while (true) {
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(&a.ctl->row_ctr, (unsigned long long)ROW_BATCH);
+        base = __shfl_sync(FULLMASK, base, 0);
+        if ((int64_t)base >= R) break;
+        const int64_t end = min((int64_t)base + ROW_BATCH, R);
+        for (int64_t i = (int64_t)base; i < end; ++i) {
+            const int64_t bound = min(a.u[i], ncols);
+            if (bound == 0) {
+                if (lane == 0) a.crp[i] = 0;
+                continue;
+            }
+            if (bound > CAPW_SYM) {
+                if (lane == 0) {
+                    push_long(i, bound, CAPB_SYM, a.listB, a.listG, a.ctl);
+                    nlong++;
+                }
+                continue;
+            }
+            const int lg = table_log2(bound, MAXLG);
+            const int T = 1 << lg;
+            for (int t = lane; t < T; t += 32) keys[t] = EMPTY;
+            __syncwarp();
+            int cnt = 0;
+            const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
+            for (int64_t p0 = as; p0 < ae; p0 += 32 / G) {
+                const int64_t p = p0 + lane / G;
+                if (p < ae) {
+                    const int32_t k = __ldg(&a.A.col[p]);
+                    const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
+                    for (int64_t q = bs + (lane % G); q < be; q += G) cnt += sym_insert(keys, __ldg(&a.B.col[q]), lg);
+                }
+            }
+            cnt = warp_sum(cnt);
+            if (lane == 0) {
+                a.crp[i] = cnt;
+                lmax = max(lmax, (unsigned long long)cnt);
+                nw++;
+            }
+            __syncwarp();
+        }
+    }
+    if (lane == 0) {
+        if (lmax) atomicMax(&a.ctl->max_nnz, lmax);
+        if (nw) atomicAdd(&a.ctl->rows_w, nw);
+    }
+}
+
+// ----------------------------------------------------------------------------- S4 symbolic, B
+
+__global__ void __launch_bounds__(THREADS_B) k_sym_b(SymArgs a) {
+    extern __shared__ int32_t keys[];
+    __shared__ int64_t s_scan[40];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    constexpr int NW = THREADS_B / 32;
+    constexpr int MAXLG = 15;  // log2(TB_SYM)
+    const unsigned n = *(volatile unsigned *)&a.ctl->nB;
+    const int64_t ncols = a.B.ncols;
+    for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
+        const int64_t i = a.listB[idx];
+        const int64_t bound = min(a.u[i], ncols);
+        const int lg = table_log2(bound, MAXLG);
+        const int T = 1 << lg;
+        for (int t = threadIdx.x; t < T; t += THREADS_B) keys[t] = EMPTY;
+        __syncthreads();
+        int cnt = 0;
+        const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
+        for (int64_t p = as + wid; p < ae; p += NW) {
+            const int32_t k = __ldg(&a.A.col[p]);
+            const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
+            for (int64_t q = bs + lane; q < be; q += 32) cnt += sym_insert(keys, __ldg(&a.B.col[q]), lg);
+        }
+        int64_t tot;
+        block_excl_scan<THREADS_B>(cnt, s_scan, &tot);
+        if (threadIdx.x == 0) {
+            a.crp[i] = tot;
+            atomicMax(&a.ctl->max_nnz, (unsigned long long)tot);
+            atomicAdd(&a.ctl->rows_b, 1ull);
+        }
+        __syncthreads();
+    }
+}
+
+// ----------------------------------------------------------------------------- S4 symbolic, G
+// Dense bitmap over all columns in this CTA's arena slot; atomicOr's return tells whether the
+// column is new.  The bitmap is cleared again before the next row (by re-walking the products
+// when that is cheaper than a sweep).
+
+__global__ void __launch_bounds__(THREADS_G) k_sym_g(SymArgs a) {
+    __shared__ int64_t s_scan[40];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    constexpr int NW = THREADS_G / 32;
+    uint32_t *bm = a.gscratch + (int64_t)blockIdx.x * a.gstride;
+    const unsigned n = *(volatile unsigned *)&a.ctl->nG;
+    const int64_t nwords = (a.B.ncols + 31) / 32;
+    for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
+        const int64_t i = a.listG[idx];
+        int cnt = 0;
+        const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
+        for (int64_t p = as + wid; p < ae; p += NW) {
+            const int32_t k = __ldg(&a.A.col[p]);
+            const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
+            for (int64_t q = bs + lane; q < be; q += 32) {
+                const int32_t c = __ldg(&a.B.col[q]);
+                const uint32_t bit = 1u << (c & 31);
+                const uint32_t old = atomicOr(&bm[c >> 5], bit);
+                cnt += (old & bit) ? 0 : 1;
+            }
+        }
+        int64_t tot;
+        block_excl_scan<THREADS_G>(cnt, s_scan, &tot);
+        if (threadIdx.x == 0) {
+            a.crp[i] = tot;
+            atomicMax(&a.ctl->max_nnz, (unsigned long long)tot);
+            atomicAdd(&a.ctl->rows_g, 1ull);
+        }
+        // clear (block_excl_scan ended with a barrier, so all atomics of this row are done)
+        if (a.u[i] < nwords) {
+            for (int64_t p = as + wid; p < ae; p += NW) {
+                const int32_t k = __ldg(&a.A.col[p]);
+                const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
+                for (int64_t q = bs + lane; q < be; q += 32) bm[__ldg(&a.B.col[q]) >> 5] = 0u;
+            }
+        } else {
+            for (int64_t w = threadIdx.x; w < nwords; w += THREADS_G) bm[w] = 0u;
+        }
+        __syncthreads();
+    }
+}
+
+// ------------------------------------------------------------------------------------- S5 scan
+
+__global__ void __launch_bounds__(1024) k_scan_reduce(const int64_t *__restrict__ x, int64_t n1,
+                                                      int64_t *__restrict__ part) {
+    __shared__ int64_t s[40];
+    const int64_t b0 = (int64_t)blockIdx.x * SCAN_TILE;
+    int64_t v = 0;
+#pragma unroll
+    for (int t = 0; t < SCAN_TILE / 1024; ++t) {
+        const int64_t i = b0 + (int64_t)threadIdx.x * (SCAN_TILE / 1024) + t;
+        if (i < n1) v += x[i];
+    }
+    int64_t tot;
+    block_excl_scan<1024>(v, s, &tot);
+    if (threadIdx.x == 0) part[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(1024) k_scan_top(int64_t *part, int64_t nb, int64_t base) {
+    __shared__ int64_t s[40];
+    int64_t carry = base;
+    for (int64_t b0 = 0; b0 < nb; b0 += 1024) {
+        const int64_t i = b0 + threadIdx.x;
+        const int64_t v = i < nb ? part[i] : 0;
+        int64_t tot;
+        const int64_t ex = block_excl_scan<1024>(v, s, &tot);
+        if (i < nb) part[i] = carry + ex;
+        carry += tot;
+    }
+}
+
+__global__ void __launch_bounds__(1024) k_scan_apply(int64_t *__restrict__ x, int64_t n1,
+                                                     const int64_t *__restrict__ part) {
+    __shared__ int64_t s[40];
+    constexpr int PER = SCAN_TILE / 1024;
+    const int64_t b0 = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * PER;
+    int64_t v[PER];
+    int64_t sum = 0;
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+        v[t] = (b0 + t < n1) ? x[b0 + t] : 0;
+        sum += v[t];
+    }
+    int64_t tot;
+    int64_t run = block_excl_scan<1024>(sum, s, &tot) + part[blockIdx.x];
+#pragma unroll
+    for (int t = 0; t < PER; ++t) {
+        if (b0 + t < n1) x[b0 + t] = run;
+        run += v[t];
+    }
+}
+
+// ------------------------------------------------------------------------------- chunk cutting
+
+__global__ void k_fill(int64_t *b, int64_t n, int64_t v) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        b[i] = v;
+}
+
+__global__ void k_cut(const int64_t *__restrict__ crp, int64_t n, int64_t capp, int64_t *__restrict__ bounds,
+                      int64_t nids) {
+    const int64_t off0 = crp[0];
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t ci = (crp[i] - off0) / capp;
+        const int64_t cp = i == 0 ? -1 : (crp[i - 1] - off0) / capp;
+        for (int64_t c = cp + 1; c <= ci && c < nids; ++c) bounds[c] = i;
+    }
+}
+
+// ------------------------------------------------------------------------------ S7 sort helpers
+
+// warp bitonic sort of (keys, vals)[0..N) ascending by key, N a power of two >= 32
+__device__ __forceinline__ void warp_bitonic(int32_t *keys, double *vals, int N) {
+    const int lane = threadIdx.x & 31;
+    for (int k = 2; k <= N; k <<= 1)
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            for (int q = lane; q < (N >> 1); q += 32) {
+                const int t = ((q & ~(j - 1)) << 1) | (q & (j - 1));
+                const int p = t | j;
+                const int32_t x = keys[t], y = keys[p];
+                const bool up = (t & k) == 0;
+                if ((x > y) == up) {
+                    keys[t] = y;
+                    keys[p] = x;
+                    const double vx = vals[t];
+                    vals[t] = vals[p];
+                    vals[p] = vx;
+                }
+            }
+            __syncwarp();
+        }
+}
+
+template <int NT>
+__device__ __forceinline__ void block_bitonic(int32_t *keys, double *vals, int N) {
+    for (int k = 2; k <= N; k <<= 1)
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            for (int q = threadIdx.x; q < (N >> 1); q += NT) {
+                const int t = ((q & ~(j - 1)) << 1) | (q & (j - 1));
+                const int p = t | j;
+                const int32_t x = keys[t], y = keys[p];
+                const bool up = (t & k) == 0;
+                if ((x > y) == up) {
+                    keys[t] = y;
+                    keys[p] = x;
+                    const double vx = vals[t];
+                    vals[t] = vals[p];
+                    vals[p] = vx;
+                }
+            }
+            __syncthreads();
+        }
+}
+
+__device__ __forceinline__ int pow2_at_least(int64_t n, int lo) {
+    int v = lo;
+    while (v < n) v <<= 1;
+    return v;
+}
+
+// ------------------------------------------------------------------------------ S6 numeric, W
+
+template <int G>
+__global__ void __launch_bounds__(WARPS_W * 32) k_num_w(NumArgs a) {
+    extern __shared__ double smem_d[];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    double *vals = smem_d + wid * TW_NUM;
+    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + WARPS_W * TW_NUM) + wid * TW_NUM;
+    constexpr int MAXLG = 9;  // log2(TW_NUM)
+    const int64_t R = a.r1 - a.r0;
+    const int64_t off0 = a.crp[a.r0];
+    while (true) {
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(&a.ctl->row_ctr, (unsigned long long)ROW_BATCH);
+        base = __shfl_sync(FULLMASK, base, 0);
+        if ((int64_t)base >= R) break;
+        const int64_t end = min((int64_t)base + ROW_BATCH, R);
+        for (int64_t li = (int64_t)base; li < end; ++li) {
+            const int64_t i = a.r0 + li;
+            const int64_t o = a.crp[i];
+            const int64_t n = a.crp[i + 1] - o;
+            if (n == 0) continue;
+            if (n > CAPW_NUM) {
+                if (lane == 0) push_long(i, n, CAPB_NUM, a.listB, a.listG, a.ctl);
+                continue;
+            }
+            const int lg = table_log2(n, MAXLG);
+            const int T = 1 << lg;
+            for (int t = lane; t < T; t += 32) {
+                keys[t] = EMPTY;
+                vals[t] = 0.0;
+            }
+            __syncwarp();
+            const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
+            for (int64_t p0 = as; p0 < ae; p0 += 32 / G) {
+                const int64_t p = p0 + lane / G;
+                if (p < ae) {
+                    const int32_t k = __ldg(&a.A.col[p]);
+                    const double av = __ldg(&a.A.val[p]);
+                    const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
+                    for (int64_t q = bs + (lane % G); q < be; q += G)
+                        num_insert(keys, vals, __ldg(&a.B.col[q]), av * __ldg(&a.B.val[q]), lg);
+                }
+            }
+            __syncwarp();
+            // in-place compaction of the occupied slots (destination <= source, one round of 32
+            // slots is read completely before any of it is written)
+            int cnt = 0;
+            for (int t0 = 0; t0 < T; t0 += 32) {
+                const int32_t k = keys[t0 + lane];
+                const double v = vals[t0 + lane];
+                const bool occ = k != EMPTY;
+                const unsigned bal = __ballot_sync(FULLMASK, occ);
+                const int dst = cnt + __popc(bal & ((1u << lane) - 1u));
+                __syncwarp();
+                if (occ) {
+                    keys[dst] = k;
+                    vals[dst] = v;
+                }
+                cnt += __popc(bal);
+                __syncwarp();
+            }
+            if (cnt != n) {
+                if (lane == 0) atomicOr(&a.ctl->err, 1u);
+                continue;
+            }
+            const int N = pow2_at_least(n, 32);
+            for (int t = (int)n + lane; t < N; t += 32) keys[t] = INT_MAX;
+            __syncwarp();
+            warp_bitonic(keys, vals, N);
+            int32_t *oc = a.out_col + (o - off0);
+            double *ov = a.out_val + (o - off0);
+            for (int t = lane; t < n; t += 32) {
+                oc[t] = keys[t];
+                ov[t] = vals[t];
+            }
+            __syncwarp();
+        }
+    }
+}
+
+// ------------------------------------------------------------------------------ S6 numeric, B
+
+__global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
+    extern __shared__ double smem_d[];
+    double *vals = smem_d;
+    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);
+    __shared__ int64_t s_scan[40];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    constexpr int NW = THREADS_B / 32;
+    constexpr int MAXLG = 14;  // log2(TB_NUM)
+    const unsigned nrows = *(volatile unsigned *)&a.ctl->nB;
+    const int64_t off0 = a.crp[a.r0];
+    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
+        const int64_t i = a.listB[idx];
+        const int64_t o = a.crp[i];
+        const int64_t n = a.crp[i + 1] - o;
+        const int lg = table_log2(n, MAXLG);
+        const int T = 1 << lg;
+        for (int t = threadIdx.x; t < T; t += THREADS_B) {
+            keys[t] = EMPTY;
+            vals[t] = 0.0;
+        }
+        __syncthreads();
+        const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
+        for (int64_t p = as + wid; p < ae; p += NW) {
+            const int32_t k = __ldg(&a.A.col[p]);
+            const double av = __ldg(&a.A.val[p]);
+            const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
+            for (int64_t q = bs + lane; q < be; q += 32)
+                num_insert(keys, vals, __ldg(&a.B.col[q]), av * __ldg(&a.B.val[q]), lg);
+        }
+        __syncthreads();
+        int64_t cnt = 0;
+        for (int t0 = 0; t0 < T; t0 += THREADS_B) {
+            const int t = t0 + threadIdx.x;
+            const int32_t k = t < T ? keys[t] : EMPTY;
+            const double v = t < T ? vals[t] : 0.0;
+            const int occ = k != EMPTY;
+            int64_t tot;
+            const int64_t ex = block_excl_scan<THREADS_B>(occ, s_scan, &tot);  // ends with a barrier
+            if (occ) {
+                keys[cnt + ex] = k;
+                vals[cnt + ex] = v;
+            }
+            cnt += tot;
+            __syncthreads();
+        }
+        if (cnt != n) {
+            if (threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
+            __syncthreads();
+            continue;
+        }
+        const int N = pow2_at_least(n, 32);
+        for (int t = (int)n + threadIdx.x; t < N; t += THREADS_B) keys[t] = INT_MAX;
+        __syncthreads();
+        block_bitonic<THREADS_B>(keys, vals, N);
+        int32_t *oc = a.out_col + (o - off0);
+        double *ov = a.out_val + (o - off0);
+        for (int t = threadIdx.x; t < n; t += THREADS_B) {
+            oc[t] = keys[t];
+            ov[t] = vals[t];
+        }
+        __syncthreads();
+    }
+}
+
+// ------------------------------------------------------------------------------ S6 numeric, G
+// Dense accumulation over all columns (§II-B): bitmap for structure (values may cancel to
+// 0.0 and must still be stored), fp64 array for values, in this CTA's arena slot.  Output is
+// produced in column order by sweeping the bitmap, which also restores the slot to zero.
+
+__global__ void __launch_bounds__(THREADS_G) k_num_g(NumArgs a) {
+    __shared__ int64_t s_scan[40];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    constexpr int NW = THREADS_G / 32;
+    uint32_t *bm = a.gbits + (int64_t)blockIdx.x * a.gstride_bits;
+    double *dv = a.gvals + (int64_t)blockIdx.x * a.gstride_vals;
+    const unsigned nrows = *(volatile unsigned *)&a.ctl->nG;
+    const int64_t nwords = (a.B.ncols + 31) / 32;
+    const int64_t off0 = a.crp[a.r0];
+    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
+        const int64_t i = a.listG[idx];
+        const int64_t o = a.crp[i];
+        const int64_t n = a.crp[i + 1] - o;
+        const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
+        for (int64_t p = as + wid; p < ae; p += NW) {
+            const int32_t k = __ldg(&a.A.col[p]);
+            const double av = __ldg(&a.A.val[p]);
+            const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
+            for (int64_t q = bs + lane; q < be; q += 32) {
+                const int32_t c = __ldg(&a.B.col[q]);
+                atomicOr(&bm[c >> 5], 1u << (c & 31));
+                atomicAdd(&dv[c], av * __ldg(&a.B.val[q]));
+            }
+        }
+        __syncthreads();
+        int32_t *oc = a.out_col + (o - off0);
+        double *ov = a.out_val + (o - off0);
+        int64_t cnt = 0;
+        for (int64_t w0 = 0; w0 < nwords; w0 += THREADS_G) {
+            const int64_t w = w0 + threadIdx.x;
+            uint32_t word = w < nwords ? __ldcg(&bm[w]) : 0u;
+            int64_t tot;
+            const int64_t ex = block_excl_scan<THREADS_G>(__popc(word), s_scan, &tot);
+            if (word) {
+                int64_t pos = cnt + ex;
+                bm[w] = 0u;
+                while (word) {
+                    const int b = __ffs(word) - 1;
+                    word &= word - 1;
+                    const int64_t c = w * 32 + b;
+                    if (pos < n) {
+                        oc[pos] = (int32_t)c;
+                        ov[pos] = __ldcg(&dv[c]);
+                    }
+                    dv[c] = 0.0;
+                    ++pos;
+                }
+            }
+            cnt += tot;
+        }
+        if (cnt != n && threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
+        __syncthreads();
+    }
+}
+
+// ------------------------------------------------------------------------------------ launchers
+
+size_t symw_smem() { return size_t(WARPS_W) * TW_SYM * sizeof(int32_t); }
+size_t numw_smem() { return size_t(WARPS_W) * TW_NUM * (sizeof(int32_t) + sizeof(double)); }
+size_t symb_smem() { return size_t(TB_SYM) * sizeof(int32_t); }
+size_t numb_smem() { return size_t(TB_NUM) * (sizeof(int32_t) + sizeof(double)); }
+
+template <int G>
+static void set_attrs_w() {
+    cudaFuncSetAttribute(k_sym_w<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symw_smem());
+    cudaFuncSetAttribute(k_num_w<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem());
+}
+
+const Grids &grids(int device, int num_sms) {
+    static Grids cache[64];
+    static bool init[64] = {false};
+    if (device < 0 || device >= 64) device = 0;
+    if (!init[device]) {
+        set_attrs_w<4>();
+        set_attrs_w<8>();
+        set_attrs_w<16>();
+        set_attrs_w<32>();
+        cudaFuncSetAttribute(k_sym_b, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symb_smem());
+        cudaFuncSetAttribute(k_num_b, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numb_smem());
+        Grids g;
+        int occ = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_count, 256, 0);
+        g.count_blocks = num_sms * (occ > 0 ? occ : 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_w<8>, WARPS_W * 32, symw_smem());
+        g.symw_blocks = num_sms * (occ > 0 ? occ : 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<8>, WARPS_W * 32, numw_smem());
+        g.numw_blocks = num_sms * (occ > 0 ? occ : 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b, THREADS_B, symb_smem());
+        g.symb_blocks = num_sms * (occ > 0 ? occ : 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_b, THREADS_B, numb_smem());
+        g.numb_blocks = num_sms * (occ > 0 ? occ : 1);
+        cache[device] = g;
+        init[device] = true;
+    }
+    return cache[device];
+}
+
+static int grid_for(int64_t n, int threads, int cap) {
+    int64_t b = (n + threads - 1) / threads;
+    if (b < 1) b = 1;
+    return (int)(b < cap ? b : cap);
+}
+
+void launch_count(const DevCSR &A, const DevCSR &B, int64_t *u, Ctl *ctl, cudaStream_t s) {
+    if (A.nrows == 0) return;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int blocks = grid_for(A.nrows, 8, grids(dev, sms).count_blocks);
+    k_count<<<blocks, 256, 0, s>>>(A, B, u, ctl);
+    LAUNCHED(1);
+}
+
+void launch_validate(const DevCSR &M, Ctl *ctl, cudaStream_t s) {
+    if (M.nrows == 0) return;
+    k_validate<<<grid_for(M.nrows, 8, 148 * 16), 256, 0, s>>>(M, ctl);
+    LAUNCHED(1);
+}
+
+void launch_rebase(int64_t *rp, int64_t n, int64_t sub, cudaStream_t s) {
+    if (n == 0 || sub == 0) return;
+    k_rebase<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(rp, n, sub);
+    LAUNCHED(1);
+}
+
+void launch_add(int64_t *crp, int64_t n, int64_t delta, cudaStream_t s) {
+    if (delta == 0) return;
+    k_add<<<grid_for(n + 1, 256, 148 * 8), 256, 0, s>>>(crp, n + 1, delta);
+    LAUNCHED(1);
+}
+
+template <int G>
+static void sym_w(const SymArgs &a, int blocks, cudaStream_t s) {
+    k_sym_w<G><<<blocks, WARPS_W * 32, symw_smem(), s>>>(a);
+    LAUNCHED(1);
+}
+template <int G>
+static void num_w(const NumArgs &a, int blocks, cudaStream_t s) {
+    k_num_w<G><<<blocks, WARPS_W * 32, numw_smem(), s>>>(a);
+    LAUNCHED(1);
+}
+
+static int group_for(const DevCSR &B, int64_t nnzB) {
+    const double avg = B.nrows > 0 ? double(nnzB) / double(B.nrows) : 0.0;
+    if (avg <= 5.0) return 4;
+    if (avg <= 10.0) return 8;
+    if (avg <= 20.0) return 16;
+    return 32;
+}
+
+static inline void rec(cudaEvent_t *ev, int k, cudaStream_t s) {
+    if (ev) cudaEventRecord(ev[k], s);
+}
+
+void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev) {
+    if (a.A.nrows == 0) return;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const Grids &g = grids(dev, num_sms);
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, 16, s);  // row_ctr, nB, nG
+    const int64_t rows = a.A.nrows;
+    const int wblocks = grid_for(rows, WARPS_W * ROW_BATCH, g.symw_blocks);
+    rec(ev, 0, s);
+    switch (a.group) {
+        case 4: sym_w<4>(a, wblocks, s); break;
+        case 8: sym_w<8>(a, wblocks, s); break;
+        case 16: sym_w<16>(a, wblocks, s); break;
+        default: sym_w<32>(a, wblocks, s); break;
+    }
+    rec(ev, 1, s);
+    k_sym_b<<<g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
+    LAUNCHED(1);
+    rec(ev, 2, s);
+    if (a.gblocks > 0) {
+        k_sym_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
+        LAUNCHED(1);
+    }
+    rec(ev, 3, s);
+}
+
+void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev) {
+    const int64_t rows = a.r1 - a.r0;
+    if (rows <= 0) return;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    const Grids &g = grids(dev, num_sms);
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, 16, s);
+    const int wblocks = grid_for(rows, WARPS_W * ROW_BATCH, g.numw_blocks);
+    rec(ev, 0, s);
+    switch (a.group) {
+        case 4: num_w<4>(a, wblocks, s); break;
+        case 8: num_w<8>(a, wblocks, s); break;
+        case 16: num_w<16>(a, wblocks, s); break;
+        default: num_w<32>(a, wblocks, s); break;
+    }
+    rec(ev, 1, s);
+    k_num_b<<<g.numb_blocks, THREADS_B, numb_smem(), s>>>(a);
+    LAUNCHED(1);
+    rec(ev, 2, s);
+    if (a.gblocks > 0) {
+        k_num_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
+        LAUNCHED(1);
+    }
+    rec(ev, 3, s);
+}
+
+void launch_scan(int64_t *crp, int64_t n, int64_t base, int64_t *tmp, cudaStream_t s) {
+    const int64_t n1 = n + 1;
+    const int64_t nb = (n1 + SCAN_TILE - 1) / SCAN_TILE;
+    k_scan_reduce<<<(unsigned)nb, 1024, 0, s>>>(crp, n1, tmp);
+    LAUNCHED(1);
+    k_scan_top<<<1, 1024, 0, s>>>(tmp, nb, base);
+    LAUNCHED(1);
+    k_scan_apply<<<(unsigned)nb, 1024, 0, s>>>(crp, n1, tmp);
+    LAUNCHED(1);
+}
+
+void launch_cut(const int64_t *crp, int64_t n, int64_t cap_prime, int64_t *bounds, int64_t nids, cudaStream_t s) {
+    k_fill<<<grid_for(nids + 1, 256, 148 * 4), 256, 0, s>>>(bounds, nids + 1, n);
+    LAUNCHED(1);
+    if (n > 0) {
+        k_cut<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(crp, n, cap_prime, bounds, nids);
+        LAUNCHED(1);
+    }
+}
+
+int choose_group(const DevCSR &B, int64_t nnzB) { return group_for(B, nnzB); }
+
+__global__ void k_gather(const int64_t *__restrict__ crp, const int64_t *__restrict__ idx, int64_t n,
+                         int64_t *__restrict__ out) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = crp[idx[i]];
+}
+
+void launch_gather(const int64_t *crp, const int64_t *idx, int64_t n, int64_t *out, cudaStream_t s) {
+    if (n > 0) {
+        k_gather<<<grid_for(n, 256, 148 * 4), 256, 0, s>>>(crp, idx, n, out);
+        LAUNCHED(1);
+    }
+}
+
+}  // namespace spg

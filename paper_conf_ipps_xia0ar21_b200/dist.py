@@ -1,0 +1,64 @@
+"""Multi-GPU row-panel deal (one process per GPU, torch.distributed over NCCL / NVLink).
+
+Rows of C are independent (§III-A: "final values within a chunk of the output
+matrix C are independent"), so A is dealt across ranks as contiguous row panels (§III-A,
+§III-D) and every rank needs all of B.  The only exchanges on the path are
+  * B (and A when A is B) reaching every GPU: a broadcast from the rank that staged it
+    (`broadcast_csr`, NCCL over NVLink/NVSwitch on a B200 box, gloo in the CPU tests);
+  * the 8-byte nnz of every rank's slice (`slice_bases`, an all_gather) so that each rank writes
+    its C rows with GLOBAL row_ptr values into its part of one logical host CSR.
+After that every rank drains its own C chunks over its own host link; nothing else crosses GPUs.
+"""
+from __future__ import annotations
+
+from typing import List, Sequence, Tuple
+
+import numpy as np
+
+
+def row_panels(row_ptr: np.ndarray, world: int, weights: np.ndarray | None = None) -> List[Tuple[int, int]]:
+    """Contiguous row ranges [r0, r1) per rank, balanced by `weights` per row (default: nnz of A's
+    rows, which is what row_ptr gives for free).  Every rank gets a range (possibly empty)."""
+    n = len(row_ptr) - 1
+    if weights is None:
+        cum = np.asarray(row_ptr, dtype=np.int64) - int(row_ptr[0])
+    else:
+        cum = np.zeros(n + 1, dtype=np.int64)
+        np.cumsum(np.asarray(weights, dtype=np.int64), out=cum[1:])
+    total = int(cum[-1])
+    cuts = [0]
+    for r in range(1, world):
+        target = (total * r + world - 1) // world if total else 0
+        c = int(np.searchsorted(cum, target, side="left")) if total else (n * r) // world
+        cuts.append(min(max(c, cuts[-1]), n))
+    cuts.append(n)
+    return [(cuts[r], cuts[r + 1]) for r in range(world)]
+
+
+def slice_bases(local_nnz: int, group=None, device=None) -> Tuple[int, int]:
+    """All-gather every rank's nnz; returns (global row_ptr base of this rank, total nnz)."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    t = torch.tensor([int(local_nnz)], dtype=torch.int64, device=device)
+    out = [torch.zeros(1, dtype=torch.int64, device=device) for _ in range(world)]
+    dist.all_gather(out, t, group=group)
+    vals = [int(x.item()) for x in out]
+    return sum(vals[:rank]), sum(vals)
+
+
+def broadcast_csr(arrays: Sequence, src: int = 0, group=None) -> None:
+    """In-place broadcast of the CSR arrays (row_ptr, col, val tensors, already allocated with the
+    right shapes on every rank) from `src` -- NCCL over NVLink on GPUs."""
+    import torch.distributed as dist
+    for a in arrays:
+        dist.broadcast(a, src=src, group=group)
+
+
+def gather_rows_global(parts: Sequence[Tuple[np.ndarray, np.ndarray, np.ndarray]]):
+    """Stitch per-rank slices (row_ptr with global values, col, val) into one CSR (tests)."""
+    rp = [parts[0][0][:1]]
+    for p in parts:
+        rp.append(p[0][1:])
+    return (np.concatenate(rp), np.concatenate([p[1] for p in parts]), np.concatenate([p[2] for p in parts]))

@@ -1,0 +1,301 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element.
+
+Bar: row_ptr and col_idx bit-identical; every value within
+|c - ref| <= 1e-12 * sum_k |a_ik b_kj| (BASELINE.json north_star), exact (bit-equal) on
+the integer-valued stencil configs.  All inputs come from `workloads` (seeded).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+from tests import closed_forms as CF
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_ipps_xia0ar21_b200 as spg  # noqa: E402
+from paper_conf_ipps_xia0ar21_b200 import capi  # noqa: E402
+
+
+def run(A, B, budget=0, **kw):
+    """plan + execute_into pinned torch buffers; returns (rp, col, val, info, chunks)."""
+    o = capi.opts(**kw)
+    with capi.Plan(A, B, budget, o) as P:
+        info = P.info()
+        rp = torch.empty(info["nrows"] + 1, dtype=torch.int64, pin_memory=True)
+        col = torch.empty(info["nnz"], dtype=torch.int32, pin_memory=True)
+        val = torch.empty(info["nnz"], dtype=torch.float64, pin_memory=True)
+        P.execute_into(rp, col, val)
+        chunks = P.chunks()
+    return rp.numpy(), col.numpy(), val.numpy(), info, chunks
+
+
+def assert_parity(A, B, rp, col, val, rows=None, exact=False, base=0):
+    E = oracle.spgemm(A, B, rows=rows)
+    if rows is None:
+        res = oracle.compare(rp, col, val, E, rows_offset=base)
+    else:
+        # gather the selected rows out of the full GPU result
+        rs = np.asarray(rows)
+        n = rp[rs + 1] - rp[rs]
+        gp = np.zeros(len(rs) + 1, dtype=np.int64)
+        np.cumsum(n, out=gp[1:])
+        idx = np.concatenate([np.arange(rp[r] - base, rp[r + 1] - base) for r in rs]) if len(rs) else np.zeros(0, int)
+        res = oracle.compare(gp, col[idx], val[idx], E)
+    assert res["ok"], res
+    if exact:
+        assert np.array_equal(val if rows is None else val[idx], E["val"])
+    return res
+
+
+# ------------------------------------------------------------------------------------- paper pins
+
+def test_fig2_example():
+    A, B = W.fig2_instance()
+    rp, col, val, info, _ = run(A, B)
+    assert list(rp) == [0, 2] and list(col) == [0, 3] and list(val) == [43.0, 14.0]
+    assert info["products"] == 3
+
+
+def test_c1_full_bit_exact():
+    """BASELINE config 0 in full, in-core: values are small integers -> bit-exact in any order."""
+    A = W.stencil_2d5(64)
+    rp, col, val, info, _ = run(A, A)
+    assert info["products"] == 100104 and info["nnz"] == 51972
+    assert_parity(A, A, rp, col, val, exact=True)
+    i = np.repeat(np.arange(A.nrows), np.diff(rp))
+    assert np.array_equal(val, CF.c1_entry(64, i, col.astype(np.int64)))
+    assert val.sum() == 264.0
+
+
+@pytest.mark.parametrize("n", [8, 24, 40])
+def test_c2_small_bit_exact(n):
+    A = W.stencil_3d27(n)
+    rp, col, val, info, _ = run(A, A)
+    p, z = CF.c2_totals(n)
+    assert info["products"] == p and info["nnz"] == z
+    assert_parity(A, A, rp, col, val, exact=True)
+    assert val.sum() == CF.c2_sum(n)
+
+
+# ------------------------------------------------------------------------------------- random
+
+@pytest.mark.parametrize("seed", range(8))
+def test_random_rectangular(seed):
+    rng = np.random.default_rng(seed)
+    m, k, n = (int(x) for x in rng.integers(1, 3000, size=3))
+    A = W.random_csr_sparse(m, k, float(rng.uniform(0.5, 12)), seed=seed)
+    B = W.random_csr_sparse(k, n, float(rng.uniform(0.5, 12)), seed=seed + 1000)
+    rp, col, val, info, _ = run(A, B, validate=True)
+    assert_parity(A, B, rp, col, val)
+
+
+@pytest.mark.parametrize("shape", [(0, 5, 7), (5, 0, 7), (6, 5, 0), (1, 1, 1), (3, 4, 5)])
+def test_degenerate(shape):
+    m, k, n = shape
+    A = W.random_csr(m, k, 0.6, seed=1, empty_rows=0.3)
+    B = W.random_csr(k, n, 0.6, seed=2, empty_rows=0.3)
+    rp, col, val, info, _ = run(A, B)
+    assert_parity(A, B, rp, col, val)
+
+
+def test_empty_b_rows_and_explicit_zeros():
+    A = W.random_csr_sparse(500, 400, 6.0, seed=3)
+    B = W.random_csr_sparse(400, 450, 6.0, seed=4)
+    # blank every third row of B, zero some values (structure must stay)
+    keep = np.ones(B.nnz, bool)
+    for r in range(0, B.nrows, 3):
+        keep[B.row_ptr[r]:B.row_ptr[r + 1]] = False
+    cnt = np.add.reduceat(keep.astype(np.int64), B.row_ptr[:-1]) * (np.diff(B.row_ptr) > 0)
+    rp = np.zeros(B.nrows + 1, np.int64)
+    np.cumsum(cnt, out=rp[1:])
+    B = W.CSR(B.nrows, B.ncols, rp, B.col[keep], B.val[keep].copy())
+    B.val[::5] = 0.0
+    A.val[::7] = 0.0
+    r, c, v, info, _ = run(A, B)
+    assert_parity(A, B, r, c, v)
+
+
+# ------------------------------------------------------------------------------------- tiers
+
+def _long_rows_case(seed=0, wide=60000, deg=240):
+    """A few rows whose products/nnz exceed the warp and CTA tiers (forces tiers B and G)."""
+    rng = np.random.default_rng(seed)
+    k = 800
+    B = W.random_csr_sparse(k, wide, deg, seed=seed + 1)
+    rows = []
+    for i in range(300):
+        if i % 100 == 0:
+            d = 300            # ~300 * 240 = 72k products over 60k columns -> G tier
+        elif i % 10 == 0:
+            d = 12             # ~2.9k products -> B tier
+        else:
+            d = int(rng.integers(0, 3))
+        rows.append(np.sort(rng.choice(k, size=d, replace=False)))
+    rp = np.zeros(301, np.int64)
+    np.cumsum([len(r) for r in rows], out=rp[1:])
+    col = np.concatenate(rows).astype(np.int32)
+    A = W.CSR(300, k, rp, col, rng.uniform(-1, 1, len(col)))
+    return A, B
+
+
+def test_tiers_warp_block_global():
+    A, B = _long_rows_case()
+    rp, col, val, info, _ = run(A, B)
+    assert info["rows_block"] > 0 and info["rows_global"] > 0 and info["rows_warp"] > 0, info
+    assert_parity(A, B, rp, col, val)
+
+
+def test_rmat_skewed():
+    A = W.rmat(14, 16, seed=5)
+    rp, col, val, info, _ = run(A, A)
+    assert_parity(A, A, rp, col, val)
+    assert info["products"] == int(oracle.products(A, A).sum())
+
+
+# ------------------------------------------------------------------------------------- out-of-core
+
+def test_forced_chunking_invariance():
+    """Chunked == unchunked, ring 1 (synchronous) == ring 2/3 (S8-S10 must not change the result)."""
+    A = W.stencil_3d27(20)
+    ref = run(A, A)
+    for kw in ({"chunk_nnz": 5000}, {"chunk_nnz": 5000, "ring": 1}, {"chunk_nnz": 777, "ring": 3},
+               {"min_chunks": 17}):
+        rp, col, val, info, chunks = run(A, A, **kw)
+        assert info["num_chunks"] > 2
+        assert np.array_equal(rp, ref[0]) and np.array_equal(col, ref[1]) and np.array_equal(val, ref[2])
+        rows, offs = chunks
+        assert rows[0] == 0 and rows[-1] == A.nrows and np.all(np.diff(offs) <= info["chunk_capacity"])
+
+
+def test_budget_forces_chunks_and_fits():
+    A = W.stencil_3d27(32)
+    nnzC = CF.c2_totals(32)[1]
+    budget = 24 << 20   # 24 MiB: A (~9 MB) + row arrays + ring << 12 * nnz(C) (~25 MB)
+    rp, col, val, info, _ = run(A, A, budget=budget)
+    assert info["nnz"] == nnzC and info["num_chunks"] >= 2 and info["arena_used"] <= budget
+    assert_parity(A, A, rp, col, val, exact=True)
+
+
+def test_one_row_per_chunk():
+    A = W.random_csr_sparse(60, 50, 4.0, seed=9)
+    B = W.random_csr_sparse(50, 70, 4.0, seed=10)
+    rp, col, val, info, chunks = run(A, B, chunk_nnz=1)
+    assert info["num_chunks"] >= 40
+    assert_parity(A, B, rp, col, val)
+
+
+def test_execute_stream_sink_matches():
+    A = W.rmat(12, 16, seed=2)
+    ref = run(A, A)
+    got_rp, got_col, got_val = [0], [], []
+    with capi.Plan(A, A, 0, capi.opts(chunk_nnz=20000, ring=2)) as P:
+        seen = []
+
+        def sink(r0, r1, rp, col, val):
+            seen.append((r0, r1))
+            got_rp.extend((rp[1:] + got_rp[-1]).tolist())
+            got_col.append(col.copy())
+            got_val.append(val.copy())
+
+        P.execute_stream(sink)
+        assert len(seen) == P.info()["num_chunks"] and seen[0][0] == 0 and seen[-1][1] == A.nrows
+    assert np.array_equal(np.array(got_rp), ref[0])
+    assert np.array_equal(np.concatenate(got_col), ref[1])
+    # values: fp64 atomics make the summation order (not the bound) run-dependent (R10)
+    assert_parity(A, A, np.array(got_rp), np.concatenate(got_col), np.concatenate(got_val))
+
+
+def test_repeat_execute_same_plan():
+    A = W.stencil_3d27(16)
+    with capi.Plan(A, A, 0, capi.opts(chunk_nnz=3000)) as P:
+        a = P.execute()
+        a = [x.copy() for x in a]
+        b = P.execute()
+        for x, y in zip(a, b):
+            assert np.array_equal(x, y)
+
+
+# ------------------------------------------------------------------------------------- device inputs
+
+def _to_dev(M, base=0):
+    class D:
+        pass
+    d = D()
+    d.nrows, d.ncols = M.nrows, M.ncols
+    pad = np.zeros(base, np.int32)
+    d.row_ptr = torch.from_numpy(M.row_ptr + base).cuda()
+    d.col = torch.from_numpy(np.concatenate([pad, M.col])).cuda()
+    d.val = torch.from_numpy(np.concatenate([pad.astype(np.float64), M.val])).cuda()
+    return d
+
+
+def test_device_inputs_with_base_and_row_panels():
+    """Device-resident operands (e.g. B after an NCCL broadcast), arbitrary row_ptr base, and a
+    row panel [row_begin, row_end) with a global row_ptr base: the union of panels == whole."""
+    A = W.rmat(12, 8, seed=7)
+    B = W.random_csr_sparse(A.ncols, 3000, 5.0, seed=8)
+    full = run(A, B)
+    dA, dB = _to_dev(A, base=13), _to_dev(B, base=5)
+    rp, col, val, _, _ = run(dA, dB, stream=torch.cuda.current_stream().cuda_stream)
+    assert np.array_equal(rp, full[0]) and np.array_equal(col, full[1])
+    assert np.array_equal(val, full[2]) or oracle.compare(rp, col, val, oracle.spgemm(A, B))["ok"]
+    cuts = [0, 700, 701, 2500, A.nrows]
+    parts = []
+    for r0, r1 in zip(cuts[:-1], cuts[1:]):
+        base = int(full[0][r0])
+        prp, pcol, pval, info, _ = run(dA, dB, row_begin=r0, row_end=r1, row_ptr_base=base)
+        assert prp[0] == base and np.array_equal(prp, full[0][r0:r1 + 1])
+        parts.append((pcol, pval))
+    assert np.array_equal(np.concatenate([p[0] for p in parts]), full[1])
+
+
+def test_workspace_from_torch():
+    A = W.stencil_3d27(12)
+    ws = torch.empty(64 << 20, dtype=torch.uint8, device="cuda")
+    rp, col, val, info, _ = run(A, A, budget=ws.numel(), workspace=ws)
+    assert info["arena_bytes"] == ws.numel()
+    assert_parity(A, A, rp, col, val, exact=True)
+
+
+# ------------------------------------------------------------------------------------- errors
+
+def test_errors():
+    A = W.random_csr(4, 5, 0.5, seed=1)
+    B = W.random_csr(6, 3, 0.5, seed=2)
+    with pytest.raises(capi.SpgemmError) as e:
+        capi.Plan(A, B)
+    assert e.value.status == capi.ERR_SHAPE
+    C = W.stencil_3d27(16)
+    with pytest.raises(capi.SpgemmError) as e:
+        capi.Plan(C, C, 1 << 16)
+    assert e.value.status == capi.ERR_BUDGET
+    bad = W.random_csr(5, 5, 0.8, seed=3)
+    bad.col = bad.col[::-1].copy()
+    with pytest.raises(capi.SpgemmError) as e:
+        capi.Plan(bad, W.identity(5), 0, capi.opts(validate=True))
+    assert e.value.status == capi.ERR_INVALID_ARGUMENT
+    with pytest.raises(capi.SpgemmError) as e:
+        capi.Plan(A, W.random_csr(5, 3, 0.5, 2), 0, capi.opts(row_begin=3, row_end=9))
+    assert e.value.status == capi.ERR_SHAPE
+    # capacity error of the one-shot API
+    AA = W.stencil_2d5(8)
+    out = [torch.empty(65, dtype=torch.int64), torch.empty(10, dtype=torch.int32), torch.empty(10, dtype=torch.float64)]
+    with pytest.raises(capi.SpgemmError) as e:
+        capi.spgemm_multiply(AA, AA, 0, None, *out, capacity=10)
+    assert e.value.status == capi.ERR_CAPACITY
+
+
+def test_multiply_one_shot():
+    A = W.stencil_2d5(16)
+    z = int(oracle.row_nnz(A, A).sum())
+    rp = torch.empty(A.nrows + 1, dtype=torch.int64, pin_memory=True)
+    col = torch.empty(z, dtype=torch.int32, pin_memory=True)
+    val = torch.empty(z, dtype=torch.float64, pin_memory=True)
+    n = capi.spgemm_multiply(A, A, 0, None, rp, col, val, capacity=z)
+    assert n == z
+    assert_parity(A, A, rp.numpy(), col.numpy(), val.numpy(), exact=True)
