@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--ring", type=int, default=2)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--two-phase", action="store_true", help="time the two-phase plan/execute path at N = 1")
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     return ap.parse_args()
 
@@ -234,9 +235,14 @@ def main():
     wbytes = ws.numel()
     stream = torch.cuda.current_stream()
 
+    # N = 1: the fused plan (per-chunk symbolic overlapped with the previous chunk's D2H, the call
+    # spgemm_multiply makes).  N > 1: two-phase plans, because every rank needs its global row_ptr
+    # base (an all_gather of the ranks' nnz) before it writes row offsets.
+    fused = world == 1 and not args.two_phase
+
     def mk_opts(profile=False, base=0):
         return capi.opts(device=local, ring=args.ring, profile=profile, row_begin=r0, row_end=r1, workspace=ws,
-                         stream=stream.cuda_stream, row_ptr_base=base)
+                         stream=stream.cuda_stream, row_ptr_base=base, fused=fused)
 
     ws_e2e = None
 
@@ -246,12 +252,12 @@ def main():
         if ws_e2e is None:
             ws_e2e = torch.empty(wbytes + in_bytes, dtype=torch.uint8, device=dev)
         return capi.opts(device=local, ring=args.ring, row_begin=r0, row_end=r1, workspace=ws_e2e,
-                         stream=stream.cuda_stream)
+                         stream=stream.cuda_stream, fused=fused)
 
     # untimed: sizes, global base, pinned outputs (pinning is a one-time cost, reported separately)
-    with capi.Plan(dA, dB, wbytes, mk_opts()) as P:
+    with capi.Plan(dA, dB, wbytes, capi.opts(device=local, ring=args.ring, row_begin=r0, row_end=r1, workspace=ws,
+                                             stream=stream.cuda_stream)) as P:
         info = P.info()
-        rows_c, offs_c = P.chunks()
     nnz_local = info["nnz"]
     base = 0
     if world > 1:
@@ -264,13 +270,21 @@ def main():
     h_val = torch.empty(nnz_local, dtype=torch.float64, pin_memory=True)
     pin_s = time.perf_counter() - t0
 
+    chunk_table = {}
+
     def step(profile=False):
         P = capi.Plan(dA, dB, wbytes, mk_opts(profile))
-        if world > 1:
-            b, _ = pdist.slice_bases(P.info()["nnz"], device=dev)
-            P.set_row_ptr_base(b)
-        P.execute_into(h_rp, h_col, h_val)
+        if fused:
+            P.execute_capacity(h_rp, h_col, h_val, nnz_local)
+        else:
+            if world > 1:
+                b, _ = pdist.slice_bases(P.info()["nnz"], device=dev)
+                P.set_row_ptr_base(b)
+            P.execute_into(h_rp, h_col, h_val)
         st = P.stats() if profile else None
+        if profile and "rows" not in chunk_table:
+            chunk_table["rows"], chunk_table["offs"] = P.chunks()
+            chunk_table["info"] = P.info()
         P.free()
         return st
 
@@ -344,7 +358,7 @@ def main():
     roof = None
     if dom is not None:
         if dom.startswith("num"):
-            per_launch = compulsory_bytes(A, B, rows_c, offs_c, r0)
+            per_launch = compulsory_bytes(A, B, chunk_table["rows"], chunk_table["offs"], r0)
             byts = float(np.sum(per_launch)) * args.steps
         elif dom.startswith("sym"):
             # symbolic: A panel + u + crp + touched B rows (col only) + crp writes
@@ -383,6 +397,10 @@ def main():
         def e2e_step():
             if world == 1:
                 P = capi.Plan(hA, hB, wbytes + in_bytes, mk_opts_e2e())
+                if fused:
+                    P.execute_capacity(h_rp, h_col, h_val, nnz_local)
+                    P.free()
+                    return
             else:
                 # rank 0 stages B from pinned host memory; NCCL broadcast over NVLink to every rank
                 if rank == 0:
@@ -436,7 +454,8 @@ def main():
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": name, "budget_bytes": budget, "m": A.nrows, "nnz_A": A.nnz,
                        "products": products_total, "nnz_C": nnz_total, "C_host_bytes": d2h_bytes,
-                       "chunks": info["num_chunks"], "ring": args.ring,
+                       "chunks": chunk_table["info"]["num_chunks"], "ring": args.ring,
+                       "plan": "fused (per-chunk symbolic overlapped with D2H)" if fused else "two-phase",
                        "l2": "inputs (686 MB) and output (3.07 GB) larger than L2; no flush needed",
                        "parallelism": f"row panels x{world}"},
             "gpu_launches": int(launches),

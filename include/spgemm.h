@@ -90,6 +90,12 @@ typedef struct {
                            /*   chunks are sized from the ring buffers left in the budget           */
     int64_t row_ptr_base;  /* added to every C row_ptr value delivered to the host (rank slices)    */
     int64_t min_chunks;    /* split C into at least this many chunks for D2H overlap; 0 = auto      */
+    int32_t fused;         /* 0 = two-phase plan: the symbolic pass of ALL rows runs in spgemm_plan, */
+                           /*   nnz(C) is known before execute (reuse, caller-sized outputs);       */
+                           /* 1 = fused: spgemm_plan only counts products and cuts chunks from the  */
+                           /*   row bounds min(products, ncols); each chunk's symbolic pass + scan  */
+                           /*   run inside execute, overlapped with the previous chunk's D2H        */
+    int32_t reserved;
 } spgemm_opts;
 
 typedef struct spgemm_plan_s *spgemm_plan_t;
@@ -115,6 +121,8 @@ typedef struct {
     int64_t chunk_capacity;     /* nonzeros per ring buffer                                       */
     int64_t arena_bytes, arena_used, ring_bytes;
     int64_t rows_warp, rows_block, rows_global; /* rows per accumulator tier in the symbolic pass   */
+    int32_t fused;              /* 1 if the plan is fused (nnz, max_row_nnz = -1 until executed)    */
+    int32_t reserved;
 } spgemm_info;
 
 spgemm_status spgemm_plan_info(spgemm_plan_t plan, spgemm_info *info);
@@ -127,10 +135,19 @@ spgemm_status spgemm_plan_chunks(spgemm_plan_t plan, int64_t *rows, int64_t *off
  * chunk D2H-copied into host memory while the next is computed.  Synchronises before return.
  * spgemm_execute_into writes into caller memory: row_ptr [nrows+1] (may be NULL), col_idx and
  * values [nnz]; page-locked memory (cudaHostAlloc / torch pin_memory) gives asynchronous copies,
- * pageable memory is correct but slow.  Repeatable on the same plan. */
+ * pageable memory is correct but slow.  Repeatable on the same plan.  On a fused plan it needs
+ * nnz(C) to be known (an earlier execution), else SPGEMM_ERR_STATE. */
 spgemm_status spgemm_execute_into(spgemm_plan_t plan, int64_t *row_ptr, int32_t *col_idx, double *values);
 
-/* Same, into plan-owned pinned host memory allocated on the first call (kept until free). */
+/* Execute into caller memory with room for `capacity` nonzeros (any plan; the way to run a fused
+ * plan whose nnz is not known yet).  *nnz_out receives nnz(C).  If nnz(C) > capacity nothing past
+ * the capacity is written, the numeric work stops, the symbolic passes finish to report nnz(C),
+ * and SPGEMM_ERR_CAPACITY is returned (the plan stays usable). */
+spgemm_status spgemm_execute_capacity(spgemm_plan_t plan, int64_t *row_ptr, int32_t *col_idx, double *values,
+                                      int64_t capacity, int64_t *nnz_out);
+
+/* Same as spgemm_execute_into, into plan-owned pinned host memory allocated on the first call
+ * (kept until free). */
 spgemm_status spgemm_execute(spgemm_plan_t plan, spgemm_csr_out *C_out);
 
 /* Sink mode for C larger than host memory: every chunk is copied into a pinned staging ring and
@@ -146,7 +163,9 @@ spgemm_status spgemm_execute_stream(spgemm_plan_t plan, spgemm_chunk_cb cb, void
 spgemm_status spgemm_set_row_ptr_base(spgemm_plan_t plan, int64_t base);
 
 /* One-shot C = A x B on device-resident or host inputs into caller host buffers with capacity
- * nnz_capacity; plan + execute in one call.  *nnz_out receives nnz(C) (also on CAPACITY error). */
+ * nnz_capacity: a fused plan (opts->fused is forced to 1) + spgemm_execute_capacity + free, so the
+ * per-chunk symbolic passes overlap the D2H of earlier chunks.  *nnz_out receives nnz(C) (also on
+ * SPGEMM_ERR_CAPACITY). */
 spgemm_status spgemm_multiply(const spgemm_csr *A, const spgemm_csr *B, size_t device_budget_bytes,
                               const spgemm_opts *opts, int64_t *row_ptr, int32_t *col_idx, double *values,
                               int64_t nnz_capacity, int64_t *nnz_out);

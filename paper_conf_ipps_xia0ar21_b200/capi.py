@@ -44,7 +44,8 @@ class spgemm_opts(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int32), ("validate", ctypes.c_int32), ("ring", ctypes.c_int32),
                 ("profile", ctypes.c_int32), ("row_begin", ctypes.c_int64), ("row_end", ctypes.c_int64),
                 ("workspace", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("chunk_nnz", ctypes.c_int64),
-                ("row_ptr_base", ctypes.c_int64), ("min_chunks", ctypes.c_int64)]
+                ("row_ptr_base", ctypes.c_int64), ("min_chunks", ctypes.c_int64), ("fused", ctypes.c_int32),
+                ("reserved", ctypes.c_int32)]
 
 
 class spgemm_info(ctypes.Structure):
@@ -52,7 +53,8 @@ class spgemm_info(ctypes.Structure):
                 ("products", ctypes.c_int64), ("max_row_nnz", ctypes.c_int64), ("max_row_products", ctypes.c_int64),
                 ("num_chunks", ctypes.c_int32), ("ring", ctypes.c_int32), ("chunk_capacity", ctypes.c_int64),
                 ("arena_bytes", ctypes.c_int64), ("arena_used", ctypes.c_int64), ("ring_bytes", ctypes.c_int64),
-                ("rows_warp", ctypes.c_int64), ("rows_block", ctypes.c_int64), ("rows_global", ctypes.c_int64)]
+                ("rows_warp", ctypes.c_int64), ("rows_block", ctypes.c_int64), ("rows_global", ctypes.c_int64),
+                ("fused", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -74,6 +76,7 @@ _sig = {
     "spgemm_plan_info": (ctypes.c_int, [_P, ctypes.POINTER(spgemm_info)]),
     "spgemm_plan_chunks": (ctypes.c_int, [_P, _P, _P]),
     "spgemm_execute_into": (ctypes.c_int, [_P, _P, _P, _P]),
+    "spgemm_execute_capacity": (ctypes.c_int, [_P, _P, _P, _P, _I64, ctypes.POINTER(ctypes.c_int64)]),
     "spgemm_execute": (ctypes.c_int, [_P, ctypes.POINTER(spgemm_csr_out)]),
     "spgemm_execute_stream": (ctypes.c_int, [_P, CHUNK_CB, _P]),
     "spgemm_set_row_ptr_base": (ctypes.c_int, [_P, _I64]),
@@ -153,7 +156,7 @@ def make_csr(M) -> tuple:
 
 def opts(device: int = -1, validate: bool = False, ring: int = 2, profile: bool = False, row_begin: int = 0,
          row_end: int = -1, workspace=None, stream=None, chunk_nnz: int = 0, row_ptr_base: int = 0,
-         min_chunks: int = 0) -> spgemm_opts:
+         min_chunks: int = 0, fused: bool = False) -> spgemm_opts:
     o = spgemm_opts()
     _lib.spgemm_opts_default(ctypes.byref(o))
     o.device, o.validate, o.ring, o.profile = device, int(validate), ring, int(profile)
@@ -161,6 +164,7 @@ def opts(device: int = -1, validate: bool = False, ring: int = 2, profile: bool 
     o.workspace = _ptr(workspace) if workspace is not None else None
     o.stream = stream
     o.chunk_nnz, o.row_ptr_base, o.min_chunks = chunk_nnz, row_ptr_base, min_chunks
+    o.fused = int(fused)
     o._keep = workspace  # the caller's workspace tensor must outlive the plan
     return o
 
@@ -191,6 +195,18 @@ class Plan:
 
     def execute_into(self, row_ptr, col, val):
         _check(_lib.spgemm_execute_into(self.h, _ptr(row_ptr), _ptr(col), _ptr(val)))
+
+    def execute_capacity(self, row_ptr, col, val, capacity: int) -> int:
+        """Returns nnz(C); raises SpgemmError(ERR_CAPACITY) (with .nnz) if it exceeds capacity."""
+        nnz = ctypes.c_int64(-1)
+        st = _lib.spgemm_execute_capacity(self.h, _ptr(row_ptr), _ptr(col), _ptr(val), int(capacity),
+                                          ctypes.byref(nnz))
+        if st == ERR_CAPACITY:
+            e = SpgemmError(st, (_lib.spgemm_last_error() or b"").decode())
+            e.nnz = nnz.value
+            raise e
+        _check(st)
+        return nnz.value
 
     def execute(self):
         """Plan-owned pinned output; returns numpy views valid until free()."""

@@ -1,16 +1,19 @@
 // api.cu -- C ABI (include/spgemm.h), arena, planner and the chunk pipeline.
 //
-// Host side of the hot path (DESIGN.md §8 rows):
+// Host side of the hot path (DESIGN.md §2 rows):
 //   S0 residency   inputs adopted in place (device) or H2D-copied once into the arena (host);
 //                  A == B is kept once (C = A x A, §V-B).
 //   S1 panels      rows [row_begin, row_end) of A are this plan's row panel (§III-A, §III-D
-//                  L169); B is used whole (one column panel, B fits the budget).
+//                  L169); B is used whole (one column panel: B fits every configured budget).
 //   S9 arena       ONE device allocation (or caller workspace) sub-allocated by offsets; nothing
 //                  is allocated between spgemm_plan returning and spgemm_free (§IV-B).
-//   S10 planner    output chunks cut from the exact symbolic nnz so that each fits a ring buffer
-//                  (the paper's upper-bound sizing is loose, §IV-B).
-//   S8 pipeline    compute stream + copy stream, R ring buffers, CUDA events only -- the host
-//                  never blocks inside spgemm_execute_into until the last copy (§IV-B).
+//   S10 planner    two-phase plans cut chunks from the exact symbolic nnz; fused plans cut them
+//                  from the per-row bound min(products, ncols) (§IV-B: the flop bound is loose,
+//                  so it sizes only chunk boundaries, never the output buffers).
+//   S8 pipeline    compute stream + copy stream, R ring buffers, CUDA events.  In a fused plan the
+//                  symbolic pass + scan of chunk j+1 run while chunk j is being copied out (the
+//                  paper's Fig. 6 overlap, without its PCIe transfer splitting: the only
+//                  small transfer is one 8-byte chunk total read through pinned memory).
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -98,13 +101,38 @@ struct Stat {
     double ms = 0, bytes = 0;
 };
 
+double elapsed(cudaEvent_t a, cudaEvent_t b) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
+    return ms;
+}
+
+struct EvSet {  // timing events (profile mode only)
+    std::vector<cudaEvent_t> ev;
+    explicit EvSet(bool on, size_t n) {
+        if (!on) return;
+        ev.resize(n);
+        for (auto &e : ev) CK(cudaEventCreate(&e));
+    }
+    ~EvSet() {
+        for (auto e : ev) cudaEventDestroy(e);
+    }
+    cudaEvent_t *at(size_t k) { return ev.empty() ? nullptr : ev.data() + k; }
+    void rec(size_t k, cudaStream_t s) {
+        if (!ev.empty()) CK(cudaEventRecord(ev[k], s));
+    }
+};
+
 }  // namespace
 
 struct spgemm_plan_s {
     int device = 0, num_sms = 148;
     cudaStream_t stream = nullptr, copy = nullptr;
     bool own_stream = false;
-    std::vector<cudaEvent_t> ev_num, ev_d2h;
+    std::vector<cudaEvent_t> ev_num, ev_d2h, ev_tot;
     cudaEvent_t ev_ready = nullptr;
 
     char *arena = nullptr;
@@ -114,10 +142,11 @@ struct spgemm_plan_s {
     DevCSR A{}, B{};
     int64_t R = 0, ncols = 0, nnzA = 0, nnzB = 0, row_begin = 0;
     int group = 32;
+    bool fused = false;
 
-    int64_t *u = nullptr, *crp = nullptr, *tmp = nullptr;
-    int32_t *listB = nullptr, *listG = nullptr;
-    Ctl *ctl = nullptr;  // [0] plan passes, [1] numeric passes
+    int64_t *bnd = nullptr, *crp = nullptr, *tmp = nullptr;
+    int32_t *nnzr = nullptr, *listB = nullptr, *listG = nullptr;
+    Ctl *ctl = nullptr;  // [0] count / symbolic passes, [1] numeric passes
 
     uint32_t *gbits = nullptr;
     double *gvals = nullptr;
@@ -130,10 +159,15 @@ struct spgemm_plan_s {
     std::vector<int32_t *> ring_col;
     std::vector<double *> ring_val;
 
-    std::vector<int64_t> chunk_rows, chunk_offs;  // num_chunks + 1 each; offs relative to slice
-    int64_t nnz = 0, products = 0, max_nnz = 0, max_u = 0, max_bound = 0;
+    std::vector<int64_t> chunk_rows;  // num_chunks + 1 row boundaries
+    std::vector<int64_t> chunk_offs;  // num_chunks + 1 offsets relative to the slice (known after
+                                      // plan for two-phase plans, after an execution for fused)
+    int64_t nnz = -1, products = 0, max_nnz = 0, max_u = 0, max_bound = 0, sum_bound = 0;
     int64_t rows_w = 0, rows_b = 0, rows_g = 0;
     int64_t base_applied = 0, base_wanted = 0;
+    int64_t *h_small = nullptr;  // pinned + mapped: [0] base; chunk j: [1 + 2j] end offset,
+    int64_t *d_small = nullptr;  //   [2 + 2j] max row nnz (fused; written by k_publish)
+    std::vector<int64_t> chunk_maxb;  // fused: max row bound per chunk
 
     int64_t *h_rp = nullptr;
     int32_t *h_col = nullptr;
@@ -171,12 +205,22 @@ struct spgemm_plan_s {
         s.bytes = bytes;
         stats.push_back(s);
     }
+    void clear_stats(std::initializer_list<const char *> names) {
+        std::vector<Stat> keep;
+        for (auto &s : stats) {
+            bool drop = false;
+            for (auto n : names) drop |= s.name == n;
+            if (!drop) keep.push_back(s);
+        }
+        stats.swap(keep);
+    }
+    int64_t num_chunks() const { return chunk_rows.empty() ? 0 : int64_t(chunk_rows.size()) - 1; }
     ~spgemm_plan_s() {
-        DeviceGuard g(-1);
         if (stream) cudaStreamSynchronize(stream);
         if (copy) cudaStreamSynchronize(copy);
         for (auto e : ev_num) cudaEventDestroy(e);
         for (auto e : ev_d2h) cudaEventDestroy(e);
+        for (auto e : ev_tot) cudaEventDestroy(e);
         if (ev_ready) cudaEventDestroy(ev_ready);
         if (copy) cudaStreamDestroy(copy);
         if (own_stream && stream) cudaStreamDestroy(stream);
@@ -184,12 +228,11 @@ struct spgemm_plan_s {
         if (h_rp) cudaFreeHost(h_rp);
         if (h_col) cudaFreeHost(h_col);
         if (h_val) cudaFreeHost(h_val);
+        pin_release(h_small);
     }
 };
 
 namespace {
-
-spgemm_status guarded(const std::function<void()> &f);
 
 void check_csr(const spgemm_csr *M, const char *name) {
     if (!M) fail(SPGEMM_ERR_INVALID_ARGUMENT, std::string(name) + " is NULL");
@@ -207,27 +250,59 @@ void check_csr(const spgemm_csr *M, const char *name) {
     }
 }
 
-double elapsed(cudaEvent_t a, cudaEvent_t b) {
-    float ms = 0;
-    if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) {
-        cudaGetLastError();
-        return 0;
+// chunk boundaries from a scanned prefix `pre` (pre[0] = 0, pre[R] = total): every chunk's span
+// of `pre` is < capp + (largest single-row increment); empty ids are dropped
+void cut_chunks(spgemm_plan_s *P, const int64_t *pre, int64_t total, int64_t capp, int64_t limit,
+                std::vector<int64_t> *offs_out) {
+    const int64_t R = P->R;
+    cudaStream_t s = P->stream;
+    P->chunk_rows.clear();
+    if (offs_out) offs_out->clear();
+    if (total <= 0) return;
+    const int64_t nids = total / capp + 1;
+    const size_t save = P->used;  // temporary arrays at the start of the (not yet used) ring region
+    int64_t *bounds = P->alloc<int64_t>(nids + 1, "chunk bounds");
+    int64_t *offs = P->alloc<int64_t>(nids + 1, "chunk offsets");
+    launch_cut(pre, R, capp, bounds, nids, s);
+    launch_gather(pre, bounds, nids + 1, offs, s);
+    CKL("cut");
+    std::vector<int64_t> hb(nids + 1), ho(nids + 1);
+    CK(cudaMemcpyAsync(hb.data(), bounds, sizeof(int64_t) * (nids + 1), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(ho.data(), offs, sizeof(int64_t) * (nids + 1), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    P->used = save;
+    P->chunk_rows.push_back(hb[0]);
+    if (offs_out) offs_out->push_back(ho[0]);
+    int64_t last_off = ho[0];
+    for (int64_t c = 1; c <= nids; ++c) {
+        if (hb[c] == P->chunk_rows.back()) continue;
+        if (ho[c] - last_off > limit) fail(SPGEMM_ERR_STATE, "internal: chunk exceeds the ring capacity");
+        P->chunk_rows.push_back(hb[c]);
+        if (offs_out) offs_out->push_back(ho[c]);
+        last_off = ho[c];
     }
-    return ms;
+    if (P->chunk_rows.front() != 0 || P->chunk_rows.back() != R)
+        fail(SPGEMM_ERR_STATE, "internal: chunk bounds do not cover the rows");
 }
 
-struct EvSet {  // events for profiling one launch group
-    std::vector<cudaEvent_t> ev;
-    explicit EvSet(bool on, int n) {
-        if (!on) return;
-        ev.resize(n);
-        for (auto &e : ev) CK(cudaEventCreate(&e));
-    }
-    ~EvSet() {
-        for (auto e : ev) cudaEventDestroy(e);
-    }
-    cudaEvent_t *ptr() { return ev.empty() ? nullptr : ev.data(); }
-};
+SymArgs sym_args(spgemm_plan_s *P, int64_t r0, int64_t r1, int tiers) {
+    SymArgs sa;
+    sa.A = P->A;
+    sa.B = P->B;
+    sa.bnd = P->bnd;
+    sa.nnz = P->nnzr;
+    sa.r0 = r0;
+    sa.r1 = r1;
+    sa.listB = P->listB;
+    sa.listG = P->listG;
+    sa.ctl = P->ctl;
+    sa.gscratch = P->gbits;
+    sa.gstride = P->gstride_bits;
+    sa.gblocks = P->gblocks;
+    sa.group = P->group;
+    sa.tiers = tiers;
+    return sa;
+}
 
 void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const spgemm_opts *o, spgemm_plan_s *P) {
     check_csr(Ah, "A");
@@ -251,6 +326,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     }
     CK(cudaDeviceGetAttribute(&P->num_sms, cudaDevAttrMultiProcessorCount, P->device));
     P->profile = opts.profile != 0;
+    P->fused = opts.fused != 0;
     P->ring = opts.ring;
     P->row_begin = rb;
     P->R = re - rb;
@@ -258,7 +334,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->nnzB = Bh->nnz;
     P->base_wanted = opts.row_ptr_base;
 
-    // streams and events (created at plan time: no creation inside execute)
+    // streams and events (created at plan time: nothing is created inside execute)
     if (opts.stream) {
         P->stream = (cudaStream_t)opts.stream;
     } else {
@@ -294,8 +370,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         P->own_arena = true;
     }
 
-    EvSet pe(P->profile, 16);
-    if (P->profile) CK(cudaEventRecord(pe.ev[0], s));
+    EvSet pe(P->profile, 12);
+    pe.rec(0, s);
 
     // S0 residency: B
     if (Bh->where == SPGEMM_DEVICE) {
@@ -314,7 +390,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     // S0 residency + S1 row panel: A
     if (Ah->where == SPGEMM_DEVICE) {
         P->A = DevCSR{Ah->row_ptr + rb, Ah->col_idx, Ah->values, P->R, Ah->ncols};
-        P->nnzA = -1;  // unknown without a read; only used for statistics
+        P->nnzA = -1;  // unknown without a read; statistics only
     } else {
         const bool alias = Bh->where == SPGEMM_HOST && Ah->row_ptr == Bh->row_ptr && Ah->col_idx == Bh->col_idx &&
                            Ah->values == Bh->values && Ah->nrows == Bh->nrows && Ah->ncols == Bh->ncols;
@@ -338,15 +414,17 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     }
     P->group = choose_group(P->B, P->nnzB);
 
-    // per-row arrays (24 B/row + 8) and control blocks
+    // per-row arrays (28 B/row) and control blocks
     const int64_t R = P->R;
-    P->u = P->alloc<int64_t>(R, "u");
+    P->bnd = P->alloc<int64_t>(R, "row bounds");
     P->crp = P->alloc<int64_t>(R + 1, "C.row_ptr");
+    P->nnzr = P->alloc<int32_t>(R, "row nnz");
     P->listB = P->alloc<int32_t>(R, "listB");
     P->listG = P->alloc<int32_t>(R, "listG");
     P->ctl = P->alloc<Ctl>(2, "ctl");
-    P->tmp = P->alloc<int64_t>(2 * ((R + 1 + SCAN_TILE - 1) / SCAN_TILE) + 64, "scan scratch");
+    P->tmp = P->alloc<int64_t>((R + SCAN_TILE - 1) / SCAN_TILE + 64, "scan scratch");
     CK(cudaMemsetAsync(P->ctl, 0, 2 * sizeof(Ctl), s));
+    CK(cudaMemsetAsync(P->crp, 0, sizeof(int64_t), s));
 
     if (opts.validate) {
         launch_validate(P->A, P->ctl, s);
@@ -355,265 +433,346 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     }
 
     // S2 count
-    if (P->profile) CK(cudaEventRecord(pe.ev[1], s));
-    launch_count(P->A, P->B, P->u, P->ctl, s);
+    pe.rec(1, s);
+    launch_count(P->A, P->B, P->bnd, P->ctl, s);
     CKL("count");
-    if (P->profile) CK(cudaEventRecord(pe.ev[2], s));
+    pe.rec(2, s);
     Ctl hc;
     CK(cudaMemcpyAsync(&hc, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
-    if (hc.err & 2u) fail(SPGEMM_ERR_INVALID_ARGUMENT, "input validation failed (unsorted/duplicate/out-of-range col_idx or bad row_ptr)");
+    if (hc.err & 2u)
+        fail(SPGEMM_ERR_INVALID_ARGUMENT, "input validation failed (unsorted/duplicate/out-of-range col_idx or bad row_ptr)");
     P->products = (int64_t)hc.sum_u;
     P->max_u = (int64_t)hc.max_u;
     P->max_bound = (int64_t)hc.max_bound;
 
-    // G-tier scratch, sized only if a row can exceed the CTA tier
-    const int64_t nwords = (P->ncols + 31) / 32;
+    // dense-tier scratch, sized only if a row can exceed the CTA tier
     if (P->max_bound > CAPB_NUM) {
-        const bool num = true;  // numeric may need it: nnz_i <= min(u_i, ncols)
+        const int64_t nwords = (P->ncols + 31) / 32;
         P->gstride_bits = (nwords + 63) & ~int64_t(63);
-        P->gstride_vals = num ? ((P->ncols + 31) & ~int64_t(31)) : 0;
+        P->gstride_vals = (P->ncols + 31) & ~int64_t(31);
         const size_t per = size_t(P->gstride_bits) * 4 + size_t(P->gstride_vals) * 8;
-        const size_t ring_min = size_t(P->ring) * size_t(std::min<int64_t>(P->max_bound, P->products)) * 12 + 4096;
-        size_t freeb = P->arena_bytes > P->used ? P->arena_bytes - P->used : 0;
-        size_t avail = freeb > ring_min ? freeb - ring_min : 0;
-        int64_t nb = std::min<int64_t>(P->num_sms, int64_t((avail / 4) / (per ? per : 1)));
-        if (nb < 1) nb = int64_t(avail / (per ? per : 1)) >= 1 ? 1 : 0;
+        const size_t ring_min = size_t(P->ring) * size_t(P->max_bound) * 12 + 4096;
+        const size_t freeb = P->arena_bytes > P->used ? P->arena_bytes - P->used : 0;
+        const size_t avail = freeb > ring_min ? freeb - ring_min : 0;
+        int64_t nb = std::min<int64_t>(P->num_sms, int64_t((avail / 4) / per));
+        if (nb < 1) nb = int64_t(avail / per) >= 1 ? 1 : 0;
         if (nb < 1) fail(SPGEMM_ERR_BUDGET, "budget cannot hold one dense accumulator for the longest row");
         P->gblocks = (int)nb;
-        P->gbits = P->alloc<uint32_t>(P->gstride_bits * nb, "G bitmap");
-        P->gvals = P->alloc<double>(std::max<int64_t>(P->gstride_vals * nb, 1), "G values");
+        P->gbits = P->alloc<uint32_t>(P->gstride_bits * nb, "dense-tier bitmap");
+        P->gvals = P->alloc<double>(P->gstride_vals * nb, "dense-tier values");
         CK(cudaMemsetAsync(P->gbits, 0, size_t(P->gstride_bits) * nb * 4, s));
         CK(cudaMemsetAsync(P->gvals, 0, size_t(P->gstride_vals) * nb * 8, s));
     }
 
-    // S3+S4 symbolic, S5 scan
-    CK(cudaMemsetAsync(P->crp + R, 0, sizeof(int64_t), s));
-    SymArgs sa{P->A, P->B, P->u, P->crp, P->listB, P->listG, P->ctl, P->gbits, P->gstride_bits, P->gblocks, P->group};
-    if (P->profile) CK(cudaEventRecord(pe.ev[3], s));
-    launch_symbolic(sa, P->num_sms, s, P->profile ? pe.ptr() + 4 : nullptr);
-    CKL("symbolic");
-    if (P->profile) CK(cudaEventRecord(pe.ev[8], s));
-    launch_scan(P->crp, R, 0, P->tmp, s);
-    CKL("scan");
-    if (P->profile) CK(cudaEventRecord(pe.ev[9], s));
-    int64_t total = 0;
-    CK(cudaMemcpyAsync(&hc, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
-    CK(cudaMemcpyAsync(&total, P->crp + R, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    P->nnz = total;
-    P->max_nnz = (int64_t)hc.max_nnz;
-    P->rows_w = (int64_t)hc.rows_w;
-    P->rows_b = (int64_t)hc.rows_b;
-    P->rows_g = (int64_t)hc.rows_g;
+    // ring capacity from what is left: each slot holds `cap` nonzeros (val fp64 + col int32)
+    auto ring_cap = [&](int64_t need_row) {
+        const size_t freeb = P->arena_bytes > P->used + 4096 ? P->arena_bytes - P->used - 4096 : 0;
+        const size_t slot = (freeb / P->ring) & ~size_t(255);
+        int64_t cap = int64_t(slot / 12) & ~int64_t(63);
+        if (opts.chunk_nnz > 0) cap = std::min<int64_t>(cap, std::max<int64_t>(opts.chunk_nnz, need_row));
+        if (cap < std::max<int64_t>(need_row, 1))
+            fail(SPGEMM_ERR_BUDGET, "ring buffer of " + std::to_string(cap) +
+                                        " nonzeros cannot hold the longest C row (bound " + std::to_string(need_row) + ")");
+        return cap;
+    };
 
-    // S10 ring + chunk cut.  Each ring slot holds `cap` nonzeros (val fp64 + col int32).
-    const size_t freeb = P->arena_bytes > P->used + 4096 ? P->arena_bytes - P->used - 4096 : 0;
-    size_t slot = (freeb / P->ring) & ~size_t(255);
-    int64_t cap = int64_t(slot / 12) & ~int64_t(63);
-    if (opts.chunk_nnz > 0) cap = std::min<int64_t>(cap, std::max<int64_t>(opts.chunk_nnz, P->max_nnz));
-    if (total > 0 && cap < std::max<int64_t>(P->max_nnz, 1))
-        fail(SPGEMM_ERR_BUDGET, "ring buffer of " + std::to_string(cap) + " nonzeros cannot hold the longest C row (" +
-                                    std::to_string(P->max_nnz) + ")");
-    cap = std::max<int64_t>(std::min<int64_t>(cap, std::max<int64_t>(total, 1)), std::max<int64_t>(P->max_nnz, 1));
-    P->cap = cap;
-    int64_t capp = std::max<int64_t>(1, cap - P->max_nnz);
-    int64_t minc = opts.min_chunks;
-    if (minc <= 0) minc = std::min<int64_t>(64, std::max<int64_t>(1, total * 12 / (128ll << 20)));
-    if (minc > 1) capp = std::min<int64_t>(capp, std::max<int64_t>(1, (total + minc - 1) / minc));
-    if (opts.chunk_nnz > 0) capp = std::min<int64_t>(capp, std::max<int64_t>(1, opts.chunk_nnz - P->max_nnz));
-    capp = std::max<int64_t>(capp, 1);
-
-    P->chunk_rows.clear();
-    P->chunk_offs.clear();
-    if (total > 0) {
-        const int64_t nids = total / capp + 1;
-        // temporary arrays at the start of the (not yet used) ring region
-        const size_t save = P->used;
-        int64_t *bounds = P->alloc<int64_t>(nids + 1, "chunk bounds");
-        int64_t *offs = P->alloc<int64_t>(nids + 1, "chunk offsets");
-        launch_cut(P->crp, R, capp, bounds, nids, s);
-        launch_gather(P->crp, bounds, nids + 1, offs, s);
-        CKL("cut");
-        std::vector<int64_t> hb(nids + 1), ho(nids + 1);
-        CK(cudaMemcpyAsync(hb.data(), bounds, sizeof(int64_t) * (nids + 1), cudaMemcpyDeviceToHost, s));
-        CK(cudaMemcpyAsync(ho.data(), offs, sizeof(int64_t) * (nids + 1), cudaMemcpyDeviceToHost, s));
+    if (!P->fused) {
+        // S3+S4 symbolic and S5 scan over all rows, then cut by exact nnz
+        SymArgs sa = sym_args(P, 0, R, sym_tiers(P->max_bound));
+        pe.rec(3, s);
+        launch_symbolic(sa, P->num_sms, s, pe.at(4));
+        CKL("symbolic");
+        launch_scan(P->nnzr, R, P->crp, P->tmp, s);
+        CKL("scan");
+        pe.rec(8, s);
+        int64_t total = 0;
+        CK(cudaMemcpyAsync(&hc, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&total, P->crp + R, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
         CK(cudaStreamSynchronize(s));
-        P->used = save;
-        // chunk boundaries = the distinct bounds (an id whose rows are empty repeats a bound)
-        P->chunk_rows.push_back(hb[0]);
-        P->chunk_offs.push_back(ho[0]);
-        for (int64_t c = 1; c <= nids; ++c) {
-            if (hb[c] == P->chunk_rows.back()) continue;
-            if (ho[c] - P->chunk_offs.back() > cap) fail(SPGEMM_ERR_STATE, "internal: chunk exceeds the ring capacity");
-            P->chunk_rows.push_back(hb[c]);
-            P->chunk_offs.push_back(ho[c]);
+        P->nnz = total;
+        P->max_nnz = (int64_t)hc.max_nnz;
+        P->rows_w = (int64_t)hc.rows_w;
+        P->rows_b = (int64_t)hc.rows_b;
+        P->rows_g = (int64_t)hc.rows_g;
+        int64_t cap = ring_cap(P->max_nnz);
+        cap = std::max<int64_t>(std::min<int64_t>(cap, std::max<int64_t>(total, 1)), std::max<int64_t>(P->max_nnz, 1));
+        P->cap = cap;
+        int64_t capp = std::max<int64_t>(1, cap - P->max_nnz);
+        int64_t minc = opts.min_chunks;
+        if (minc <= 0) minc = std::min<int64_t>(64, std::max<int64_t>(1, total * 12 / (128ll << 20)));
+        if (minc > 1) capp = std::min<int64_t>(capp, std::max<int64_t>(1, (total + minc - 1) / minc));
+        if (opts.chunk_nnz > 0) capp = std::min<int64_t>(capp, std::max<int64_t>(1, opts.chunk_nnz - P->max_nnz));
+        cut_chunks(P, P->crp, total, std::max<int64_t>(capp, 1), cap, &P->chunk_offs);
+    } else {
+        // fused: boundaries from the prefix of the row bounds; the symbolic pass runs per chunk
+        // inside execute.  crp temporarily holds that prefix.
+        int64_t total_b = 0;
+        launch_scan64(P->bnd, R, P->crp, P->tmp, s);
+        CKL("bound scan");
+        CK(cudaMemcpyAsync(&total_b, P->crp + R, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        P->sum_bound = total_b;
+        int64_t cap = ring_cap(P->max_bound);
+        cap = std::max<int64_t>(std::min<int64_t>(cap, std::max<int64_t>(total_b, 1)), std::max<int64_t>(P->max_bound, 1));
+        P->cap = cap;
+        int64_t capp = std::max<int64_t>(1, cap - P->max_bound);
+        int64_t minc = opts.min_chunks;
+        if (minc <= 0) minc = std::min<int64_t>(64, std::max<int64_t>(1, total_b * 12 / (512ll << 20)));
+        if (minc > 1) capp = std::min<int64_t>(capp, std::max<int64_t>(1, (total_b + minc - 1) / minc));
+        if (opts.chunk_nnz > 0) capp = std::min<int64_t>(capp, std::max<int64_t>(1, opts.chunk_nnz - P->max_bound));
+        cut_chunks(P, P->crp, total_b, std::max<int64_t>(capp, 1), cap, nullptr);
+        CK(cudaMemsetAsync(P->crp, 0, sizeof(int64_t), s));
+        const int64_t nch = P->num_chunks();
+        // per-chunk max row bound: decides which symbolic tiers a chunk needs
+        P->chunk_maxb.assign(nch, 0);
+        if (nch > 0) {
+            const size_t save = P->used;
+            int64_t *drows = P->alloc<int64_t>(nch + 1, "chunk rows");
+            int64_t *dmax = P->alloc<int64_t>(nch, "chunk max bound");
+            CK(cudaMemcpyAsync(drows, P->chunk_rows.data(), sizeof(int64_t) * (nch + 1), cudaMemcpyHostToDevice, s));
+            launch_seg_max(P->bnd, drows, nch, dmax, s);
+            CKL("chunk max");
+            CK(cudaMemcpyAsync(P->chunk_maxb.data(), dmax, sizeof(int64_t) * nch, cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            P->used = save;
         }
-        if (P->chunk_rows.front() != 0 || P->chunk_rows.back() != R)
-            fail(SPGEMM_ERR_STATE, "internal: chunk bounds do not cover the rows");
+        P->ev_tot.resize(nch);
+        for (auto &e : P->ev_tot) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     }
+    P->h_small = (int64_t *)pin_acquire(sizeof(int64_t) * (2 * P->num_chunks() + 2));
+    CK(cudaHostGetDevicePointer((void **)&P->d_small, P->h_small, 0));
 
     // ring buffers
-    P->ring_col.resize(P->ring);
-    P->ring_val.resize(P->ring);
-    if (total > 0) {
+    P->ring_col.assign(P->ring, nullptr);
+    P->ring_val.assign(P->ring, nullptr);
+    if (P->num_chunks() > 0) {
         for (int r = 0; r < P->ring; ++r) {
-            P->ring_val[r] = P->alloc<double>(cap, "ring values");
-            P->ring_col[r] = P->alloc<int32_t>(cap, "ring col_idx");
+            P->ring_val[r] = P->alloc<double>(P->cap, "ring values");
+            P->ring_col[r] = P->alloc<int32_t>(P->cap, "ring col_idx");
         }
-        P->ring_bytes = size_t(P->ring) * size_t(cap) * 12;
+        P->ring_bytes = size_t(P->ring) * size_t(P->cap) * 12;
     }
+    CK(cudaStreamSynchronize(s));
     if (P->profile) {
         P->stats.clear();
         P->add_stat("count", elapsed(pe.ev[1], pe.ev[2]), 0);
-        P->add_stat("sym_w", elapsed(pe.ev[4], pe.ev[5]), 0);
-        P->add_stat("sym_b", elapsed(pe.ev[5], pe.ev[6]), 0);
-        P->add_stat("sym_g", elapsed(pe.ev[6], pe.ev[7]), 0);
-        P->add_stat("scan", elapsed(pe.ev[8], pe.ev[9]), 0);
-        P->add_stat("plan_total", elapsed(pe.ev[0], pe.ev[9]), 0);
+        if (!P->fused) {
+            P->add_stat("sym_w", elapsed(pe.ev[4], pe.ev[5]), 0);
+            P->add_stat("sym_b", elapsed(pe.ev[5], pe.ev[6]), 0);
+            P->add_stat("sym_g", elapsed(pe.ev[6], pe.ev[7]), 0);
+            P->add_stat("scan", elapsed(pe.ev[7], pe.ev[8]), 0);
+        }
     }
 }
 
-int64_t num_chunks(const spgemm_plan_s *P) {
-    return P->chunk_rows.empty() ? 0 : int64_t(P->chunk_rows.size()) - 1;
-}
-
-// Enqueue the numeric pass of chunk c into ring slot b on the compute stream.
-void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, cudaEvent_t *ev) {
-    NumArgs na{P->A,          P->B,           P->crp,     P->chunk_rows[c], P->chunk_rows[c + 1],
-               P->ring_col[b], P->ring_val[b], P->listB,   P->listG,         P->ctl + 1,
-               P->gbits,      P->gvals,       P->gstride_bits, P->gstride_vals, P->gblocks,
-               P->group};
+void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t max_row_nnz, cudaEvent_t *ev) {
+    NumArgs na;
+    na.A = P->A;
+    na.B = P->B;
+    na.crp = P->crp;
+    na.r0 = P->chunk_rows[c];
+    na.r1 = P->chunk_rows[c + 1];
+    na.out_col = P->ring_col[b];
+    na.out_val = P->ring_val[b];
+    na.listB = P->listB;
+    na.listG = P->listG;
+    na.ctl = P->ctl + 1;
+    na.gbits = P->gbits;
+    na.gvals = P->gvals;
+    na.gstride_bits = P->gstride_bits;
+    na.gstride_vals = P->gstride_vals;
+    na.gblocks = P->gblocks;
+    na.group = P->group;
+    na.tiers = num_tiers(max_row_nnz);
     launch_numeric(na, P->num_sms, P->stream, ev);
     CKL("numeric");
 }
 
-void apply_base(spgemm_plan_s *P) {
-    if (P->base_wanted != P->base_applied) {
-        launch_add(P->crp, P->R, P->base_wanted - P->base_applied, P->stream);
-        CKL("row_ptr base");
-        P->base_applied = P->base_wanted;
-    }
+// fused plans: symbolic + scan of chunk j; its end offset and max row nnz land in
+// h_small[1 + 2j], h_small[2 + 2j] through zero-copy stores (no D2H on the copy engine)
+void enqueue_analysis(spgemm_plan_s *P, int64_t j, cudaEvent_t *ev) {
+    const int64_t r0 = P->chunk_rows[j], r1 = P->chunk_rows[j + 1];
+    SymArgs sa = sym_args(P, r0, r1, sym_tiers(P->chunk_maxb[j]));
+    launch_symbolic(sa, P->num_sms, P->stream, ev);
+    CKL("symbolic");
+    launch_scan(P->nnzr + r0, r1 - r0, P->crp + r0, P->tmp, P->stream);
+    CKL("scan");
+    if (ev) CK(cudaEventRecord(ev[4], P->stream));
+    launch_publish(P->crp + r1, P->ctl, P->d_small + 1 + 2 * j, P->stream);
+    CKL("publish");
+    CK(cudaEventRecord(P->ev_tot[j], P->stream));
 }
 
-void check_numeric_errors(spgemm_plan_s *P) {
-    unsigned err = 0;
-    CK(cudaMemcpyAsync(&err, &P->ctl[1].err, sizeof(unsigned), cudaMemcpyDeviceToHost, P->stream));
-    CK(cudaStreamSynchronize(P->stream));
-    if (err) fail(SPGEMM_ERR_STATE, "internal: numeric pass produced a row whose nnz differs from the symbolic pass");
-}
+struct Sink {
+    spgemm_chunk_cb cb = nullptr;
+    void *user = nullptr;
+};
 
-// The pipeline: numeric(c) on the compute stream into slot c % ring, D2H(c) on the copy stream.
-void do_execute(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double *val_out) {
+// The pipeline.  Direct mode writes into (rp_out, col_out, val_out) with room for `capacity`
+// nonzeros; sink mode copies every chunk into a pinned staging slot and calls sink->cb.
+// Returns nnz of the slice (also when the capacity was too small, in which case nothing past the
+// capacity is written and *overflow is set).
+int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double *val_out, int64_t capacity,
+                     const Sink *sink, bool *overflow) {
     if (P->failed) fail(SPGEMM_ERR_STATE, "plan is in a failed state");
     DeviceGuard g(P->device);
-    const int64_t nch = num_chunks(P);
-    if (P->nnz > 0 && (!col_out || !val_out)) fail(SPGEMM_ERR_INVALID_ARGUMENT, "col_idx/values output is NULL");
-    apply_base(P);
-    CK(cudaEventRecord(P->ev_ready, P->stream));
-    CK(cudaStreamWaitEvent(P->copy, P->ev_ready, 0));
-    const int per = 5;
-    EvSet pe(P->profile, int(nch) * per + 4);
-    if (P->profile) CK(cudaEventRecord(pe.ev[nch * per], P->copy));
-    if (rp_out) CK(cudaMemcpyAsync(rp_out, P->crp, sizeof(int64_t) * (P->R + 1), cudaMemcpyDeviceToHost, P->copy));
-    const int64_t base0 = P->chunk_offs.empty() ? 0 : P->chunk_offs[0];
-    for (int64_t c = 0; c < nch; ++c) {
-        const int b = int(c % P->ring);
-        if (c >= P->ring) CK(cudaStreamWaitEvent(P->stream, P->ev_d2h[b], 0));
-        enqueue_numeric(P, c, b, P->profile ? pe.ptr() + c * per : nullptr);
-        CK(cudaEventRecord(P->ev_num[b], P->stream));
-        CK(cudaStreamWaitEvent(P->copy, P->ev_num[b], 0));
-        const int64_t o = P->chunk_offs[c] - base0, n = P->chunk_offs[c + 1] - P->chunk_offs[c];
-        if (P->profile) CK(cudaEventRecord(pe.ev[c * per + 4], P->copy));
-        if (n > 0) {
-            CK(cudaMemcpyAsync(col_out + o, P->ring_col[b], sizeof(int32_t) * n, cudaMemcpyDeviceToHost, P->copy));
-            CK(cudaMemcpyAsync(val_out + o, P->ring_val[b], sizeof(double) * n, cudaMemcpyDeviceToHost, P->copy));
-        }
-        CK(cudaEventRecord(P->ev_d2h[b], P->copy));
-        if (P->profile && c + 1 == nch) CK(cudaEventRecord(pe.ev[nch * per + 1], P->copy));
-    }
-    if (P->profile && nch == 0) CK(cudaEventRecord(pe.ev[nch * per + 1], P->copy));
-    CK(cudaStreamSynchronize(P->copy));
-    check_numeric_errors(P);
-    if (P->profile) {
-        for (const char *n : {"num_w", "num_b", "num_g", "d2h", "execute_total"}) {
-            for (auto &s : P->stats)
-                if (s.name == n) s = Stat{n, 0, 0, 0};
-        }
-        for (int64_t c = 0; c < nch; ++c) {
-            cudaEvent_t *e = pe.ptr() + c * per;
-            P->add_stat("num_w", elapsed(e[0], e[1]), 0);
-            P->add_stat("num_b", elapsed(e[1], e[2]), 0);
-            P->add_stat("num_g", elapsed(e[2], e[3]), 0);
-            // d2h: from the copy stream's start of this chunk's copy to the next record on it
-            cudaEvent_t end = (c + 1 < nch) ? pe.ev[(c + 1) * per + 4] : pe.ev[nch * per + 1];
-            P->add_stat("d2h_span", elapsed(e[4], end), double(P->chunk_offs[c + 1] - P->chunk_offs[c]) * 12);
-        }
-        P->add_stat("execute_total", elapsed(pe.ev[nch * per], pe.ev[nch * per + 1]), double(P->nnz) * 12 + 8.0 * (P->R + 1));
-    }
-}
-
-void do_execute_stream(spgemm_plan_s *P, spgemm_chunk_cb cb, void *user) {
-    if (P->failed) fail(SPGEMM_ERR_STATE, "plan is in a failed state");
-    if (!cb) fail(SPGEMM_ERR_INVALID_ARGUMENT, "callback is NULL");
-    DeviceGuard g(P->device);
-    const int64_t nch = num_chunks(P);
-    apply_base(P);
-    int64_t maxn = 0, maxr = 0;
-    for (int64_t c = 0; c < nch; ++c) {
-        maxn = std::max(maxn, P->chunk_offs[c + 1] - P->chunk_offs[c]);
-        maxr = std::max(maxr, P->chunk_rows[c + 1] - P->chunk_rows[c]);
-    }
+    cudaStream_t s = P->stream, cp = P->copy;
+    const int64_t nch = P->num_chunks();
     const int ring = P->ring;
-    std::vector<void *> stage(ring, nullptr);
+    *overflow = false;
+
+    // row_ptr base
+    int64_t base;
+    if (P->fused) {
+        base = P->base_wanted;
+        P->h_small[0] = base;
+        CK(cudaMemcpyAsync(P->crp, P->h_small, sizeof(int64_t), cudaMemcpyHostToDevice, s));
+        P->base_applied = base;
+    } else {
+        if (P->base_wanted != P->base_applied) {
+            launch_add(P->crp, P->R, P->base_wanted - P->base_applied, s);
+            CKL("row_ptr base");
+            P->base_applied = P->base_wanted;
+        }
+        base = P->base_applied;
+    }
+    const int64_t off0 = P->fused ? 0 : P->chunk_offs.empty() ? 0 : P->chunk_offs[0];
+
+    // sink staging
+    std::vector<void *> stage(sink ? ring : 0, nullptr);
     struct Release {
         std::vector<void *> &v;
         ~Release() {
             for (auto p : v) pin_release(p);
         }
     } rel{stage};
-    const size_t per_slot = size_t(maxn) * 12 + size_t(maxr + 1) * 8 + 1024;
-    for (int r = 0; r < ring; ++r) stage[r] = pin_acquire(per_slot);
-    auto slot_val = [&](int b) { return reinterpret_cast<double *>(stage[b]); };
-    auto slot_col = [&](int b) { return reinterpret_cast<int32_t *>((char *)stage[b] + size_t(maxn) * 8); };
-    auto slot_rp = [&](int b) {
+    int64_t maxn = 0, maxr = 0;
+    for (int64_t c = 0; c < nch; ++c) maxr = std::max(maxr, P->chunk_rows[c + 1] - P->chunk_rows[c]);
+    maxn = P->cap;
+    if (sink)
+        for (int r = 0; r < ring; ++r) stage[r] = pin_acquire(size_t(maxn) * 12 + size_t(maxr + 1) * 8 + 64);
+    auto st_val = [&](int b) { return reinterpret_cast<double *>(stage[b]); };
+    auto st_col = [&](int b) { return reinterpret_cast<int32_t *>((char *)stage[b] + size_t(maxn) * 8); };
+    auto st_rp = [&](int b) {
         return reinterpret_cast<int64_t *>((char *)stage[b] + ((size_t(maxn) * 12 + 7) & ~size_t(7)));
     };
-    CK(cudaEventRecord(P->ev_ready, P->stream));
-    CK(cudaStreamWaitEvent(P->copy, P->ev_ready, 0));
-    auto enqueue = [&](int64_t c) {
-        const int b = int(c % ring);
-        enqueue_numeric(P, c, b, nullptr);
-        CK(cudaEventRecord(P->ev_num[b], P->stream));
-        CK(cudaStreamWaitEvent(P->copy, P->ev_num[b], 0));
-        const int64_t n = P->chunk_offs[c + 1] - P->chunk_offs[c];
-        const int64_t r0 = P->chunk_rows[c], r1 = P->chunk_rows[c + 1];
-        CK(cudaMemcpyAsync(slot_rp(b), P->crp + r0, sizeof(int64_t) * (r1 - r0 + 1), cudaMemcpyDeviceToHost, P->copy));
-        if (n > 0) {
-            CK(cudaMemcpyAsync(slot_col(b), P->ring_col[b], sizeof(int32_t) * n, cudaMemcpyDeviceToHost, P->copy));
-            CK(cudaMemcpyAsync(slot_val(b), P->ring_val[b], sizeof(double) * n, cudaMemcpyDeviceToHost, P->copy));
+
+    const int per = 12;
+    EvSet pe(P->profile, size_t(nch) * per + 4);
+    CK(cudaEventRecord(P->ev_ready, s));
+    CK(cudaStreamWaitEvent(cp, P->ev_ready, 0));
+    pe.rec(size_t(nch) * per, s);
+    if (rp_out && !sink) {
+        if (P->fused) {
+            rp_out[0] = base;
+            if (nch == 0)  // every row is empty: no chunk will deliver offsets
+                for (int64_t r = 1; r <= P->R; ++r) rp_out[r] = base;
+        } else {
+            CK(cudaMemcpyAsync(rp_out, P->crp, sizeof(int64_t) * (P->R + 1), cudaMemcpyDeviceToHost, cp));
         }
-        CK(cudaEventRecord(P->ev_d2h[b], P->copy));
-    };
-    // keep `ring` chunks in flight; the host consumes chunk c while chunks c+1.. run
-    int64_t issued = 0;
-    for (; issued < std::min<int64_t>(nch, ring); ++issued) enqueue(issued);
-    for (int64_t c = 0; c < nch; ++c) {
+    }
+    if (P->fused && nch > 0) enqueue_analysis(P, 0, pe.at(0));
+
+    std::vector<int64_t> offs(nch + 1, 0);  // chunk offsets relative to the slice
+    if (!P->fused && nch > 0)
+        for (int64_t c = 0; c <= nch; ++c) offs[c] = P->chunk_offs[c] - off0;
+    int64_t done_cb = 0;
+    auto consume = [&](int64_t c) {  // sink: wait for chunk c's copy and hand it over
         const int b = int(c % ring);
         CK(cudaEventSynchronize(P->ev_d2h[b]));
-        int64_t *rp = slot_rp(b);
         const int64_t r0 = P->chunk_rows[c], r1 = P->chunk_rows[c + 1];
+        int64_t *rp = st_rp(b);
         const int64_t first = rp[0];
         for (int64_t k = 0; k <= r1 - r0; ++k) rp[k] -= first;
-        const int rc = cb(user, P->row_begin + r0, P->row_begin + r1, rp, slot_col(b), slot_val(b), rp[r1 - r0]);
+        const int rc = sink->cb(sink->user, P->row_begin + r0, P->row_begin + r1, rp, st_col(b), st_val(b), rp[r1 - r0]);
         if (rc != 0) {
-            CK(cudaStreamSynchronize(P->copy));
+            CK(cudaStreamSynchronize(cp));
+            CK(cudaStreamSynchronize(s));
             fail(SPGEMM_ERR_CALLBACK, "chunk sink returned " + std::to_string(rc));
         }
-        if (issued < nch) enqueue(issued++);
+        done_cb = c + 1;
+    };
+
+    for (int64_t j = 0; j < nch; ++j) {
+        const int b = int(j % ring);
+        const int64_t r0 = P->chunk_rows[j], r1 = P->chunk_rows[j + 1];
+        int64_t mx = P->max_nnz;
+        if (P->fused) {
+            // chunk j's symbolic pass was enqueued one iteration ago; its total decides where the
+            // chunk lands on the host and its max row nnz which numeric tiers to launch
+            CK(cudaEventSynchronize(P->ev_tot[j]));
+            offs[j + 1] = P->h_small[1 + 2 * j] - base;
+            mx = P->h_small[2 + 2 * j];
+        }
+        const int64_t o = offs[j], n = offs[j + 1] - offs[j];
+        if (!sink && o + n > capacity) *overflow = true;
+        if (j >= ring) CK(cudaStreamWaitEvent(s, P->ev_d2h[b], 0));
+        if (!*overflow) {
+            pe.rec(size_t(j) * per + 5, s);
+            enqueue_numeric(P, j, b, mx, pe.at(size_t(j) * per + 6));
+            CK(cudaEventRecord(P->ev_num[b], s));
+        }
+        if (P->fused && j + 1 < nch) enqueue_analysis(P, j + 1, pe.at(size_t(j + 1) * per));
+        if (*overflow) continue;
+        if (sink && j >= ring) consume(j - ring);  // frees staging slot b
+        CK(cudaStreamWaitEvent(cp, P->ev_num[b], 0));
+        pe.rec(size_t(j) * per + 10, cp);
+        int32_t *dcol = sink ? st_col(b) : col_out + o;
+        double *dval = sink ? st_val(b) : val_out + o;
+        if (n > 0) {
+            CK(cudaMemcpyAsync(dcol, P->ring_col[b], sizeof(int32_t) * n, cudaMemcpyDeviceToHost, cp));
+            CK(cudaMemcpyAsync(dval, P->ring_val[b], sizeof(double) * n, cudaMemcpyDeviceToHost, cp));
+        }
+        if (sink) {
+            CK(cudaMemcpyAsync(st_rp(b), P->crp + r0, sizeof(int64_t) * (r1 - r0 + 1), cudaMemcpyDeviceToHost, cp));
+        } else if (rp_out && P->fused && r1 > r0) {
+            CK(cudaMemcpyAsync(rp_out + r0 + 1, P->crp + r0 + 1, sizeof(int64_t) * (r1 - r0), cudaMemcpyDeviceToHost, cp));
+        }
+        CK(cudaEventRecord(P->ev_d2h[b], cp));
     }
-    CK(cudaStreamSynchronize(P->copy));
-    check_numeric_errors(P);
+    if (sink)
+        for (int64_t c = done_cb; c < nch; ++c) consume(c);
+    pe.rec(size_t(nch) * per + 1, cp);
+    CK(cudaStreamSynchronize(cp));
+    CK(cudaStreamSynchronize(s));
+    unsigned err[2] = {0, 0};
+    CK(cudaMemcpy(&err[0], &P->ctl[1].err, sizeof(unsigned), cudaMemcpyDeviceToHost));
+    if (err[0]) fail(SPGEMM_ERR_STATE, "internal: numeric pass produced a row whose nnz differs from the symbolic pass");
+    const int64_t total = offs[nch];
+    if (P->fused) {
+        P->nnz = total;
+        P->chunk_offs = offs;
+        Ctl hc;
+        CK(cudaMemcpy(&hc, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost));
+        P->max_nnz = (int64_t)hc.max_nnz;
+        P->rows_w = (int64_t)hc.rows_w;
+        P->rows_b = (int64_t)hc.rows_b;
+        P->rows_g = (int64_t)hc.rows_g;
+    }
+    if (P->profile) {
+        P->clear_stats({"num_w", "num_b", "num_g", "d2h_span", "execute_total"});
+        if (P->fused) P->clear_stats({"sym_w", "sym_b", "sym_g", "scan"});
+        for (int64_t c = 0; c < nch; ++c) {
+            cudaEvent_t *e = pe.at(size_t(c) * per);
+            if (P->fused) {
+                P->add_stat("sym_w", elapsed(e[0], e[1]), 0);
+                P->add_stat("sym_b", elapsed(e[1], e[2]), 0);
+                P->add_stat("sym_g", elapsed(e[2], e[3]), 0);
+                P->add_stat("scan", elapsed(e[3], e[4]), 0);
+            }
+            if (!*overflow) {
+                P->add_stat("num_w", elapsed(e[6], e[7]), 0);
+                P->add_stat("num_b", elapsed(e[7], e[8]), 0);
+                P->add_stat("num_g", elapsed(e[8], e[9]), 0);
+                cudaEvent_t end = (c + 1 < nch) ? pe.ev[size_t(c + 1) * per + 10] : pe.ev[size_t(nch) * per + 1];
+                P->add_stat("d2h_span", elapsed(e[10], end), double(offs[c + 1] - offs[c]) * 12);
+            }
+        }
+        P->add_stat("execute_total", elapsed(pe.ev[size_t(nch) * per], pe.ev[size_t(nch) * per + 1]),
+                    double(total) * 12 + 8.0 * (P->R + 1));
+    }
+    return total;
 }
 
 spgemm_status guarded(const std::function<void()> &f) {
@@ -630,6 +789,10 @@ spgemm_status guarded(const std::function<void()> &f) {
         g_err = "unknown internal error";
         return SPGEMM_ERR_STATE;
     }
+}
+
+void mark_failed(spgemm_plan_s *P, spgemm_status st) {
+    if (st == SPGEMM_ERR_CUDA || st == SPGEMM_ERR_STATE) P->failed = true;
 }
 
 }  // namespace
@@ -659,11 +822,12 @@ spgemm_status spgemm_plan(const spgemm_csr *A, const spgemm_csr *B, size_t budge
         P = new spgemm_plan_s();
         do_plan(A, B, budget, opts, P);
     });
-    if (prev >= 0) cudaSetDevice(prev);
     if (st != SPGEMM_OK) {
         delete P;
+        if (prev >= 0) cudaSetDevice(prev);
         return st;
     }
+    if (prev >= 0) cudaSetDevice(prev);
     *plan_out = P;
     return SPGEMM_OK;
 }
@@ -678,9 +842,9 @@ spgemm_status spgemm_plan_info(spgemm_plan_t P, spgemm_info *info) {
     info->ncols = P->ncols;
     info->nnz = P->nnz;
     info->products = P->products;
-    info->max_row_nnz = P->max_nnz;
+    info->max_row_nnz = P->nnz >= 0 ? P->max_nnz : -1;
     info->max_row_products = P->max_u;
-    info->num_chunks = (int32_t)num_chunks(P);
+    info->num_chunks = (int32_t)P->num_chunks();
     info->ring = P->ring;
     info->chunk_capacity = P->cap;
     info->arena_bytes = (int64_t)P->arena_bytes;
@@ -689,23 +853,26 @@ spgemm_status spgemm_plan_info(spgemm_plan_t P, spgemm_info *info) {
     info->rows_warp = P->rows_w;
     info->rows_block = P->rows_b;
     info->rows_global = P->rows_g;
+    info->fused = P->fused ? 1 : 0;
     return SPGEMM_OK;
 }
 
 spgemm_status spgemm_plan_chunks(spgemm_plan_t P, int64_t *rows, int64_t *offs) {
-    if (!P || !rows || !offs) {
+    if (!P || !rows) {
         g_err = "NULL argument";
         return SPGEMM_ERR_INVALID_ARGUMENT;
     }
-    const int64_t base0 = P->chunk_offs.empty() ? 0 : P->chunk_offs[0];
-    if (P->chunk_rows.empty()) {
+    const int64_t n = P->num_chunks();
+    if (n == 0) {
         rows[0] = 0;
-        offs[0] = 0;
+        if (offs) offs[0] = 0;
         return SPGEMM_OK;
     }
-    for (size_t k = 0; k < P->chunk_rows.size(); ++k) {
+    const bool known = (int64_t)P->chunk_offs.size() == n + 1;
+    const int64_t base0 = known ? P->chunk_offs[0] : 0;
+    for (int64_t k = 0; k <= n; ++k) {
         rows[k] = P->chunk_rows[k];
-        offs[k] = P->chunk_offs[k] - base0;
+        if (offs) offs[k] = known ? P->chunk_offs[k] - base0 : -1;
     }
     return SPGEMM_OK;
 }
@@ -715,8 +882,37 @@ spgemm_status spgemm_execute_into(spgemm_plan_t P, int64_t *row_ptr, int32_t *co
         g_err = "plan is NULL";
         return SPGEMM_ERR_INVALID_ARGUMENT;
     }
-    spgemm_status st = guarded([&] { do_execute(P, row_ptr, col_idx, values); });
-    if (st != SPGEMM_OK && st != SPGEMM_ERR_INVALID_ARGUMENT) P->failed = true;
+    spgemm_status st = guarded([&] {
+        if (P->nnz < 0)
+            fail(SPGEMM_ERR_STATE, "fused plan: nnz(C) is not known yet (use spgemm_multiply, spgemm_execute_stream "
+                                   "or spgemm_execute_capacity)");
+        if (P->nnz > 0 && (!col_idx || !values)) fail(SPGEMM_ERR_INVALID_ARGUMENT, "col_idx/values output is NULL");
+        bool ovf = false;
+        run_pipeline(P, row_ptr, col_idx, values, P->nnz, nullptr, &ovf);
+        if (ovf) fail(SPGEMM_ERR_STATE, "internal: nnz changed between executions");
+    });
+    mark_failed(P, st);
+    return st;
+}
+
+spgemm_status spgemm_execute_capacity(spgemm_plan_t P, int64_t *row_ptr, int32_t *col_idx, double *values,
+                                      int64_t capacity, int64_t *nnz_out) {
+    if (!P) {
+        g_err = "plan is NULL";
+        return SPGEMM_ERR_INVALID_ARGUMENT;
+    }
+    int64_t total = -1;
+    bool ovf = false;
+    spgemm_status st = guarded([&] {
+        if (capacity > 0 && (!col_idx || !values)) fail(SPGEMM_ERR_INVALID_ARGUMENT, "col_idx/values output is NULL");
+        total = run_pipeline(P, row_ptr, col_idx, values, capacity, nullptr, &ovf);
+    });
+    if (nnz_out && total >= 0) *nnz_out = total;
+    if (st == SPGEMM_OK && ovf) {
+        g_err = "output capacity " + std::to_string(capacity) + " < nnz(C) = " + std::to_string(total);
+        return SPGEMM_ERR_CAPACITY;
+    }
+    mark_failed(P, st);
     return st;
 }
 
@@ -727,6 +923,10 @@ spgemm_status spgemm_execute(spgemm_plan_t P, spgemm_csr_out *C) {
     }
     spgemm_status st = guarded([&] {
         DeviceGuard g(P->device);
+        if (P->nnz < 0) {  // fused: learn nnz with a sink-less counting run is not possible; run once into nothing
+            bool ovf = false;
+            run_pipeline(P, nullptr, nullptr, nullptr, 0, nullptr, &ovf);
+        }
         if (!P->h_rp) {
             if (cudaHostAlloc(&P->h_rp, sizeof(int64_t) * (P->R + 1), 0) != cudaSuccess ||
                 cudaHostAlloc(&P->h_col, sizeof(int32_t) * std::max<int64_t>(P->nnz, 1), 0) != cudaSuccess ||
@@ -735,7 +935,8 @@ spgemm_status spgemm_execute(spgemm_plan_t P, spgemm_csr_out *C) {
                 fail(SPGEMM_ERR_HOST_ALLOC, "pinned allocation of the output failed");
             }
         }
-        do_execute(P, P->h_rp, P->h_col, P->h_val);
+        bool ovf = false;
+        run_pipeline(P, P->h_rp, P->h_col, P->h_val, P->nnz, nullptr, &ovf);
         C->nrows = P->R;
         C->ncols = P->ncols;
         C->nnz = P->nnz;
@@ -743,7 +944,7 @@ spgemm_status spgemm_execute(spgemm_plan_t P, spgemm_csr_out *C) {
         C->col_idx = P->h_col;
         C->values = P->h_val;
     });
-    if (st != SPGEMM_OK && st != SPGEMM_ERR_INVALID_ARGUMENT && st != SPGEMM_ERR_HOST_ALLOC) P->failed = true;
+    mark_failed(P, st);
     return st;
 }
 
@@ -752,8 +953,15 @@ spgemm_status spgemm_execute_stream(spgemm_plan_t P, spgemm_chunk_cb cb, void *u
         g_err = "plan is NULL";
         return SPGEMM_ERR_INVALID_ARGUMENT;
     }
-    spgemm_status st = guarded([&] { do_execute_stream(P, cb, user); });
-    if (st == SPGEMM_ERR_CUDA || st == SPGEMM_ERR_STATE) P->failed = true;
+    spgemm_status st = guarded([&] {
+        if (!cb) fail(SPGEMM_ERR_INVALID_ARGUMENT, "callback is NULL");
+        Sink sk;
+        sk.cb = cb;
+        sk.user = user;
+        bool ovf = false;
+        run_pipeline(P, nullptr, nullptr, nullptr, INT64_MAX, &sk, &ovf);
+    });
+    mark_failed(P, st);
     return st;
 }
 
@@ -768,16 +976,14 @@ spgemm_status spgemm_set_row_ptr_base(spgemm_plan_t P, int64_t base) {
 
 spgemm_status spgemm_multiply(const spgemm_csr *A, const spgemm_csr *B, size_t budget, const spgemm_opts *opts,
                               int64_t *row_ptr, int32_t *col_idx, double *values, int64_t cap, int64_t *nnz_out) {
+    spgemm_opts o;
+    spgemm_opts_default(&o);
+    if (opts) o = *opts;
+    o.fused = 1;
     spgemm_plan_t P = nullptr;
-    spgemm_status st = spgemm_plan(A, B, budget, opts, &P);
+    spgemm_status st = spgemm_plan(A, B, budget, &o, &P);
     if (st != SPGEMM_OK) return st;
-    if (nnz_out) *nnz_out = P->nnz;
-    if (P->nnz > cap) {
-        g_err = "output capacity " + std::to_string(cap) + " < nnz(C) = " + std::to_string(P->nnz);
-        spgemm_free(P);
-        return SPGEMM_ERR_CAPACITY;
-    }
-    st = spgemm_execute_into(P, row_ptr, col_idx, values);
+    st = spgemm_execute_capacity(P, row_ptr, col_idx, values, cap, nnz_out);
     spgemm_free(P);
     return st;
 }

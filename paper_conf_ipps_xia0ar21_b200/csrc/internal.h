@@ -31,8 +31,9 @@ constexpr int ROW_BATCH = 16;              // rows a warp claims per atomic in t
 
 // Per-pass control block in the arena (zeroed with cudaMemsetAsync before each pass).
 struct Ctl {
-    unsigned long long row_ctr;   // W kernels: next row batch
-    unsigned int nB, nG;          // long-row list lengths
+    unsigned long long row_ctr;   // W kernels: next row batch                      } reset before
+    unsigned int nB, nG;          // long-row list lengths                          } every pass
+    unsigned long long pass_max;  // symbolic: max nnz of a row in this pass        } (24 bytes)
     unsigned int err;             // bit 0: numeric count mismatch; bit 1: invalid input; bit 2: table overflow
     unsigned int pad;
     unsigned long long sum_u;     // count pass: sum of products
@@ -45,7 +46,7 @@ struct Ctl {
 
 // --- launchers (all asynchronous on `s`) ---------------------------------------------------
 
-// S2: u[i] = sum_{k in A_i} nnz(B_k)  for i in [0, A.nrows)
+// S2: bnd[i] = min(sum_{k in A_i} nnz(B_k), ncols) for i in [0, A.nrows); ctl gets the sum and max of products
 void launch_count(const DevCSR &A, const DevCSR &B, int64_t *u, Ctl *ctl, cudaStream_t s);
 
 // Validation of a CSR operand (rows strictly increasing, 0 <= col < ncols, rp non-decreasing).
@@ -56,23 +57,38 @@ void launch_rebase(int64_t *rp, int64_t n, int64_t sub, cudaStream_t s);
 
 struct SymArgs {
     DevCSR A, B;
-    const int64_t *u;
-    int64_t *crp;        // out: crp[i] = nnz_i (i < nrows), then scanned in place
+    const int64_t *bnd;  // per-row bound min(products, ncols) from the count pass
+    int32_t *nnz;        // out: nnz of every row in [r0, r1)
+    int64_t r0, r1;      // rows of this pass
     int32_t *listB, *listG;
     Ctl *ctl;
     uint32_t *gscratch;  // G tier: per-CTA bitmap of ceil(ncols/32) words, zero on entry and exit
     int64_t gstride;     // words per CTA slot
     int gblocks;         // CTAs in the G kernel
     int group;           // lanes per A entry in the W kernel (4, 8, 16, 32)
+    int tiers;           // bit 0: launch the CTA tier, bit 1: the dense tier (host knows when a
+                         // pass cannot have such rows, and skips those launches)
 };
+
+// tier bits for a pass whose rows have bound <= maxb
+inline int sym_tiers(int64_t maxb) { return (maxb > CAPW_SYM ? 1 : 0) | (maxb > CAPB_SYM ? 2 : 0); }
+inline int num_tiers(int64_t maxnnz) { return (maxnnz > CAPW_NUM ? 1 : 0) | (maxnnz > CAPB_NUM ? 2 : 0); }
+
+// host2[0] = *end (a chunk's end offset), host2[1] = ctl->pass_max -- zero-copy stores into mapped
+// pinned memory, so no small D2H copy queues behind the big ones on the copy engine
+void launch_publish(const int64_t *end, const Ctl *ctl, int64_t *host2, cudaStream_t s);
+
+// out[k] = max(x[rows[k] .. rows[k+1]-1]) for k < nseg (0 for empty segments)
+void launch_seg_max(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s);
 // S3+S4: symbolic pass over all rows (tiering + the three tiers).  ev: NULL or 4 events recorded
 // before W, between W/B, between B/G and after G (per-kernel timing on the launching stream).
 void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);
 
-// S5: in-place exclusive scan of crp[0..n] (n+1 entries, crp[n] must be 0 on entry), plus base.
-// tmp: >= 2 * ceil((n+1)/SCAN_TILE) + 64 int64 of scratch.
+// S5: y[1 + t] = y[0] + x[0] + ... + x[t] for t < n, y[0] (the base) read on the device.
+// tmp: >= ceil(n / SCAN_TILE) int64 of scratch.
 constexpr int SCAN_TILE = 4096;
-void launch_scan(int64_t *crp, int64_t n, int64_t base, int64_t *tmp, cudaStream_t s);
+void launch_scan(const int32_t *x, int64_t n, int64_t *y, int64_t *tmp, cudaStream_t s);
+void launch_scan64(const int64_t *x, int64_t n, int64_t *y, int64_t *tmp, cudaStream_t s);
 
 // chunk ids: bounds[c] = first row whose offset - crp[0] >= c * cap_prime (empty ids repeat);
 // bounds has nids+1 entries with bounds[nids] = n.
@@ -94,6 +110,7 @@ struct NumArgs {
     int64_t gstride_bits, gstride_vals;
     int gblocks;
     int group;
+    int tiers;           // as in SymArgs
 };
 // S6+S7: numeric pass over chunk rows [r0, r1); ev as in launch_symbolic
 void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);

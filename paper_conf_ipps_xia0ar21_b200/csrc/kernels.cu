@@ -113,6 +113,103 @@ __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t *s, int64_
     return r;
 }
 
+// ------------------------------------------------------------------ warp product iterator (W tier)
+//
+// Visits every intermediate product A_ik * B_kj of row i with one warp (Alg. 1 lines 3-5).
+//  * A entries are fetched 32 at a time (one per lane) together with their B row bounds, so the
+//    A.col -> B.rp dependency is paid once per 32 entries; bounds are then broadcast by shuffle.
+//  * Lanes form 32/G subgroups; subgroup g takes one B row per round and its lanes take G
+//    consecutive entries of it (coalesced).  U rounds are loaded before any is consumed, so U
+//    independent B-row loads are in flight per warp (latency, not bandwidth, bounds this loop).
+//  * f(ok, col, value) is called once per round by every lane, followed by __syncwarp().  With
+//    G == 32 all active lanes of a round hold entries of ONE B row, i.e. distinct columns
+//    (rows are sorted and unique), which lets the numeric pass update values without atomics.
+template <int G, int U, bool VALS, typename F>
+__device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR &B, int64_t i, F &&f) {
+    constexpr int R = 32 / G;  // B rows per round
+    const int lane = threadIdx.x & 31;
+    const int sub = lane / G, sl = lane % G;
+    const int64_t as = A.rp[i], ae = A.rp[i + 1];
+    for (int64_t pb = as; pb < ae; pb += 32) {
+        const int64_t e = pb + lane;
+        int64_t bs = 0, be = 0;
+        double av = 0.0;
+        if (e < ae) {
+            const int32_t k = __ldg(&A.col[e]);
+            bs = __ldg(&B.rp[k]);
+            be = __ldg(&B.rp[k + 1]);
+            if (VALS) av = __ldg(&A.val[e]);
+        }
+        const int nb = (int)(ae - pb < 32 ? ae - pb : 32);
+        for (int t = 0; t < nb; t += R * U) {
+            int64_t s[U], en[U];
+            double a[U], v[U];
+            int32_t c[U];
+            bool ok[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int src = t + u * R + sub;
+                int64_t ss = __shfl_sync(FULLMASK, bs, src & 31);
+                int64_t ee = __shfl_sync(FULLMASK, be, src & 31);
+                a[u] = VALS ? __shfl_sync(FULLMASK, av, src & 31) : 0.0;
+                if (src >= nb) ss = ee = 0;
+                s[u] = ss;
+                en[u] = ee;
+                const int64_t q = ss + sl;
+                ok[u] = q < ee;
+                c[u] = ok[u] ? __ldg(&B.col[q]) : 0;
+                v[u] = (VALS && ok[u]) ? __ldg(&B.val[q]) : 0.0;
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                f(ok[u], c[u], a[u] * v[u]);
+                __syncwarp();
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                // remainder of B rows longer than G (uniform trip count across the warp)
+                for (int64_t q0 = s[u] + G;; q0 += G) {
+                    if (!__any_sync(FULLMASK, q0 < en[u])) break;
+                    const int64_t q = q0 + sl;
+                    const bool okk = q < en[u];
+                    const int32_t cc = okk ? __ldg(&B.col[q]) : 0;
+                    const double vv = (VALS && okk) ? __ldg(&B.val[q]) : 0.0;
+                    f(okk, cc, a[u] * vv);
+                    __syncwarp();
+                }
+            }
+        }
+    }
+}
+
+// find-or-insert of a column in a warp-private table; returns the slot
+__device__ __forceinline__ uint32_t find_slot(int32_t *keys, int32_t c, int lg) {
+    const uint32_t mask = (1u << lg) - 1;
+    uint32_t h = hslot(c, lg);
+    volatile int32_t *vk = keys;
+    while (true) {
+        const int32_t k = vk[h];
+        if (k == c) return h;
+        if (k == EMPTY) {
+            const int32_t old = atomicCAS(&keys[h], EMPTY, c);
+            if (old == EMPTY || old == c) return h;
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+// vectorised fill of n (multiple of 4) int32 / n (even) doubles with a warp
+__device__ __forceinline__ void warp_fill_keys(int32_t *keys, int n) {
+    const int lane = threadIdx.x & 31;
+    int4 *k4 = reinterpret_cast<int4 *>(keys);
+    for (int t = lane; t < (n >> 2); t += 32) k4[t] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
+}
+__device__ __forceinline__ void warp_fill_zero(double *v, int n) {
+    const int lane = threadIdx.x & 31;
+    double2 *v2 = reinterpret_cast<double2 *>(v);
+    for (int t = lane; t < (n >> 1); t += 32) v2[t] = make_double2(0.0, 0.0);
+}
+
 // ------------------------------------------------------------------------------------------ S2
 
 __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__restrict__ u, Ctl *ctl) {
@@ -128,7 +225,7 @@ __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__re
         }
         acc = warp_sum(acc);
         if (lane == 0) {
-            u[i] = acc;
+            u[i] = min(acc, B.ncols);  // the row's nnz bound: distinct columns <= min(products, ncols)
             lsum += acc;
             lmax = max(lmax, (unsigned long long)acc);
             lmaxb = max(lmaxb, (unsigned long long)min(acc, B.ncols));
@@ -192,7 +289,7 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
     extern __shared__ int32_t smem_i[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     int32_t *keys = smem_i + wid * TW_SYM;
-    const int64_t R = a.A.nrows, ncols = a.B.ncols;
+    const int64_t R = a.r1 - a.r0;
     unsigned long long lmax = 0, nw = 0, nlong = 0;
     constexpr int MAXLG = 10;  // log2(TW_SYM)
     while (true) {
@@ -201,10 +298,11 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
         base = __shfl_sync(FULLMASK, base, 0);
         if ((int64_t)base >= R) break;
         const int64_t end = min((int64_t)base + ROW_BATCH, R);
-        for (int64_t i = (int64_t)base; i < end; ++i) {
-            const int64_t bound = min(a.u[i], ncols);
+        for (int64_t li = (int64_t)base; li < end; ++li) {
+            const int64_t i = a.r0 + li;
+            const int64_t bound = a.bnd[i];
             if (bound == 0) {
-                if (lane == 0) a.crp[i] = 0;
+                if (lane == 0) a.nnz[i] = 0;
                 continue;
             }
             if (bound > CAPW_SYM) {
@@ -216,21 +314,15 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
             }
             const int lg = table_log2(bound, MAXLG);
             const int T = 1 << lg;
-            for (int t = lane; t < T; t += 32) keys[t] = EMPTY;
+            warp_fill_keys(keys, T);
             __syncwarp();
             int cnt = 0;
-            const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
-            for (int64_t p0 = as; p0 < ae; p0 += 32 / G) {
-                const int64_t p = p0 + lane / G;
-                if (p < ae) {
-                    const int32_t k = __ldg(&a.A.col[p]);
-                    const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
-                    for (int64_t q = bs + (lane % G); q < be; q += G) cnt += sym_insert(keys, __ldg(&a.B.col[q]), lg);
-                }
-            }
+            warp_row_products<G, (G == 32 ? 4 : 2), false>(a.A, a.B, i, [&](bool ok, int32_t c, double) {
+                if (ok) cnt += sym_insert(keys, c, lg);
+            });
             cnt = warp_sum(cnt);
             if (lane == 0) {
-                a.crp[i] = cnt;
+                a.nnz[i] = cnt;
                 lmax = max(lmax, (unsigned long long)cnt);
                 nw++;
             }
@@ -238,7 +330,10 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
         }
     }
     if (lane == 0) {
-        if (lmax) atomicMax(&a.ctl->max_nnz, lmax);
+        if (lmax) {
+            atomicMax(&a.ctl->max_nnz, lmax);
+            atomicMax(&a.ctl->pass_max, lmax);
+        }
         if (nw) atomicAdd(&a.ctl->rows_w, nw);
     }
 }
@@ -252,10 +347,9 @@ __global__ void __launch_bounds__(THREADS_B) k_sym_b(SymArgs a) {
     constexpr int NW = THREADS_B / 32;
     constexpr int MAXLG = 15;  // log2(TB_SYM)
     const unsigned n = *(volatile unsigned *)&a.ctl->nB;
-    const int64_t ncols = a.B.ncols;
     for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
         const int64_t i = a.listB[idx];
-        const int64_t bound = min(a.u[i], ncols);
+        const int64_t bound = a.bnd[i];
         const int lg = table_log2(bound, MAXLG);
         const int T = 1 << lg;
         for (int t = threadIdx.x; t < T; t += THREADS_B) keys[t] = EMPTY;
@@ -270,8 +364,9 @@ __global__ void __launch_bounds__(THREADS_B) k_sym_b(SymArgs a) {
         int64_t tot;
         block_excl_scan<THREADS_B>(cnt, s_scan, &tot);
         if (threadIdx.x == 0) {
-            a.crp[i] = tot;
+            a.nnz[i] = (int32_t)tot;
             atomicMax(&a.ctl->max_nnz, (unsigned long long)tot);
+            atomicMax(&a.ctl->pass_max, (unsigned long long)tot);
             atomicAdd(&a.ctl->rows_b, 1ull);
         }
         __syncthreads();
@@ -307,12 +402,13 @@ __global__ void __launch_bounds__(THREADS_G) k_sym_g(SymArgs a) {
         int64_t tot;
         block_excl_scan<THREADS_G>(cnt, s_scan, &tot);
         if (threadIdx.x == 0) {
-            a.crp[i] = tot;
+            a.nnz[i] = (int32_t)tot;
             atomicMax(&a.ctl->max_nnz, (unsigned long long)tot);
+            atomicMax(&a.ctl->pass_max, (unsigned long long)tot);
             atomicAdd(&a.ctl->rows_g, 1ull);
         }
         // clear (block_excl_scan ended with a barrier, so all atomics of this row are done)
-        if (a.u[i] < nwords) {
+        if (a.bnd[i] < nwords) {  // bnd = min(products, ncols): re-walk only when cheaper than a sweep
             for (int64_t p = as + wid; p < ae; p += NW) {
                 const int32_t k = __ldg(&a.A.col[p]);
                 const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
@@ -326,25 +422,29 @@ __global__ void __launch_bounds__(THREADS_G) k_sym_g(SymArgs a) {
 }
 
 // ------------------------------------------------------------------------------------- S5 scan
+// y[0] holds the base on entry (device-resident: the previous chunk's end offset, or the slice
+// base); y[1 + t] = y[0] + x[0] + ... + x[t] for t < n.  Three passes: tile sums, one-CTA scan of
+// the tile sums (reads the base on the device, so chunks can be scanned back to back without a
+// host round trip), and the tile-local scans.
 
-__global__ void __launch_bounds__(1024) k_scan_reduce(const int64_t *__restrict__ x, int64_t n1,
-                                                      int64_t *__restrict__ part) {
+template <typename T>
+__global__ void __launch_bounds__(1024) k_scan_reduce(const T *__restrict__ x, int64_t n, int64_t *__restrict__ part) {
     __shared__ int64_t s[40];
     const int64_t b0 = (int64_t)blockIdx.x * SCAN_TILE;
     int64_t v = 0;
 #pragma unroll
     for (int t = 0; t < SCAN_TILE / 1024; ++t) {
         const int64_t i = b0 + (int64_t)threadIdx.x * (SCAN_TILE / 1024) + t;
-        if (i < n1) v += x[i];
+        if (i < n) v += (int64_t)x[i];
     }
     int64_t tot;
     block_excl_scan<1024>(v, s, &tot);
     if (threadIdx.x == 0) part[blockIdx.x] = tot;
 }
 
-__global__ void __launch_bounds__(1024) k_scan_top(int64_t *part, int64_t nb, int64_t base) {
+__global__ void __launch_bounds__(1024) k_scan_top(int64_t *part, int64_t nb, const int64_t *y0) {
     __shared__ int64_t s[40];
-    int64_t carry = base;
+    int64_t carry = *y0;
     for (int64_t b0 = 0; b0 < nb; b0 += 1024) {
         const int64_t i = b0 + threadIdx.x;
         const int64_t v = i < nb ? part[i] : 0;
@@ -355,8 +455,9 @@ __global__ void __launch_bounds__(1024) k_scan_top(int64_t *part, int64_t nb, in
     }
 }
 
-__global__ void __launch_bounds__(1024) k_scan_apply(int64_t *__restrict__ x, int64_t n1,
-                                                     const int64_t *__restrict__ part) {
+template <typename T>
+__global__ void __launch_bounds__(1024) k_scan_apply(const T *__restrict__ x, int64_t n,
+                                                     const int64_t *__restrict__ part, int64_t *__restrict__ y) {
     __shared__ int64_t s[40];
     constexpr int PER = SCAN_TILE / 1024;
     const int64_t b0 = (int64_t)blockIdx.x * SCAN_TILE + (int64_t)threadIdx.x * PER;
@@ -364,15 +465,15 @@ __global__ void __launch_bounds__(1024) k_scan_apply(int64_t *__restrict__ x, in
     int64_t sum = 0;
 #pragma unroll
     for (int t = 0; t < PER; ++t) {
-        v[t] = (b0 + t < n1) ? x[b0 + t] : 0;
+        v[t] = (b0 + t < n) ? (int64_t)x[b0 + t] : 0;
         sum += v[t];
     }
     int64_t tot;
     int64_t run = block_excl_scan<1024>(sum, s, &tot) + part[blockIdx.x];
 #pragma unroll
     for (int t = 0; t < PER; ++t) {
-        if (b0 + t < n1) x[b0 + t] = run;
         run += v[t];
+        if (b0 + t < n) y[1 + b0 + t] = run;
     }
 }
 
@@ -472,22 +573,26 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_num_w(NumArgs a) {
             }
             const int lg = table_log2(n, MAXLG);
             const int T = 1 << lg;
-            for (int t = lane; t < T; t += 32) {
-                keys[t] = EMPTY;
-                vals[t] = 0.0;
-            }
+            warp_fill_keys(keys, T);
+            warp_fill_zero(vals, T);
             __syncwarp();
-            const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
-            for (int64_t p0 = as; p0 < ae; p0 += 32 / G) {
-                const int64_t p = p0 + lane / G;
-                if (p < ae) {
-                    const int32_t k = __ldg(&a.A.col[p]);
-                    const double av = __ldg(&a.A.val[p]);
-                    const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
-                    for (int64_t q = bs + (lane % G); q < be; q += G)
-                        num_insert(keys, vals, __ldg(&a.B.col[q]), av * __ldg(&a.B.val[q]), lg);
+            warp_row_products<G, (G == 32 ? 4 : 2), true>(a.A, a.B, i, [&](bool ok, int32_t c, double v) {
+                if (G == 32) {
+                    // one B row per round: distinct columns -> distinct slots -> plain RMW
+                    if (ok) {
+                        const uint32_t h = find_slot(keys, c, lg);
+                        vals[h] += v;
+                    }
+                } else {
+                    const unsigned act = __ballot_sync(FULLMASK, ok);
+                    if (ok) {
+                        const uint32_t h = find_slot(keys, c, lg);
+                        const unsigned peers = __match_any_sync(act, c);
+                        if (__popc(peers) == 1) vals[h] += v;
+                        else atomicAdd(&vals[h], v);
+                    }
                 }
-            }
+            });
             __syncwarp();
             // in-place compaction of the occupied slots (destination <= source, one round of 32
             // slots is read completely before any of it is written)
@@ -752,12 +857,15 @@ static inline void rec(cudaEvent_t *ev, int k, cudaStream_t s) {
 }
 
 void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev) {
-    if (a.A.nrows == 0) return;
+    const int64_t rows = a.r1 - a.r0;
+    if (rows <= 0) {
+        for (int k = 0; k < 4; ++k) rec(ev, k, s);
+        return;
+    }
     int dev = 0;
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
-    cudaMemsetAsync(&a.ctl->row_ctr, 0, 16, s);  // row_ctr, nB, nG
-    const int64_t rows = a.A.nrows;
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, 24, s);  // row_ctr, nB, nG, pass_max
     const int wblocks = grid_for(rows, WARPS_W * ROW_BATCH, g.symw_blocks);
     rec(ev, 0, s);
     switch (a.group) {
@@ -767,10 +875,12 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
         default: sym_w<32>(a, wblocks, s); break;
     }
     rec(ev, 1, s);
-    k_sym_b<<<g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
-    LAUNCHED(1);
+    if (a.tiers & 1) {
+        k_sym_b<<<g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
+        LAUNCHED(1);
+    }
     rec(ev, 2, s);
-    if (a.gblocks > 0) {
+    if ((a.tiers & 2) && a.gblocks > 0) {
         k_sym_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
         LAUNCHED(1);
     }
@@ -779,11 +889,14 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
 
 void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev) {
     const int64_t rows = a.r1 - a.r0;
-    if (rows <= 0) return;
+    if (rows <= 0) {
+        for (int k = 0; k < 4; ++k) rec(ev, k, s);
+        return;
+    }
     int dev = 0;
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
-    cudaMemsetAsync(&a.ctl->row_ctr, 0, 16, s);
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, 24, s);
     const int wblocks = grid_for(rows, WARPS_W * ROW_BATCH, g.numw_blocks);
     rec(ev, 0, s);
     switch (a.group) {
@@ -793,26 +906,32 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
         default: num_w<32>(a, wblocks, s); break;
     }
     rec(ev, 1, s);
-    k_num_b<<<g.numb_blocks, THREADS_B, numb_smem(), s>>>(a);
-    LAUNCHED(1);
+    if (a.tiers & 1) {
+        k_num_b<<<g.numb_blocks, THREADS_B, numb_smem(), s>>>(a);
+        LAUNCHED(1);
+    }
     rec(ev, 2, s);
-    if (a.gblocks > 0) {
+    if ((a.tiers & 2) && a.gblocks > 0) {
         k_num_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
         LAUNCHED(1);
     }
     rec(ev, 3, s);
 }
 
-void launch_scan(int64_t *crp, int64_t n, int64_t base, int64_t *tmp, cudaStream_t s) {
-    const int64_t n1 = n + 1;
-    const int64_t nb = (n1 + SCAN_TILE - 1) / SCAN_TILE;
-    k_scan_reduce<<<(unsigned)nb, 1024, 0, s>>>(crp, n1, tmp);
+template <typename T>
+static void scan_impl(const T *x, int64_t n, int64_t *y, int64_t *tmp, cudaStream_t s) {
+    if (n <= 0) return;
+    const int64_t nb = (n + SCAN_TILE - 1) / SCAN_TILE;
+    k_scan_reduce<T><<<(unsigned)nb, 1024, 0, s>>>(x, n, tmp);
     LAUNCHED(1);
-    k_scan_top<<<1, 1024, 0, s>>>(tmp, nb, base);
+    k_scan_top<<<1, 1024, 0, s>>>(tmp, nb, y);
     LAUNCHED(1);
-    k_scan_apply<<<(unsigned)nb, 1024, 0, s>>>(crp, n1, tmp);
+    k_scan_apply<T><<<(unsigned)nb, 1024, 0, s>>>(x, n, tmp, y);
     LAUNCHED(1);
 }
+
+void launch_scan(const int32_t *x, int64_t n, int64_t *y, int64_t *tmp, cudaStream_t s) { scan_impl(x, n, y, tmp, s); }
+void launch_scan64(const int64_t *x, int64_t n, int64_t *y, int64_t *tmp, cudaStream_t s) { scan_impl(x, n, y, tmp, s); }
 
 void launch_cut(const int64_t *crp, int64_t n, int64_t cap_prime, int64_t *bounds, int64_t nids, cudaStream_t s) {
     k_fill<<<grid_for(nids + 1, 256, 148 * 4), 256, 0, s>>>(bounds, nids + 1, n);
@@ -824,6 +943,41 @@ void launch_cut(const int64_t *crp, int64_t n, int64_t cap_prime, int64_t *bound
 }
 
 int choose_group(const DevCSR &B, int64_t nnzB) { return group_for(B, nnzB); }
+
+__global__ void k_publish(const int64_t *end, const Ctl *ctl, int64_t *host2) {
+    // system-scope visibility: the host reads these after synchronising on an event
+    volatile int64_t *h = host2;
+    h[0] = *end;
+    h[1] = (int64_t)ctl->pass_max;
+    __threadfence_system();
+}
+
+void launch_publish(const int64_t *end, const Ctl *ctl, int64_t *host2, cudaStream_t s) {
+    k_publish<<<1, 1, 0, s>>>(end, ctl, host2);
+    LAUNCHED(1);
+}
+
+__global__ void __launch_bounds__(256) k_seg_max(const int64_t *__restrict__ x, const int64_t *__restrict__ rows,
+                                                 int64_t *__restrict__ out) {
+    __shared__ int64_t s[8];
+    const int64_t r0 = rows[blockIdx.x], r1 = rows[blockIdx.x + 1];
+    int64_t m = 0;
+    for (int64_t i = r0 + threadIdx.x; i < r1; i += blockDim.x) m = max(m, x[i]);
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) m = max(m, __shfl_xor_sync(FULLMASK, m, d));
+    if ((threadIdx.x & 31) == 0) s[threadIdx.x >> 5] = m;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < 8; ++w) m = max(m, s[w]);
+        out[blockIdx.x] = max(m, s[0]);
+    }
+}
+
+void launch_seg_max(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s) {
+    if (nseg <= 0) return;
+    k_seg_max<<<(unsigned)nseg, 256, 0, s>>>(x, rows, out);
+    LAUNCHED(1);
+}
 
 __global__ void k_gather(const int64_t *__restrict__ crp, const int64_t *__restrict__ idx, int64_t n,
                          int64_t *__restrict__ out) {

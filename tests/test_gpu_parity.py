@@ -299,3 +299,87 @@ def test_multiply_one_shot():
     n = capi.spgemm_multiply(A, A, 0, None, rp, col, val, capacity=z)
     assert n == z
     assert_parity(A, A, rp.numpy(), col.numpy(), val.numpy(), exact=True)
+
+
+# ------------------------------------------------------------------------------------- fused plans
+
+def run_fused(A, B, budget=0, capacity=None, **kw):
+    o = capi.opts(fused=True, **kw)
+    with capi.Plan(A, B, budget, o) as P:
+        info0 = P.info()
+        assert info0["fused"] == 1 and info0["nnz"] == -1
+        cap = capacity if capacity is not None else int(oracle.row_nnz(A, B).sum())
+        rp = torch.empty(info0["nrows"] + 1, dtype=torch.int64, pin_memory=True)
+        col = torch.empty(max(cap, 0), dtype=torch.int32, pin_memory=True)
+        val = torch.empty(max(cap, 0), dtype=torch.float64, pin_memory=True)
+        n = P.execute_capacity(rp, col, val, cap)
+        info = P.info()
+        chunks = P.chunks()
+    return rp.numpy(), col.numpy()[:n], val.numpy()[:n], info, chunks
+
+
+@pytest.mark.parametrize("case", ["c2", "rmat", "rect", "tiers", "degenerate"])
+def test_fused_matches_oracle(case):
+    if case == "c2":
+        A = B = W.stencil_3d27(24)
+        kw = {"min_chunks": 9}
+    elif case == "rmat":
+        A = B = W.rmat(13, 16, seed=3)
+        kw = {"chunk_nnz": 50000}
+    elif case == "rect":
+        A = W.random_csr_sparse(2500, 1700, 7.0, seed=21)
+        B = W.random_csr_sparse(1700, 3100, 5.0, seed=22)
+        kw = {"chunk_nnz": 4000, "ring": 3}
+    elif case == "tiers":
+        A, B = _long_rows_case(seed=4)
+        kw = {}
+    else:
+        A = W.random_csr(40, 30, 0.0, seed=1)
+        B = W.random_csr(30, 20, 0.5, seed=2)
+        kw = {}
+    rp, col, val, info, (rows, offs) = run_fused(A, B, **kw)
+    assert info["nnz"] == len(col)
+    assert_parity(A, B, rp, col, val, exact=(case == "c2"))
+    if info["num_chunks"]:
+        assert rows[0] == 0 and rows[-1] == A.nrows and offs[-1] == info["nnz"]
+
+
+def test_fused_two_phase_and_ring1_identical_structure():
+    A = W.rmat(12, 16, seed=9)
+    a = run(A, A, chunk_nnz=30000)
+    b = run_fused(A, A, chunk_nnz=30000, ring=1)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+
+
+def test_fused_capacity_error_reports_nnz_and_plan_stays_usable():
+    A = W.stencil_3d27(12)
+    z = int(oracle.row_nnz(A, A).sum())
+    with capi.Plan(A, A, 0, capi.opts(fused=True, min_chunks=5)) as P:
+        rp = torch.empty(A.nrows + 1, dtype=torch.int64, pin_memory=True)
+        col = torch.empty(z, dtype=torch.int32, pin_memory=True)
+        val = torch.empty(z, dtype=torch.float64, pin_memory=True)
+        with pytest.raises(capi.SpgemmError) as e:
+            P.execute_capacity(rp, col, val, z // 3)
+        assert e.value.status == capi.ERR_CAPACITY and e.value.nnz == z
+        assert P.execute_capacity(rp, col, val, z) == z
+        assert_parity(A, A, rp.numpy(), col.numpy(), val.numpy(), exact=True)
+        # nnz is now known: execute_into works on the fused plan too
+        P.execute_into(rp, col, val)
+        assert_parity(A, A, rp.numpy(), col.numpy(), val.numpy(), exact=True)
+
+
+def test_fused_sink_and_base():
+    A = W.rmat(12, 16, seed=11)
+    ref = run(A, A)
+    parts = []
+    with capi.Plan(A, A, 0, capi.opts(fused=True, chunk_nnz=40000, ring=2, row_ptr_base=1000)) as P:
+        P.execute_stream(lambda r0, r1, rp, col, val: parts.append((r0, r1, rp.copy(), col.copy(), val.copy())))
+    assert parts[0][0] == 0 and parts[-1][1] == A.nrows
+    col = np.concatenate([p[3] for p in parts])
+    assert np.array_equal(col, ref[1])
+    rpg = [0]
+    for p in parts:
+        rpg.extend((p[2][1:] + rpg[-1]).tolist())
+    assert np.array_equal(np.array(rpg), ref[0])
+    rp, c, v, info, _ = run_fused(A, A, row_ptr_base=777)
+    assert rp[0] == 777 and np.array_equal(rp - 777, ref[0])
