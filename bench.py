@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--two-phase", action="store_true", help="time the two-phase plan/execute path at N = 1")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"])
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     return ap.parse_args()
 
@@ -204,11 +205,18 @@ def main():
     from paper_conf_ipps_xia0ar21_b200 import dist as pdist
 
     world, rank, local = dist_env()
+    # one rank per GPU; --dist-backend gloo lets the multi-rank path run several ranks on one GPU
+    # (a test of the control flow only: NCCL refuses two ranks on one device)
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(args.dist_backend)
 
+    cdev = dev if (world > 1 and args.dist_backend == "nccl") else None  # collective tensors' device
     A, B, budget, name = load_config(args)
     same = A is B
     panels = pdist.row_panels(A.row_ptr, world)
@@ -261,7 +269,7 @@ def main():
     nnz_local = info["nnz"]
     base = 0
     if world > 1:
-        base, nnz_total = pdist.slice_bases(nnz_local, device=dev)
+        base, nnz_total = pdist.slice_bases(nnz_local, device=cdev)
     else:
         nnz_total = nnz_local
     t0 = time.perf_counter()
@@ -278,7 +286,7 @@ def main():
             P.execute_capacity(h_rp, h_col, h_val, nnz_local)
         else:
             if world > 1:
-                b, _ = pdist.slice_bases(P.info()["nnz"], device=dev)
+                b, _ = pdist.slice_bases(P.info()["nnz"], device=cdev)
                 P.set_row_ptr_base(b)
             P.execute_into(h_rp, h_col, h_val)
         st = P.stats() if profile else None
@@ -312,12 +320,12 @@ def main():
     ms = e0.elapsed_time(e1)
     t_max = ms
     if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([ms], dtype=torch.float64, device=cdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         t_max = float(t.item())
     products_total = info["products"]
     if world > 1:
-        products_total = pdist.slice_bases(info["products"], device=dev)[1]
+        products_total = pdist.slice_bases(info["products"], device=cdev)[1]
     value = 2.0 * products_total * args.steps / (t_max / 1e3) / 1e9
 
     # parity spot check of the last step's output (sampled rows vs the oracle)
@@ -407,13 +415,19 @@ def main():
                     dB.row_ptr.copy_(hB.row_ptr, non_blocking=True)
                     dB.col.copy_(hB.col, non_blocking=True)
                     dB.val.copy_(hB.val, non_blocking=True)
-                pdist.broadcast_csr([dB.row_ptr, dB.col, dB.val], src=0)
+                if cdev is not None:
+                    pdist.broadcast_csr([dB.row_ptr, dB.col, dB.val], src=0)
+                else:  # gloo control-flow test: stage through host tensors
+                    hb = [x.cpu() for x in (dB.row_ptr, dB.col, dB.val)]
+                    pdist.broadcast_csr(hb, src=0)
+                    for x, y in zip((dB.row_ptr, dB.col, dB.val), hb):
+                        x.copy_(y)
                 if not same:
                     dA.row_ptr.copy_(hA.row_ptr, non_blocking=True)
                     dA.col.copy_(hA.col, non_blocking=True)
                     dA.val.copy_(hA.val, non_blocking=True)
                 P = capi.Plan(dA, dB, wbytes, mk_opts())
-                b, _ = pdist.slice_bases(P.info()["nnz"], device=dev)
+                b, _ = pdist.slice_bases(P.info()["nnz"], device=cdev)
                 P.set_row_ptr_base(b)
             P.execute_into(h_rp, h_col, h_val)
             P.free()
@@ -430,7 +444,7 @@ def main():
         barrier()
         ems = f0.elapsed_time(f1)
         if world > 1:
-            t = torch.tensor([ems], dtype=torch.float64, device=dev)
+            t = torch.tensor([ems], dtype=torch.float64, device=cdev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
         e2e = {"value": 2.0 * products_total * args.steps / (ems / 1e3) / 1e9, "unit": "GFLOP/s",

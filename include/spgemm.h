@@ -182,6 +182,12 @@ typedef struct {
 /* Fills up to max entries; returns the number of classes in *n. */
 spgemm_status spgemm_stats(spgemm_plan_t plan, spgemm_kernel_stat *stats, int32_t max, int32_t *n);
 
+/* Timeline of the last execution with opts.profile = 1: 6 doubles per chunk, milliseconds from the
+ * start of the execution -- symbolic start, symbolic end (fused plans; -1 otherwise), numeric
+ * start, numeric end (compute stream), copy start, copy end (copy stream).  *n = 6 x chunks; up to
+ * max values are written. */
+spgemm_status spgemm_timeline(spgemm_plan_t plan, double *out, int64_t max, int64_t *n);
+
 /* NULL-safe; frees the arena (if library-owned), streams, events and plan-owned host memory. */
 void spgemm_free(spgemm_plan_t plan);
 

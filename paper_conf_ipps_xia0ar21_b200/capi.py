@@ -292,3 +292,17 @@ def kernel_launches() -> int:
 
 def release_cache():
     _lib.spgemm_release_cache()
+
+
+_lib.spgemm_timeline.restype = ctypes.c_int
+_lib.spgemm_timeline.argtypes = [_P, _P, _I64, ctypes.POINTER(ctypes.c_int64)]
+EXPORTED = EXPORTED + ("spgemm_timeline",)
+
+
+def timeline(plan: "Plan") -> np.ndarray:
+    """[chunks, 6] ms: symbolic start/end, numeric start/end, copy start/end (profile plans)."""
+    n = ctypes.c_int64()
+    _check(_lib.spgemm_timeline(plan.h, None, 0, ctypes.byref(n)))
+    out = np.zeros(max(n.value, 1), dtype=np.float64)
+    _check(_lib.spgemm_timeline(plan.h, out.ctypes.data, n.value, ctypes.byref(n)))
+    return out[:n.value].reshape(-1, 6)

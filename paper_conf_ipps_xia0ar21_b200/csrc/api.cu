@@ -18,6 +18,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <functional>
 #include <mutex>
@@ -145,7 +146,10 @@ struct spgemm_plan_s {
     bool fused = false;
 
     int64_t *bnd = nullptr, *crp = nullptr, *tmp = nullptr;
-    int32_t *nnzr = nullptr, *listB = nullptr, *listG = nullptr;
+    int32_t *nnzr = nullptr, *listB = nullptr, *listG = nullptr;  // symbolic long-row lists
+    int32_t *listBn = nullptr, *listGn = nullptr;                  // numeric long-row lists
+    cudaStream_t astream = nullptr;  // fused plans: symbolic passes run here, ahead of the numeric
+    bool own_astream = false;
     Ctl *ctl = nullptr;  // [0] count / symbolic passes, [1] numeric passes
 
     uint32_t *gbits = nullptr;
@@ -175,6 +179,7 @@ struct spgemm_plan_s {
 
     bool profile = false;
     std::vector<Stat> stats;
+    std::vector<double> timeline;  // profile: 6 times (ms) per chunk of the last execution
     bool failed = false;
 
     size_t take(size_t bytes, const char *what) {
@@ -222,6 +227,10 @@ struct spgemm_plan_s {
         for (auto e : ev_d2h) cudaEventDestroy(e);
         for (auto e : ev_tot) cudaEventDestroy(e);
         if (ev_ready) cudaEventDestroy(ev_ready);
+        if (astream && own_astream) {
+            cudaStreamSynchronize(astream);
+            cudaStreamDestroy(astream);
+        }
         if (copy) cudaStreamDestroy(copy);
         if (own_stream && stream) cudaStreamDestroy(stream);
         if (own_arena && arena) cudaFree(arena);
@@ -251,7 +260,9 @@ void check_csr(const spgemm_csr *M, const char *name) {
 }
 
 // chunk boundaries from a scanned prefix `pre` (pre[0] = 0, pre[R] = total): every chunk's span
-// of `pre` is < capp + (largest single-row increment); empty ids are dropped
+// of `pre` is < capp + (largest single-row increment); empty ids are dropped.  The first chunks
+// ramp up (1/4, 3/8, 1/2, 3/4 of capp, then capp) so that the first D2H starts
+// early and each later chunk is computed while the previous one is being copied.
 void cut_chunks(spgemm_plan_s *P, const int64_t *pre, int64_t total, int64_t capp, int64_t limit,
                 std::vector<int64_t> *offs_out) {
     const int64_t R = P->R;
@@ -259,6 +270,9 @@ void cut_chunks(spgemm_plan_s *P, const int64_t *pre, int64_t total, int64_t cap
     P->chunk_rows.clear();
     if (offs_out) offs_out->clear();
     if (total <= 0) return;
+    constexpr int F = 8;
+    const bool ramp = capp >= F && total / capp >= 4;
+    if (ramp) capp /= F;
     const int64_t nids = total / capp + 1;
     const size_t save = P->used;  // temporary arrays at the start of the (not yet used) ring region
     int64_t *bounds = P->alloc<int64_t>(nids + 1, "chunk bounds");
@@ -274,7 +288,17 @@ void cut_chunks(spgemm_plan_s *P, const int64_t *pre, int64_t total, int64_t cap
     P->chunk_rows.push_back(hb[0]);
     if (offs_out) offs_out->push_back(ho[0]);
     int64_t last_off = ho[0];
-    for (int64_t c = 1; c <= nids; ++c) {
+    // ids (fine units when ramping) that close a chunk
+    std::vector<int64_t> ends;
+    {
+        static const int units[] = {2, 3, 4, 6};
+        int64_t id = 0;
+        for (int k = 0; id < nids; ++k) {
+            id += ramp ? (k < 4 ? units[k] : F) : 1;
+            ends.push_back(std::min(id, nids));
+        }
+    }
+    for (int64_t c : ends) {
         if (hb[c] == P->chunk_rows.back()) continue;
         if (ho[c] - last_off > limit) fail(SPGEMM_ERR_STATE, "internal: chunk exceeds the ring capacity");
         P->chunk_rows.push_back(hb[c]);
@@ -421,6 +445,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->nnzr = P->alloc<int32_t>(R, "row nnz");
     P->listB = P->alloc<int32_t>(R, "listB");
     P->listG = P->alloc<int32_t>(R, "listG");
+    P->listBn = P->alloc<int32_t>(R, "numeric listB");
+    P->listGn = P->alloc<int32_t>(R, "numeric listG");
     P->ctl = P->alloc<Ctl>(2, "ctl");
     P->tmp = P->alloc<int64_t>((R + SCAN_TILE - 1) / SCAN_TILE + 64, "scan scratch");
     CK(cudaMemsetAsync(P->ctl, 0, 2 * sizeof(Ctl), s));
@@ -539,6 +565,15 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         }
         P->ev_tot.resize(nch);
         for (auto &e : P->ev_tot) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        // the symbolic passes get their own stream so that chunk j+1's symbolic pass overlaps
+        // chunk j's numeric pass -- unless both would use the dense-tier scratch
+        const char *ser = getenv("SPGEMM_SERIAL_ANALYSIS");  // ablation knob
+        if (P->gblocks > 0 || (ser && ser[0] == '1')) {
+            P->astream = P->stream;
+        } else {
+            CK(cudaStreamCreateWithFlags(&P->astream, cudaStreamNonBlocking));
+            P->own_astream = true;
+        }
     }
     P->h_small = (int64_t *)pin_acquire(sizeof(int64_t) * (2 * P->num_chunks() + 2));
     CK(cudaHostGetDevicePointer((void **)&P->d_small, P->h_small, 0));
@@ -553,9 +588,11 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         }
         P->ring_bytes = size_t(P->ring) * size_t(P->cap) * 12;
     }
+    pe.rec(9, s);
     CK(cudaStreamSynchronize(s));
     if (P->profile) {
         P->stats.clear();
+        P->add_stat("plan_device_span", elapsed(pe.ev[0], pe.ev[9]), 0);
         P->add_stat("count", elapsed(pe.ev[1], pe.ev[2]), 0);
         if (!P->fused) {
             P->add_stat("sym_w", elapsed(pe.ev[4], pe.ev[5]), 0);
@@ -575,8 +612,8 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t max_row_nnz, cu
     na.r1 = P->chunk_rows[c + 1];
     na.out_col = P->ring_col[b];
     na.out_val = P->ring_val[b];
-    na.listB = P->listB;
-    na.listG = P->listG;
+    na.listB = P->listBn;
+    na.listG = P->listGn;
     na.ctl = P->ctl + 1;
     na.gbits = P->gbits;
     na.gvals = P->gvals;
@@ -593,15 +630,16 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t max_row_nnz, cu
 // h_small[1 + 2j], h_small[2 + 2j] through zero-copy stores (no D2H on the copy engine)
 void enqueue_analysis(spgemm_plan_s *P, int64_t j, cudaEvent_t *ev) {
     const int64_t r0 = P->chunk_rows[j], r1 = P->chunk_rows[j + 1];
+    cudaStream_t as = P->astream;
     SymArgs sa = sym_args(P, r0, r1, sym_tiers(P->chunk_maxb[j]));
-    launch_symbolic(sa, P->num_sms, P->stream, ev);
+    launch_symbolic(sa, P->num_sms, as, ev);
     CKL("symbolic");
-    launch_scan(P->nnzr + r0, r1 - r0, P->crp + r0, P->tmp, P->stream);
+    launch_scan(P->nnzr + r0, r1 - r0, P->crp + r0, P->tmp, as);
     CKL("scan");
-    if (ev) CK(cudaEventRecord(ev[4], P->stream));
-    launch_publish(P->crp + r1, P->ctl, P->d_small + 1 + 2 * j, P->stream);
+    if (ev) CK(cudaEventRecord(ev[4], as));
+    launch_publish(P->crp + r1, P->ctl, P->d_small + 1 + 2 * j, as);
     CKL("publish");
-    CK(cudaEventRecord(P->ev_tot[j], P->stream));
+    CK(cudaEventRecord(P->ev_tot[j], as));
 }
 
 struct Sink {
@@ -627,7 +665,10 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
     if (P->fused) {
         base = P->base_wanted;
         P->h_small[0] = base;
-        CK(cudaMemcpyAsync(P->crp, P->h_small, sizeof(int64_t), cudaMemcpyHostToDevice, s));
+        // the analysis stream starts after everything already queued on the compute stream
+        CK(cudaEventRecord(P->ev_ready, s));
+        CK(cudaStreamWaitEvent(P->astream, P->ev_ready, 0));
+        CK(cudaMemcpyAsync(P->crp, P->h_small, sizeof(int64_t), cudaMemcpyHostToDevice, P->astream));
         P->base_applied = base;
     } else {
         if (P->base_wanted != P->base_applied) {
@@ -708,6 +749,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         const int64_t o = offs[j], n = offs[j + 1] - offs[j];
         if (!sink && o + n > capacity) *overflow = true;
         if (j >= ring) CK(cudaStreamWaitEvent(s, P->ev_d2h[b], 0));
+        if (P->fused) CK(cudaStreamWaitEvent(s, P->ev_tot[j], 0));  // (already complete: host waited)
         if (!*overflow) {
             pe.rec(size_t(j) * per + 5, s);
             enqueue_numeric(P, j, b, mx, pe.at(size_t(j) * per + 6));
@@ -729,6 +771,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         } else if (rp_out && P->fused && r1 > r0) {
             CK(cudaMemcpyAsync(rp_out + r0 + 1, P->crp + r0 + 1, sizeof(int64_t) * (r1 - r0), cudaMemcpyDeviceToHost, cp));
         }
+        pe.rec(size_t(j) * per + 11, cp);
         CK(cudaEventRecord(P->ev_d2h[b], cp));
     }
     if (sink)
@@ -736,6 +779,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
     pe.rec(size_t(nch) * per + 1, cp);
     CK(cudaStreamSynchronize(cp));
     CK(cudaStreamSynchronize(s));
+    if (P->astream && P->astream != s) CK(cudaStreamSynchronize(P->astream));
     unsigned err[2] = {0, 0};
     CK(cudaMemcpy(&err[0], &P->ctl[1].err, sizeof(unsigned), cudaMemcpyDeviceToHost));
     if (err[0]) fail(SPGEMM_ERR_STATE, "internal: numeric pass produced a row whose nnz differs from the symbolic pass");
@@ -771,6 +815,23 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         }
         P->add_stat("execute_total", elapsed(pe.ev[size_t(nch) * per], pe.ev[size_t(nch) * per + 1]),
                     double(total) * 12 + 8.0 * (P->R + 1));
+        // timeline: per chunk [analysis start, end, numeric start, end, copy start, end] in ms
+        P->timeline.assign(size_t(nch) * 6, -1.0);
+        cudaEvent_t t0 = pe.ev[size_t(nch) * per];
+        for (int64_t c = 0; c < nch; ++c) {
+            cudaEvent_t *e = pe.at(size_t(c) * per);
+            double *t = &P->timeline[size_t(c) * 6];
+            if (P->fused) {
+                t[0] = elapsed(t0, e[0]);
+                t[1] = elapsed(t0, e[4]);
+            }
+            if (!*overflow) {
+                t[2] = elapsed(t0, e[6]);
+                t[3] = elapsed(t0, e[9]);
+                t[4] = elapsed(t0, e[10]);
+                t[5] = elapsed(t0, e[11]);
+            }
+        }
     }
     return total;
 }
@@ -1001,6 +1062,16 @@ spgemm_status spgemm_stats(spgemm_plan_t P, spgemm_kernel_stat *out, int32_t max
         out[k].ms = P->stats[k].ms;
         out[k].bytes = P->stats[k].bytes;
     }
+    return SPGEMM_OK;
+}
+
+spgemm_status spgemm_timeline(spgemm_plan_t P, double *out, int64_t max, int64_t *n) {
+    if (!P || !n) {
+        g_err = "NULL argument";
+        return SPGEMM_ERR_INVALID_ARGUMENT;
+    }
+    *n = (int64_t)P->timeline.size();
+    for (int64_t k = 0; k < max && k < *n && out; ++k) out[k] = P->timeline[k];
     return SPGEMM_OK;
 }
 

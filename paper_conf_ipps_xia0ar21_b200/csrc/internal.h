@@ -68,6 +68,7 @@ struct SymArgs {
     int group;           // lanes per A entry in the W kernel (4, 8, 16, 32)
     int tiers;           // bit 0: launch the CTA tier, bit 1: the dense tier (host knows when a
                          // pass cannot have such rows, and skips those launches)
+    int batch;           // rows per claim in the W kernel (set by the launcher)
 };
 
 // tier bits for a pass whose rows have bound <= maxb
@@ -111,6 +112,7 @@ struct NumArgs {
     int gblocks;
     int group;
     int tiers;           // as in SymArgs
+    int batch;
 };
 // S6+S7: numeric pass over chunk rows [r0, r1); ev as in launch_symbolic
 void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);
@@ -131,7 +133,7 @@ const Grids &grids(int device, int num_sms);
 long long kernel_launches();
 
 size_t symw_smem();
-size_t numw_smem();
+size_t numw_smem(bool wide);
 size_t symb_smem();
 size_t numb_smem();
 

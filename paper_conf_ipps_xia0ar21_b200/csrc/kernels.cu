@@ -294,10 +294,10 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
     constexpr int MAXLG = 10;  // log2(TW_SYM)
     while (true) {
         unsigned long long base = 0;
-        if (lane == 0) base = atomicAdd(&a.ctl->row_ctr, (unsigned long long)ROW_BATCH);
+        if (lane == 0) base = atomicAdd(&a.ctl->row_ctr, (unsigned long long)a.batch);
         base = __shfl_sync(FULLMASK, base, 0);
         if ((int64_t)base >= R) break;
-        const int64_t end = min((int64_t)base + ROW_BATCH, R);
+        const int64_t end = min((int64_t)base + a.batch, R);
         for (int64_t li = (int64_t)base; li < end; ++li) {
             const int64_t i = a.r0 + li;
             const int64_t bound = a.bnd[i];
@@ -547,21 +547,83 @@ __device__ __forceinline__ int pow2_at_least(int64_t n, int lo) {
 
 // ------------------------------------------------------------------------------ S6 numeric, W
 
-template <int G>
+// Register bitonic sort of 32*E packed keys held E per lane (element e = r*32 + lane), ascending;
+// partners within a lane for j >= 32, across lanes (shfl_xor) for j < 32.
+template <typename K, int E>
+__device__ __forceinline__ void reg_bitonic(K (&x)[E]) {
+    const int lane = threadIdx.x & 31;
+    constexpr int N = 32 * E;
+#pragma unroll
+    for (int k = 2; k <= N; k <<= 1) {
+#pragma unroll
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            if (j >= 32) {
+#pragma unroll
+                for (int r = 0; r < E; ++r) {
+                    const int p = r ^ (j >> 5);
+                    if (p > r) {
+                        const bool up = (((r << 5) | lane) & k) == 0;
+                        const K u = x[r], v = x[p];
+                        const bool sw = (u > v) == up;
+                        x[r] = sw ? v : u;
+                        x[p] = sw ? u : v;
+                    }
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < E; ++r) {
+                    const K y = __shfl_xor_sync(FULLMASK, x[r], j);
+                    const bool up = (((r << 5) | lane) & k) == 0;
+                    const bool keep_min = ((lane & j) == 0) == up;
+                    x[r] = keep_min ? (y < x[r] ? y : x[r]) : (y > x[r] ? y : x[r]);
+                }
+            }
+        }
+    }
+}
+
+// load n packed keys (column << 9 | slot) from smem, sort them in registers and write the row
+// out in column order: col from the key, value gathered from its hash slot (S7, §II-B)
+template <typename K, int E>
+__device__ __forceinline__ void sort_emit(const K *pk, int n, const double *vals, int32_t *oc, double *ov) {
+    const int lane = threadIdx.x & 31;
+    K x[E];
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+        const int e = (r << 5) | lane;
+        x[r] = e < n ? pk[e] : ~K(0);
+    }
+    __syncwarp();
+    reg_bitonic<K, E>(x);
+#pragma unroll
+    for (int r = 0; r < E; ++r) {
+        const int e = (r << 5) | lane;
+        if (e < n) {
+            oc[e] = (int32_t)(x[r] >> 9);
+            ov[e] = vals[(int)(x[r] & 511u)];
+        }
+    }
+}
+
+template <int G, bool WIDE>
 __global__ void __launch_bounds__(WARPS_W * 32) k_num_w(NumArgs a) {
     extern __shared__ double smem_d[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     double *vals = smem_d + wid * TW_NUM;
     int32_t *keys = reinterpret_cast<int32_t *>(smem_d + WARPS_W * TW_NUM) + wid * TW_NUM;
+    // WIDE (ncols > 2^23): 64-bit packed keys staged after the key tables
+    unsigned long long *stage = reinterpret_cast<unsigned long long *>(
+                                    reinterpret_cast<int32_t *>(smem_d + WARPS_W * TW_NUM) + WARPS_W * TW_NUM) +
+                                wid * TW_NUM;
     constexpr int MAXLG = 9;  // log2(TW_NUM)
     const int64_t R = a.r1 - a.r0;
     const int64_t off0 = a.crp[a.r0];
     while (true) {
         unsigned long long base = 0;
-        if (lane == 0) base = atomicAdd(&a.ctl->row_ctr, (unsigned long long)ROW_BATCH);
+        if (lane == 0) base = atomicAdd(&a.ctl->row_ctr, (unsigned long long)a.batch);
         base = __shfl_sync(FULLMASK, base, 0);
         if ((int64_t)base >= R) break;
-        const int64_t end = min((int64_t)base + ROW_BATCH, R);
+        const int64_t end = min((int64_t)base + a.batch, R);
         for (int64_t li = (int64_t)base; li < end; ++li) {
             const int64_t i = a.r0 + li;
             const int64_t o = a.crp[i];
@@ -594,19 +656,20 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_num_w(NumArgs a) {
                 }
             });
             __syncwarp();
-            // in-place compaction of the occupied slots (destination <= source, one round of 32
-            // slots is read completely before any of it is written)
+            // compaction of the occupied slots into packed sort keys (column << 9 | slot): in place
+            // in `keys` for 32-bit keys (destination <= source, a round of 32 slots is read before
+            // any of it is written), into the warp's staging array for 64-bit keys.  Values stay
+            // in their slots and are gathered by slot after the sort.
             int cnt = 0;
             for (int t0 = 0; t0 < T; t0 += 32) {
                 const int32_t k = keys[t0 + lane];
-                const double v = vals[t0 + lane];
                 const bool occ = k != EMPTY;
                 const unsigned bal = __ballot_sync(FULLMASK, occ);
                 const int dst = cnt + __popc(bal & ((1u << lane) - 1u));
                 __syncwarp();
                 if (occ) {
-                    keys[dst] = k;
-                    vals[dst] = v;
+                    if (WIDE) stage[dst] = ((unsigned long long)(uint32_t)k << 9) | (unsigned)(t0 + lane);
+                    else reinterpret_cast<uint32_t *>(keys)[dst] = ((uint32_t)k << 9) | (uint32_t)(t0 + lane);
                 }
                 cnt += __popc(bal);
                 __syncwarp();
@@ -615,15 +678,26 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_num_w(NumArgs a) {
                 if (lane == 0) atomicOr(&a.ctl->err, 1u);
                 continue;
             }
-            const int N = pow2_at_least(n, 32);
-            for (int t = (int)n + lane; t < N; t += 32) keys[t] = INT_MAX;
-            __syncwarp();
-            warp_bitonic(keys, vals, N);
             int32_t *oc = a.out_col + (o - off0);
             double *ov = a.out_val + (o - off0);
-            for (int t = lane; t < n; t += 32) {
-                oc[t] = keys[t];
-                ov[t] = vals[t];
+            const int E = pow2_at_least((n + 31) / 32, 1);
+            if (WIDE) {
+                switch (E) {
+                    case 1: sort_emit<unsigned long long, 1>(stage, (int)n, vals, oc, ov); break;
+                    case 2: sort_emit<unsigned long long, 2>(stage, (int)n, vals, oc, ov); break;
+                    case 4: sort_emit<unsigned long long, 4>(stage, (int)n, vals, oc, ov); break;
+                    case 8: sort_emit<unsigned long long, 8>(stage, (int)n, vals, oc, ov); break;
+                    default: sort_emit<unsigned long long, 16>(stage, (int)n, vals, oc, ov); break;
+                }
+            } else {
+                const uint32_t *pk = reinterpret_cast<const uint32_t *>(keys);
+                switch (E) {
+                    case 1: sort_emit<uint32_t, 1>(pk, (int)n, vals, oc, ov); break;
+                    case 2: sort_emit<uint32_t, 2>(pk, (int)n, vals, oc, ov); break;
+                    case 4: sort_emit<uint32_t, 4>(pk, (int)n, vals, oc, ov); break;
+                    case 8: sort_emit<uint32_t, 8>(pk, (int)n, vals, oc, ov); break;
+                    default: sort_emit<uint32_t, 16>(pk, (int)n, vals, oc, ov); break;
+                }
             }
             __syncwarp();
         }
@@ -759,14 +833,17 @@ __global__ void __launch_bounds__(THREADS_G) k_num_g(NumArgs a) {
 // ------------------------------------------------------------------------------------ launchers
 
 size_t symw_smem() { return size_t(WARPS_W) * TW_SYM * sizeof(int32_t); }
-size_t numw_smem() { return size_t(WARPS_W) * TW_NUM * (sizeof(int32_t) + sizeof(double)); }
+size_t numw_smem(bool wide) {
+    return size_t(WARPS_W) * TW_NUM * (sizeof(int32_t) + sizeof(double) + (wide ? sizeof(unsigned long long) : 0));
+}
 size_t symb_smem() { return size_t(TB_SYM) * sizeof(int32_t); }
 size_t numb_smem() { return size_t(TB_NUM) * (sizeof(int32_t) + sizeof(double)); }
 
 template <int G>
 static void set_attrs_w() {
     cudaFuncSetAttribute(k_sym_w<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symw_smem());
-    cudaFuncSetAttribute(k_num_w<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem());
+    cudaFuncSetAttribute(k_num_w<G, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(false));
+    cudaFuncSetAttribute(k_num_w<G, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(true));
 }
 
 const Grids &grids(int device, int num_sms) {
@@ -786,7 +863,7 @@ const Grids &grids(int device, int num_sms) {
         g.count_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_w<8>, WARPS_W * 32, symw_smem());
         g.symw_blocks = num_sms * (occ > 0 ? occ : 1);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<8>, WARPS_W * 32, numw_smem());
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false>, WARPS_W * 32, numw_smem(false));
         g.numw_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b, THREADS_B, symb_smem());
         g.symb_blocks = num_sms * (occ > 0 ? occ : 1);
@@ -796,6 +873,14 @@ const Grids &grids(int device, int num_sms) {
         init[device] = true;
     }
     return cache[device];
+}
+
+// rows a warp claims per atomic: large batches amortise the counter, small ones keep every SM
+// busy on small chunks (at least ~4 claims per resident warp)
+static int batch_for(int64_t rows, int full_blocks) {
+    const int64_t warps = int64_t(full_blocks) * WARPS_W;
+    int64_t b = rows / (warps * 4);
+    return (int)(b < 1 ? 1 : (b > ROW_BATCH ? ROW_BATCH : b));
 }
 
 static int grid_for(int64_t n, int threads, int cap) {
@@ -840,7 +925,8 @@ static void sym_w(const SymArgs &a, int blocks, cudaStream_t s) {
 }
 template <int G>
 static void num_w(const NumArgs &a, int blocks, cudaStream_t s) {
-    k_num_w<G><<<blocks, WARPS_W * 32, numw_smem(), s>>>(a);
+    if (a.B.ncols > (int64_t(1) << 23)) k_num_w<G, true><<<blocks, WARPS_W * 32, numw_smem(true), s>>>(a);
+    else k_num_w<G, false><<<blocks, WARPS_W * 32, numw_smem(false), s>>>(a);
     LAUNCHED(1);
 }
 
@@ -866,13 +952,15 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
     cudaMemsetAsync(&a.ctl->row_ctr, 0, 24, s);  // row_ctr, nB, nG, pass_max
-    const int wblocks = grid_for(rows, WARPS_W * ROW_BATCH, g.symw_blocks);
+    SymArgs aw = a;
+    aw.batch = batch_for(rows, g.symw_blocks);
+    const int wblocks = grid_for(rows, WARPS_W * aw.batch, g.symw_blocks);
     rec(ev, 0, s);
     switch (a.group) {
-        case 4: sym_w<4>(a, wblocks, s); break;
-        case 8: sym_w<8>(a, wblocks, s); break;
-        case 16: sym_w<16>(a, wblocks, s); break;
-        default: sym_w<32>(a, wblocks, s); break;
+        case 4: sym_w<4>(aw, wblocks, s); break;
+        case 8: sym_w<8>(aw, wblocks, s); break;
+        case 16: sym_w<16>(aw, wblocks, s); break;
+        default: sym_w<32>(aw, wblocks, s); break;
     }
     rec(ev, 1, s);
     if (a.tiers & 1) {
@@ -897,13 +985,15 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
     cudaMemsetAsync(&a.ctl->row_ctr, 0, 24, s);
-    const int wblocks = grid_for(rows, WARPS_W * ROW_BATCH, g.numw_blocks);
+    NumArgs aw = a;
+    aw.batch = batch_for(rows, g.numw_blocks);
+    const int wblocks = grid_for(rows, WARPS_W * aw.batch, g.numw_blocks);
     rec(ev, 0, s);
     switch (a.group) {
-        case 4: num_w<4>(a, wblocks, s); break;
-        case 8: num_w<8>(a, wblocks, s); break;
-        case 16: num_w<16>(a, wblocks, s); break;
-        default: num_w<32>(a, wblocks, s); break;
+        case 4: num_w<4>(aw, wblocks, s); break;
+        case 8: num_w<8>(aw, wblocks, s); break;
+        case 16: num_w<16>(aw, wblocks, s); break;
+        default: num_w<32>(aw, wblocks, s); break;
     }
     rec(ev, 1, s);
     if (a.tiers & 1) {

@@ -150,6 +150,21 @@ def test_tiers_warp_block_global():
     assert_parity(A, B, rp, col, val)
 
 
+@pytest.mark.parametrize("fused", [False, True])
+def test_wide_column_space(fused):
+    """ncols > 2^23: the numeric sort switches to 64-bit packed keys (column << 9 | slot)."""
+    n = (1 << 23) + 4099
+    B = W.random_csr_sparse(300, n, 40.0, seed=31)
+    B.col[-3:] = [n - 3, n - 2, n - 1]  # touch the top of the column range (rows stay sorted)
+    B.col = np.ascontiguousarray(B.col)
+    last = B.nrows - 1
+    seg = np.sort(np.unique(B.col[B.row_ptr[last]:B.row_ptr[last + 1]]))
+    assert len(seg) == B.row_ptr[last + 1] - B.row_ptr[last]
+    A = W.random_csr_sparse(500, 300, 6.0, seed=32)
+    r = run_fused(A, B) if fused else run(A, B)
+    assert_parity(A, B, r[0], r[1], r[2])
+
+
 def test_rmat_skewed():
     A = W.rmat(14, 16, seed=5)
     rp, col, val, info, _ = run(A, A)
