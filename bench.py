@@ -243,10 +243,11 @@ def main():
     wbytes = ws.numel()
     stream = torch.cuda.current_stream()
 
-    # N = 1: the fused plan (per-chunk symbolic overlapped with the previous chunk's D2H, the call
-    # spgemm_multiply makes).  N > 1: two-phase plans, because every rank needs its global row_ptr
-    # base (an all_gather of the ranks' nnz) before it writes row offsets.
-    fused = world == 1 and not args.two_phase
+    # Fused plans (per-chunk symbolic overlapped with the previous chunk's D2H, the call
+    # spgemm_multiply makes).  With N > 1 ranks each rank's global row_ptr base is the sum of the
+    # earlier ranks' nnz, known after execution: an 8-byte all_gather, then spgemm_rebase_host on
+    # the rank's row_ptr slice.  --two-phase: plans whose symbolic pass runs in spgemm_plan.
+    fused = not args.two_phase
 
     def mk_opts(profile=False, base=0):
         return capi.opts(device=local, ring=args.ring, profile=profile, row_begin=r0, row_end=r1, workspace=ws,
@@ -283,7 +284,10 @@ def main():
     def step(profile=False):
         P = capi.Plan(dA, dB, wbytes, mk_opts(profile))
         if fused:
-            P.execute_capacity(h_rp, h_col, h_val, nnz_local)
+            z = P.execute_capacity(h_rp, h_col, h_val, nnz_local)
+            if world > 1:
+                b, _ = pdist.slice_bases(z, device=cdev)
+                capi.rebase_host(h_rp, b)
         else:
             if world > 1:
                 b, _ = pdist.slice_bases(P.info()["nnz"], device=cdev)
@@ -427,6 +431,12 @@ def main():
                     dA.col.copy_(hA.col, non_blocking=True)
                     dA.val.copy_(hA.val, non_blocking=True)
                 P = capi.Plan(dA, dB, wbytes, mk_opts())
+                if fused:
+                    z = P.execute_capacity(h_rp, h_col, h_val, nnz_local)
+                    b, _ = pdist.slice_bases(z, device=cdev)
+                    capi.rebase_host(h_rp, b)
+                    P.free()
+                    return
                 b, _ = pdist.slice_bases(P.info()["nnz"], device=cdev)
                 P.set_row_ptr_base(b)
             P.execute_into(h_rp, h_col, h_val)

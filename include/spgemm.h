@@ -158,6 +158,10 @@ typedef int (*spgemm_chunk_cb)(void *user, int64_t row0, int64_t row1, const int
                                const int32_t *col_idx, const double *values, int64_t nnz);
 spgemm_status spgemm_execute_stream(spgemm_plan_t plan, spgemm_chunk_cb cb, void *user);
 
+/* Add `delta` to n host row_ptr entries (multi-GPU with fused plans: a rank's global base is known
+ * only after every rank has counted its nnz, i.e. after execution).  Host memory, in place. */
+spgemm_status spgemm_rebase_host(int64_t *row_ptr, int64_t n, int64_t delta);
+
 /* Change the base added to C row_ptr values (multi-GPU: global offset of this rank's slice,
  * known after the ranks exchange their nnz).  Applies to the next execute. */
 spgemm_status spgemm_set_row_ptr_base(spgemm_plan_t plan, int64_t base);

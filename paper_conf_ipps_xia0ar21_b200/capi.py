@@ -306,3 +306,14 @@ def timeline(plan: "Plan") -> np.ndarray:
     out = np.zeros(max(n.value, 1), dtype=np.float64)
     _check(_lib.spgemm_timeline(plan.h, out.ctypes.data, n.value, ctypes.byref(n)))
     return out[:n.value].reshape(-1, 6)
+
+
+_lib.spgemm_rebase_host.restype = ctypes.c_int
+_lib.spgemm_rebase_host.argtypes = [_P, _I64, _I64]
+EXPORTED = EXPORTED + ("spgemm_rebase_host",)
+
+
+def rebase_host(row_ptr, delta: int) -> None:
+    """row_ptr[:] += delta in place (host int64 array / tensor), in the library."""
+    n = row_ptr.shape[0]
+    _check(_lib.spgemm_rebase_host(_ptr(row_ptr), int(n), int(delta)))

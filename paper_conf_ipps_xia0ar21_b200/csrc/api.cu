@@ -1026,6 +1026,16 @@ spgemm_status spgemm_execute_stream(spgemm_plan_t P, spgemm_chunk_cb cb, void *u
     return st;
 }
 
+spgemm_status spgemm_rebase_host(int64_t *row_ptr, int64_t n, int64_t delta) {
+    if (n > 0 && !row_ptr) {
+        g_err = "row_ptr is NULL";
+        return SPGEMM_ERR_INVALID_ARGUMENT;
+    }
+    if (delta == 0) return SPGEMM_OK;
+    for (int64_t i = 0; i < n; ++i) row_ptr[i] += delta;
+    return SPGEMM_OK;
+}
+
 spgemm_status spgemm_set_row_ptr_base(spgemm_plan_t P, int64_t base) {
     if (!P) {
         g_err = "plan is NULL";

@@ -606,7 +606,7 @@ __device__ __forceinline__ void sort_emit(const K *pk, int n, const double *vals
 }
 
 template <int G, bool WIDE>
-__global__ void __launch_bounds__(WARPS_W * 32) k_num_w(NumArgs a) {
+__global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
     extern __shared__ double smem_d[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     double *vals = smem_d + wid * TW_NUM;

@@ -42,3 +42,6 @@ for label, kw in [("fused_ring2", dict(fused=True, ring=2)), ("fused_ring3", dic
         print(f"  c{c:02d} sym {t[c,0]:7.3f}-{t[c,1]:7.3f}  num {t[c,2]:7.3f}-{t[c,3]:7.3f}  d2h {t[c,4]:7.3f}-{t[c,5]:7.3f}  gap {t[c,4]-(t[c-1,5] if c else 0):6.3f}")
 os.makedirs("gpurun_out", exist_ok=True)
 json.dump(out, open("gpurun_out/timeline.json", "w"))
+for label, v in out.items():
+    st = v["stats"]
+    print(label, {k: round(st[k]["ms"], 3) for k in ("sym_w", "num_w", "scan", "d2h_span", "execute_total") if k in st})
