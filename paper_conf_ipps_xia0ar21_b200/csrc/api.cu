@@ -150,6 +150,11 @@ struct spgemm_plan_s {
     int32_t *listBn = nullptr, *listGn = nullptr;                  // numeric long-row lists
     cudaStream_t astream = nullptr;  // fused plans: symbolic passes run here, ahead of the numeric
     bool own_astream = false;
+    cudaStream_t hstream = nullptr;         // host B: value pieces H2D
+    std::vector<cudaEvent_t> ev_piece;      // one per value piece, in upload order
+    std::vector<int64_t> bpiece_rows;       // B row boundaries of the pieces
+    std::vector<int> chunk_wait;            // per chunk: last piece its numeric pass reads (-1: none)
+    bool a_alias = false;
     Ctl *ctl = nullptr;  // [0] count / symbolic passes, [1] numeric passes
 
     uint32_t *gbits = nullptr;
@@ -231,6 +236,11 @@ struct spgemm_plan_s {
             cudaStreamSynchronize(astream);
             cudaStreamDestroy(astream);
         }
+        if (hstream) {
+            cudaStreamSynchronize(hstream);
+            cudaStreamDestroy(hstream);
+        }
+        for (auto e : ev_piece) cudaEventDestroy(e);
         if (copy) cudaStreamDestroy(copy);
         if (own_stream && stream) cudaStreamDestroy(stream);
         if (own_arena && arena) cudaFree(arena);
@@ -397,7 +407,11 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     EvSet pe(P->profile, 12);
     pe.rec(0, s);
 
-    // S0 residency: B
+    // S0 residency: B.  Host operands: row_ptr and col_idx now (the count and symbolic passes need
+    // only the structure); the values follow in row pieces on the H2D stream, overlapping the
+    // planning and the first chunks (the numeric pass of a chunk waits for the pieces it reads).
+    std::vector<std::pair<size_t, size_t>> bval_pieces;  // (element offset, count)
+    double *bval_dev = nullptr;
     if (Bh->where == SPGEMM_DEVICE) {
         P->B = DevCSR{Bh->row_ptr, Bh->col_idx, Bh->values, Bh->nrows, Bh->ncols};
     } else {
@@ -405,10 +419,20 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         int32_t *c = P->alloc<int32_t>(Bh->nnz, "B.col_idx");
         double *v = P->alloc<double>(Bh->nnz, "B.values");
         CK(cudaMemcpyAsync(rp, Bh->row_ptr, sizeof(int64_t) * (Bh->nrows + 1), cudaMemcpyHostToDevice, s));
-        if (Bh->nnz) {
-            CK(cudaMemcpyAsync(c, Bh->col_idx, sizeof(int32_t) * Bh->nnz, cudaMemcpyHostToDevice, s));
-            CK(cudaMemcpyAsync(v, Bh->values, sizeof(double) * Bh->nnz, cudaMemcpyHostToDevice, s));
+        if (Bh->nnz) CK(cudaMemcpyAsync(c, Bh->col_idx, sizeof(int32_t) * Bh->nnz, cudaMemcpyHostToDevice, s));
+        // pieces of ~32 MB of values, cut at row boundaries
+        const int64_t target = std::max<int64_t>(1, (32ll << 20) / 8);
+        P->bpiece_rows.push_back(0);
+        int64_t r = 0;
+        while (r < Bh->nrows) {
+            const int64_t want = Bh->row_ptr[r] + target;
+            int64_t e = std::upper_bound(Bh->row_ptr + r + 1, Bh->row_ptr + Bh->nrows + 1, want) - Bh->row_ptr - 1;
+            e = std::max<int64_t>(e, r + 1);
+            bval_pieces.push_back({size_t(Bh->row_ptr[r]), size_t(Bh->row_ptr[e] - Bh->row_ptr[r])});
+            P->bpiece_rows.push_back(e);
+            r = e;
         }
+        bval_dev = v;
         P->B = DevCSR{rp, c, v, Bh->nrows, Bh->ncols};
     }
     // S0 residency + S1 row panel: A
@@ -422,6 +446,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         P->nnzA = p1 - p0;
         if (alias) {
             P->A = DevCSR{P->B.rp + rb, P->B.col, P->B.val, P->R, Ah->ncols};
+            P->a_alias = true;
         } else {
             int64_t *rp = P->alloc<int64_t>(P->R + 1, "A.row_ptr");
             int32_t *c = P->alloc<int32_t>(p1 - p0, "A.col_idx");
@@ -434,6 +459,21 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
             launch_rebase(rp, P->R + 1, p0, s);
             CKL("rebase");
             P->A = DevCSR{rp, c, v, P->R, Ah->ncols};
+        }
+    }
+    // start the B value pieces (host operands) on their own stream, one event per piece
+    if (!bval_pieces.empty()) {
+        CK(cudaStreamCreateWithFlags(&P->hstream, cudaStreamNonBlocking));
+        CK(cudaEventRecord(P->ev_ready, s));  // allocation order: after everything queued so far
+        CK(cudaStreamWaitEvent(P->hstream, P->ev_ready, 0));
+        P->ev_piece.resize(bval_pieces.size());
+        for (size_t k = 0; k < bval_pieces.size(); ++k) {
+            const auto &pc = bval_pieces[k];
+            if (pc.second)
+                CK(cudaMemcpyAsync(bval_dev + pc.first, Bh->values + pc.first, sizeof(double) * pc.second,
+                                   cudaMemcpyHostToDevice, P->hstream));
+            CK(cudaEventCreateWithFlags(&P->ev_piece[k], cudaEventDisableTiming));
+            CK(cudaEventRecord(P->ev_piece[k], P->hstream));
         }
     }
     P->group = choose_group(P->B, P->nnzB);
@@ -573,6 +613,31 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         } else {
             CK(cudaStreamCreateWithFlags(&P->astream, cudaStreamNonBlocking));
             P->own_astream = true;
+        }
+    }
+    // host operands: the last value piece each chunk's numeric pass reads (largest B row touched;
+    // with A aliasing B also the chunk's own rows)
+    {
+        const int64_t nch = P->num_chunks();
+        P->chunk_wait.assign(nch, -1);
+        if (!P->ev_piece.empty() && nch > 0) {
+            const size_t save = P->used;
+            int64_t *drows = P->alloc<int64_t>(nch + 1, "chunk rows");
+            int64_t *dmax = P->alloc<int64_t>(nch, "chunk max column");
+            std::vector<int64_t> hmax(nch);
+            CK(cudaMemcpyAsync(drows, P->chunk_rows.data(), sizeof(int64_t) * (nch + 1), cudaMemcpyHostToDevice, s));
+            launch_seg_max_col(P->A, drows, nch, dmax, s);
+            CKL("chunk max column");
+            CK(cudaMemcpyAsync(hmax.data(), dmax, sizeof(int64_t) * nch, cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            P->used = save;
+            for (int64_t j = 0; j < nch; ++j) {
+                int64_t need = hmax[j];
+                if (P->a_alias) need = std::max<int64_t>(need, rb + P->chunk_rows[j + 1] - 1);
+                if (need < 0) continue;
+                const auto it = std::upper_bound(P->bpiece_rows.begin(), P->bpiece_rows.end(), need);
+                P->chunk_wait[j] = int(it - P->bpiece_rows.begin()) - 1;
+            }
         }
     }
     P->h_small = (int64_t *)pin_acquire(sizeof(int64_t) * (2 * P->num_chunks() + 2));
@@ -750,6 +815,8 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         if (!sink && o + n > capacity) *overflow = true;
         if (j >= ring) CK(cudaStreamWaitEvent(s, P->ev_d2h[b], 0));
         if (P->fused) CK(cudaStreamWaitEvent(s, P->ev_tot[j], 0));  // (already complete: host waited)
+        if (!P->chunk_wait.empty() && P->chunk_wait[j] >= 0)       // host operands: value pieces
+            CK(cudaStreamWaitEvent(s, P->ev_piece[P->chunk_wait[j]], 0));
         if (!*overflow) {
             pe.rec(size_t(j) * per + 5, s);
             enqueue_numeric(P, j, b, mx, pe.at(size_t(j) * per + 6));

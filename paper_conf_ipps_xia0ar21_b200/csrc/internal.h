@@ -79,6 +79,9 @@ inline int num_tiers(int64_t maxnnz) { return (maxnnz > CAPW_NUM ? 1 : 0) | (max
 // pinned memory, so no small D2H copy queues behind the big ones on the copy engine
 void launch_publish(const int64_t *end, const Ctl *ctl, int64_t *host2, cudaStream_t s);
 
+// out[k] = largest column index in A's rows [rows[k], rows[k+1]) (-1 if none)
+void launch_seg_max_col(const DevCSR &A, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s);
+
 // out[k] = max(x[rows[k] .. rows[k+1]-1]) for k < nseg (0 for empty segments)
 void launch_seg_max(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s);
 // S3+S4: symbolic pass over all rows (tiering + the three tiers).  ev: NULL or 4 events recorded

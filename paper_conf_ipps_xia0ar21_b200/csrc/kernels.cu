@@ -1063,6 +1063,30 @@ __global__ void __launch_bounds__(256) k_seg_max(const int64_t *__restrict__ x, 
     }
 }
 
+// out[k] = largest column index in A's rows [rows[k], rows[k+1]) (-1 if they hold no entry): the
+// last row of B a chunk reads
+__global__ void __launch_bounds__(256) k_seg_max_col(DevCSR A, const int64_t *__restrict__ rows,
+                                                     int64_t *__restrict__ out) {
+    __shared__ int s[8];
+    const int64_t p0 = A.rp[rows[blockIdx.x]], p1 = A.rp[rows[blockIdx.x + 1]];
+    int m = -1;
+    for (int64_t p = p0 + threadIdx.x; p < p1; p += blockDim.x) m = max(m, A.col[p]);
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) m = max(m, __shfl_xor_sync(FULLMASK, m, d));
+    if ((threadIdx.x & 31) == 0) s[threadIdx.x >> 5] = m;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < 8; ++w) m = max(m, s[w]);
+        out[blockIdx.x] = max(m, s[0]);
+    }
+}
+
+void launch_seg_max_col(const DevCSR &A, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s) {
+    if (nseg <= 0) return;
+    k_seg_max_col<<<(unsigned)nseg, 256, 0, s>>>(A, rows, out);
+    LAUNCHED(1);
+}
+
 void launch_seg_max(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s) {
     if (nseg <= 0) return;
     k_seg_max<<<(unsigned)nseg, 256, 0, s>>>(x, rows, out);
