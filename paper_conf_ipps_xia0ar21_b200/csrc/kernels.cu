@@ -582,9 +582,10 @@ __device__ __forceinline__ void reg_bitonic(K (&x)[E]) {
     }
 }
 
-// load n packed keys (column << 9 | slot) from smem, sort them in registers and write the row
-// out in column order: col from the key, value gathered from its hash slot (S7, §II-B)
-template <typename K, int E>
+// load n packed keys (column << SB | slot) from smem or global memory, sort them in registers and
+// write the row out in column order: col from the key, value gathered from its hash slot in
+// shared memory (S7, §II-B).  pk may alias ov: all loads complete before any store.
+template <typename K, int E, int SB = 9>
 __device__ __forceinline__ void sort_emit(const K *pk, int n, const double *vals, int32_t *oc, double *ov) {
     const int lane = threadIdx.x & 31;
     K x[E];
@@ -599,8 +600,8 @@ __device__ __forceinline__ void sort_emit(const K *pk, int n, const double *vals
     for (int r = 0; r < E; ++r) {
         const int e = (r << 5) | lane;
         if (e < n) {
-            oc[e] = (int32_t)(x[r] >> 9);
-            ov[e] = vals[(int)(x[r] & 511u)];
+            oc[e] = (int32_t)(x[r] >> SB);
+            ov[e] = vals[(int)(x[r] & ((1u << SB) - 1u))];
         }
     }
 }
@@ -711,6 +712,7 @@ __global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
     double *vals = smem_d;
     int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);
     __shared__ int64_t s_scan[40];
+    __shared__ int s_cnt[64], s_cur[64], s_start[64], s_mm[3], s_occ[THREADS_B / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     constexpr int NW = THREADS_B / 32;
     constexpr int MAXLG = 14;  // log2(TB_NUM)
@@ -736,6 +738,94 @@ __global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
                 num_insert(keys, vals, __ldg(&a.B.col[q]), av * __ldg(&a.B.val[q]), lg);
         }
         __syncthreads();
+        int32_t *oc = a.out_col + (o - off0);
+        double *ov = a.out_val + (o - off0);
+        // S7 for CTA rows: one MSD pass (bucket by column within the row's column range), the
+        // packed keys (column << 14 | slot) staged in the row's own output value area, then each
+        // bucket sorted by one warp in registers.  A bucket over 512 entries (very clustered
+        // columns) sends the row to the general path: compaction + shared-memory bitonic.
+        const int P = min(64, max(1, (int)((n + 255) / 256)));
+        if (threadIdx.x < 64) s_cnt[threadIdx.x] = 0;
+        if (threadIdx.x == 0) {
+            s_mm[0] = INT_MAX;
+            s_mm[1] = -1;
+        }
+        __syncthreads();
+        {
+            int lmin = INT_MAX, lmax = -1, occ = 0;
+            for (int t = threadIdx.x; t < T; t += THREADS_B) {
+                const int32_t k = keys[t];
+                if (k != EMPTY) {
+                    lmin = min(lmin, k);
+                    lmax = max(lmax, k);
+                    ++occ;
+                }
+            }
+#pragma unroll
+            for (int d = 16; d > 0; d >>= 1) {
+                lmin = min(lmin, __shfl_xor_sync(FULLMASK, lmin, d));
+                lmax = max(lmax, __shfl_xor_sync(FULLMASK, lmax, d));
+                occ += __shfl_xor_sync(FULLMASK, occ, d);
+            }
+            if (lane == 0) {
+                atomicMin(&s_mm[0], lmin);
+                atomicMax(&s_mm[1], lmax);
+                s_occ[wid] = occ;
+            }
+        }
+        __syncthreads();
+        int occ_total = 0;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) occ_total += s_occ[w];
+        if (occ_total != n) {
+            if (threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
+            __syncthreads();
+            continue;
+        }
+        const int64_t lo = s_mm[0], span = (int64_t)s_mm[1] - lo + 1;
+        for (int t = threadIdx.x; t < T; t += THREADS_B) {
+            const int32_t k = keys[t];
+            if (k != EMPTY) atomicAdd(&s_cnt[(int)(((int64_t)k - lo) * P / span)], 1);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int run = 0, big = 0;
+            for (int b = 0; b < P; ++b) {
+                s_start[b] = run;
+                s_cur[b] = run;
+                run += s_cnt[b];
+                big = max(big, s_cnt[b]);
+            }
+            s_mm[2] = big;
+        }
+        __syncthreads();
+        if (s_mm[2] <= 512) {
+            unsigned long long *stage = reinterpret_cast<unsigned long long *>(ov);
+            for (int t = threadIdx.x; t < T; t += THREADS_B) {
+                const int32_t k = keys[t];
+                if (k != EMPTY) {
+                    const int pos = atomicAdd(&s_cur[(int)(((int64_t)k - lo) * P / span)], 1);
+                    stage[pos] = ((unsigned long long)(uint32_t)k << 14) | (unsigned)t;
+                }
+            }
+            __syncthreads();  // staged keys (global) visible to the block
+            for (int b = wid; b < P; b += NW) {
+                const int st = s_start[b], m = s_cnt[b];
+                if (m == 0) continue;
+                const int E = pow2_at_least((m + 31) / 32, 1);
+                const unsigned long long *pk = stage + st;
+                switch (E) {
+                    case 1: sort_emit<unsigned long long, 1, 14>(pk, m, vals, oc + st, ov + st); break;
+                    case 2: sort_emit<unsigned long long, 2, 14>(pk, m, vals, oc + st, ov + st); break;
+                    case 4: sort_emit<unsigned long long, 4, 14>(pk, m, vals, oc + st, ov + st); break;
+                    case 8: sort_emit<unsigned long long, 8, 14>(pk, m, vals, oc + st, ov + st); break;
+                    default: sort_emit<unsigned long long, 16, 14>(pk, m, vals, oc + st, ov + st); break;
+                }
+            }
+            __syncthreads();
+            continue;
+        }
+        // general path: in-place compaction + shared-memory bitonic sort
         int64_t cnt = 0;
         for (int t0 = 0; t0 < T; t0 += THREADS_B) {
             const int t = t0 + threadIdx.x;
@@ -751,17 +841,10 @@ __global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
             cnt += tot;
             __syncthreads();
         }
-        if (cnt != n) {
-            if (threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
-            __syncthreads();
-            continue;
-        }
         const int N = pow2_at_least(n, 32);
         for (int t = (int)n + threadIdx.x; t < N; t += THREADS_B) keys[t] = INT_MAX;
         __syncthreads();
         block_bitonic<THREADS_B>(keys, vals, N);
-        int32_t *oc = a.out_col + (o - off0);
-        double *ov = a.out_val + (o - off0);
         for (int t = threadIdx.x; t < n; t += THREADS_B) {
             oc[t] = keys[t];
             ov[t] = vals[t];
