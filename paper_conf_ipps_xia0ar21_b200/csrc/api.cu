@@ -157,8 +157,12 @@ struct spgemm_plan_s {
     bool a_alias = false;
     Ctl *ctl = nullptr;  // [0] count / symbolic passes, [1] numeric passes
 
-    uint32_t *gbits = nullptr;
+    uint32_t *gbits = nullptr, *gbits_sym = nullptr;
     double *gvals = nullptr;
+    int32_t *hkeys_num = nullptr, *hkeys_sym = nullptr;
+    double *hvals_num = nullptr;
+    int hblocks = 0;
+    int32_t *listH = nullptr, *listHn = nullptr;
     int64_t gstride_bits = 0, gstride_vals = 0;
     int gblocks = 0;
 
@@ -329,10 +333,14 @@ SymArgs sym_args(spgemm_plan_s *P, int64_t r0, int64_t r1, int tiers) {
     sa.r1 = r1;
     sa.listB = P->listB;
     sa.listG = P->listG;
+    sa.listH = P->listH;
     sa.ctl = P->ctl;
-    sa.gscratch = P->gbits;
+    sa.gscratch = P->gbits_sym;
     sa.gstride = P->gstride_bits;
     sa.gblocks = P->gblocks;
+    sa.hkeys = P->hkeys_sym;
+    sa.hstride = TH_SYM;
+    sa.hblocks = P->hblocks;
     sa.group = P->group;
     sa.tiers = tiers;
     return sa;
@@ -487,6 +495,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->listG = P->alloc<int32_t>(R, "listG");
     P->listBn = P->alloc<int32_t>(R, "numeric listB");
     P->listGn = P->alloc<int32_t>(R, "numeric listG");
+    P->listH = P->alloc<int32_t>(R, "listH");
+    P->listHn = P->alloc<int32_t>(R, "numeric listH");
     P->ctl = P->alloc<Ctl>(2, "ctl");
     P->tmp = P->alloc<int64_t>((R + SCAN_TILE - 1) / SCAN_TILE + 64, "scan scratch");
     CK(cudaMemsetAsync(P->ctl, 0, 2 * sizeof(Ctl), s));
@@ -512,23 +522,44 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->max_u = (int64_t)hc.max_u;
     P->max_bound = (int64_t)hc.max_bound;
 
-    // dense-tier scratch, sized only if a row can exceed the CTA tier
+    // arena-resident accumulator scratch, sized only if a row can exceed the CTA tier:
+    //   H (global hash, per CTA: TH_NUM keys + values for the numeric pass, TH_SYM keys for the
+    //   symbolic pass -- separate, so both passes may run concurrently on two streams) and
+    //   G (dense, per CTA: a bitmap for each pass + fp64 [ncols] for the numeric pass).
+    //   Together at most 1/4 of what is left after the smallest ring.
     if (P->max_bound > CAPB_NUM) {
         const int64_t nwords = (P->ncols + 31) / 32;
-        P->gstride_bits = (nwords + 63) & ~int64_t(63);
-        P->gstride_vals = (P->ncols + 31) & ~int64_t(31);
-        const size_t per = size_t(P->gstride_bits) * 4 + size_t(P->gstride_vals) * 8;
         const size_t ring_min = size_t(P->ring) * size_t(P->max_bound) * 12 + 4096;
         const size_t freeb = P->arena_bytes > P->used ? P->arena_bytes - P->used : 0;
-        const size_t avail = freeb > ring_min ? freeb - ring_min : 0;
-        int64_t nb = std::min<int64_t>(P->num_sms, int64_t((avail / 4) / per));
-        if (nb < 1) nb = int64_t(avail / per) >= 1 ? 1 : 0;
-        if (nb < 1) fail(SPGEMM_ERR_BUDGET, "budget cannot hold one dense accumulator for the longest row");
-        P->gblocks = (int)nb;
-        P->gbits = P->alloc<uint32_t>(P->gstride_bits * nb, "dense-tier bitmap");
-        P->gvals = P->alloc<double>(P->gstride_vals * nb, "dense-tier values");
-        CK(cudaMemsetAsync(P->gbits, 0, size_t(P->gstride_bits) * nb * 4, s));
-        CK(cudaMemsetAsync(P->gvals, 0, size_t(P->gstride_vals) * nb * 8, s));
+        const size_t avail = freeb > ring_min ? (freeb - ring_min) / 4 : 0;
+        // H
+        const size_t hper = size_t(TH_NUM) * 12 + size_t(TH_SYM) * 4;
+        int64_t nh = std::min<int64_t>(2 * P->num_sms, int64_t((avail / 2) / hper));
+        // G (always some: the H pass hands clustered rows to it)
+        P->gstride_bits = (nwords + 63) & ~int64_t(63);
+        P->gstride_vals = (P->ncols + 31) & ~int64_t(31);
+        const size_t gper = size_t(P->gstride_bits) * 8 + size_t(P->gstride_vals) * 8;
+        const size_t gavail = avail - size_t(std::max<int64_t>(nh, 0)) * hper;
+        const int64_t gwant = P->max_bound > CAPH_NUM ? P->num_sms : 8;
+        int64_t ng = std::min<int64_t>(gwant, int64_t(gavail / gper));
+        if (ng < 1) {
+            const size_t fb = P->arena_bytes > P->used + ring_min ? P->arena_bytes - P->used - ring_min : 0;
+            ng = fb >= gper ? 1 : 0;
+        }
+        if (ng < 1) fail(SPGEMM_ERR_BUDGET, "budget cannot hold one dense accumulator for the longest row");
+        P->gblocks = (int)ng;
+        P->gbits = P->alloc<uint32_t>(P->gstride_bits * ng, "dense-tier bitmap (numeric)");
+        P->gbits_sym = P->alloc<uint32_t>(P->gstride_bits * ng, "dense-tier bitmap (symbolic)");
+        P->gvals = P->alloc<double>(P->gstride_vals * ng, "dense-tier values");
+        CK(cudaMemsetAsync(P->gbits, 0, size_t(P->gstride_bits) * ng * 4, s));
+        CK(cudaMemsetAsync(P->gbits_sym, 0, size_t(P->gstride_bits) * ng * 4, s));
+        CK(cudaMemsetAsync(P->gvals, 0, size_t(P->gstride_vals) * ng * 8, s));
+        if (nh > 0) {
+            P->hblocks = (int)nh;
+            P->hkeys_num = P->alloc<int32_t>(TH_NUM * nh, "global-hash keys (numeric)");
+            P->hvals_num = P->alloc<double>(TH_NUM * nh, "global-hash values (numeric)");
+            P->hkeys_sym = P->alloc<int32_t>(TH_SYM * nh, "global-hash keys (symbolic)");
+        }
     }
 
     // ring capacity from what is left: each slot holds `cap` nonzeros (val fp64 + col int32)
@@ -606,9 +637,9 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         P->ev_tot.resize(nch);
         for (auto &e : P->ev_tot) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
         // the symbolic passes get their own stream so that chunk j+1's symbolic pass overlaps
-        // chunk j's numeric pass -- unless both would use the dense-tier scratch
+        // chunk j's numeric pass (the two passes have separate lists and arena scratch)
         const char *ser = getenv("SPGEMM_SERIAL_ANALYSIS");  // ablation knob
-        if (P->gblocks > 0 || (ser && ser[0] == '1')) {
+        if (ser && ser[0] == '1') {
             P->astream = P->stream;
         } else {
             CK(cudaStreamCreateWithFlags(&P->astream, cudaStreamNonBlocking));
@@ -679,12 +710,17 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t max_row_nnz, cu
     na.out_val = P->ring_val[b];
     na.listB = P->listBn;
     na.listG = P->listGn;
+    na.listH = P->listHn;
     na.ctl = P->ctl + 1;
     na.gbits = P->gbits;
     na.gvals = P->gvals;
     na.gstride_bits = P->gstride_bits;
     na.gstride_vals = P->gstride_vals;
     na.gblocks = P->gblocks;
+    na.hkeys = P->hkeys_num;
+    na.hvals = P->hvals_num;
+    na.hstride = TH_NUM;
+    na.hblocks = P->hblocks;
     na.group = P->group;
     na.tiers = num_tiers(max_row_nnz);
     launch_numeric(na, P->num_sms, P->stream, ev);

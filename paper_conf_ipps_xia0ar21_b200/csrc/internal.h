@@ -27,13 +27,19 @@ constexpr int THREADS_B = 512;
 constexpr int TB_SYM = 32768, CAPB_SYM = 24576;
 constexpr int TB_NUM = 16384, CAPB_NUM = 12288;
 constexpr int THREADS_G = 512;
+// H: one CTA, hash table in this CTA's arena slice (L2-resident for typical rows), same bucket sort
+constexpr int64_t TH_SYM = int64_t(1) << 20, CAPH_SYM = (TH_SYM / 4) * 3;
+constexpr int64_t TH_NUM = int64_t(1) << 19, CAPH_NUM = (TH_NUM / 4) * 3;
+constexpr int THREADS_H = 512;
+constexpr int HBUCKETS = 2048;             // max MSD buckets of an H row (<= 512 entries each)
 constexpr int ROW_BATCH = 16;              // rows a warp claims per atomic in the W kernels
 
 // Per-pass control block in the arena (zeroed with cudaMemsetAsync before each pass).
 struct Ctl {
     unsigned long long row_ctr;   // W kernels: next row batch                      } reset before
     unsigned int nB, nG;          // long-row list lengths                          } every pass
-    unsigned long long pass_max;  // symbolic: max nnz of a row in this pass        } (24 bytes)
+    unsigned long long pass_max;  // symbolic: max nnz of a row in this pass        } (32 bytes)
+    unsigned int nH, pad0;        // global-hash list length                        }
     unsigned int err;             // bit 0: numeric count mismatch; bit 1: invalid input; bit 2: table overflow
     unsigned int pad;
     unsigned long long sum_u;     // count pass: sum of products
@@ -60,20 +66,27 @@ struct SymArgs {
     const int64_t *bnd;  // per-row bound min(products, ncols) from the count pass
     int32_t *nnz;        // out: nnz of every row in [r0, r1)
     int64_t r0, r1;      // rows of this pass
-    int32_t *listB, *listG;
+    int32_t *listB, *listG, *listH;
     Ctl *ctl;
     uint32_t *gscratch;  // G tier: per-CTA bitmap of ceil(ncols/32) words, zero on entry and exit
     int64_t gstride;     // words per CTA slot
     int gblocks;         // CTAs in the G kernel
+    int32_t *hkeys;      // H tier: per-CTA key table of hstride slots
+    int64_t hstride;
+    int hblocks;
     int group;           // lanes per A entry in the W kernel (4, 8, 16, 32)
-    int tiers;           // bit 0: launch the CTA tier, bit 1: the dense tier (host knows when a
-                         // pass cannot have such rows, and skips those launches)
+    int tiers;           // bit 0: launch the CTA tier, bit 1: the dense tier, bit 2: the global-hash
+                         // tier (host knows when a pass cannot have such rows and skips launches)
     int batch;           // rows per claim in the W kernel (set by the launcher)
 };
 
 // tier bits for a pass whose rows have bound <= maxb
-inline int sym_tiers(int64_t maxb) { return (maxb > CAPW_SYM ? 1 : 0) | (maxb > CAPB_SYM ? 2 : 0); }
-inline int num_tiers(int64_t maxnnz) { return (maxnnz > CAPW_NUM ? 1 : 0) | (maxnnz > CAPB_NUM ? 2 : 0); }
+inline int sym_tiers(int64_t maxb) {
+    return (maxb > CAPW_SYM ? 1 : 0) | (maxb > CAPH_SYM ? 2 : 0) | (maxb > CAPB_SYM ? 4 : 0);
+}
+inline int num_tiers(int64_t maxnnz) {
+    return (maxnnz > CAPW_NUM ? 1 : 0) | (maxnnz > CAPH_NUM ? 2 : 0) | (maxnnz > CAPB_NUM ? 4 : 0);
+}
 
 // host2[0] = *end (a chunk's end offset), host2[1] = ctl->pass_max -- zero-copy stores into mapped
 // pinned memory, so no small D2H copy queues behind the big ones on the copy engine
@@ -107,12 +120,16 @@ struct NumArgs {
     int64_t r0, r1;      // chunk rows
     int32_t *out_col;    // ring slot: nnz of the chunk
     double *out_val;
-    int32_t *listB, *listG;
+    int32_t *listB, *listG, *listH;
     Ctl *ctl;
     uint32_t *gbits;     // G tier scratch: per CTA gstride_bits words of bitmap ...
     double *gvals;       // ... and gstride_vals doubles, all zero on entry and exit
     int64_t gstride_bits, gstride_vals;
     int gblocks;
+    int32_t *hkeys;      // H tier: per-CTA table of hstride slots (keys + values)
+    double *hvals;
+    int64_t hstride;
+    int hblocks;
     int group;
     int tiers;           // as in SymArgs
     int batch;

@@ -182,6 +182,72 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
     }
 }
 
+// ------------------------------------------------------------------ CTA product iterator (B/H/G)
+//
+// Visits every product of row i with a whole CTA, load-balanced: A entries are taken BATCH at a
+// time, a block scan of their B-row lengths flattens the products, and thread t handles products
+// t, t + NT, ...  (coalesced B loads), locating its A entry by binary search in shared memory.
+// One warp per A entry would leave the CTA waiting on the longest B row -- a hub row of a
+// power-law graph holds thousands of entries.
+constexpr int PBATCH = 1024;
+struct ProdSmem {
+    int64_t off[PBATCH + 1];
+    int64_t bs[PBATCH];
+    double a[PBATCH];
+    int64_t scan[40];
+};
+
+template <int NT, bool VALS, typename F>
+__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmem &sm,
+                                                   F &&f) {
+    constexpr int PER = PBATCH / NT;
+    const int64_t as = A.rp[i], ae = A.rp[i + 1];
+    for (int64_t pb = as; pb < ae; pb += PBATCH) {
+        const int nb = (int)(ae - pb < PBATCH ? ae - pb : PBATCH);
+        int64_t lens[PER];
+        int64_t sum = 0;
+#pragma unroll
+        for (int r = 0; r < PER; ++r) {
+            const int e = threadIdx.x * PER + r;
+            int64_t bs = 0, len = 0;
+            double av = 0.0;
+            if (e < nb) {
+                const int32_t k = __ldg(&A.col[pb + e]);
+                bs = __ldg(&B.rp[k]);
+                len = __ldg(&B.rp[k + 1]) - bs;
+                if (VALS) av = __ldg(&A.val[pb + e]);
+            }
+            if (e < PBATCH) {
+                sm.bs[e] = bs;
+                if (VALS) sm.a[e] = av;
+            }
+            lens[r] = len;
+            sum += len;
+        }
+        int64_t tot;
+        int64_t run = block_excl_scan<NT>(sum, sm.scan, &tot);
+#pragma unroll
+        for (int r = 0; r < PER; ++r) {
+            const int e = threadIdx.x * PER + r;
+            if (e < nb) sm.off[e] = run;
+            run += lens[r];
+        }
+        if (threadIdx.x == 0) sm.off[nb] = tot;
+        __syncthreads();
+        for (int64_t q = threadIdx.x; q < tot; q += NT) {
+            int lo = 0, hi = nb;  // invariant: off[lo] <= q < off[hi]
+            while (hi - lo > 1) {
+                const int mid = (lo + hi) >> 1;
+                if (sm.off[mid] <= q) lo = mid;
+                else hi = mid;
+            }
+            const int64_t pos = sm.bs[lo] + (q - sm.off[lo]);
+            f(__ldg(&B.col[pos]), VALS ? sm.a[lo] * __ldg(&B.val[pos]) : 0.0);
+        }
+        __syncthreads();
+    }
+}
+
 // find-or-insert of a column in a warp-private table; returns the slot
 __device__ __forceinline__ uint32_t find_slot(int32_t *keys, int32_t c, int lg) {
     const uint32_t mask = (1u << lg) - 1;
@@ -267,11 +333,16 @@ __global__ void k_add(int64_t *rp, int64_t n, int64_t d) {
 
 // ------------------------------------------------------------------------ tier classification
 
-__device__ __forceinline__ void push_long(int64_t i, int64_t bound, int64_t capB, int32_t *listB, int32_t *listG,
-                                          Ctl *ctl) {
+// rows too long for a warp: CTA tier (shared-memory hash) up to capB, global-hash tier up to capH
+// (when that tier has scratch), dense tier beyond
+__device__ __forceinline__ void push_long(int64_t i, int64_t bound, int64_t capB, int64_t capH, bool have_h,
+                                          int32_t *listB, int32_t *listH, int32_t *listG, Ctl *ctl) {
     if (bound <= capB) {
         unsigned idx = atomicAdd(&ctl->nB, 1u);
         listB[idx] = (int32_t)i;
+    } else if (have_h && bound <= capH) {
+        unsigned idx = atomicAdd(&ctl->nH, 1u);
+        listH[idx] = (int32_t)i;
     } else {
         unsigned idx = atomicAdd(&ctl->nG, 1u);
         listG[idx] = (int32_t)i;
@@ -307,7 +378,7 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
             }
             if (bound > CAPW_SYM) {
                 if (lane == 0) {
-                    push_long(i, bound, CAPB_SYM, a.listB, a.listG, a.ctl);
+                    push_long(i, bound, CAPB_SYM, CAPH_SYM, a.hblocks > 0, a.listB, a.listH, a.listG, a.ctl);
                     nlong++;
                 }
                 continue;
@@ -343,8 +414,7 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
 __global__ void __launch_bounds__(THREADS_B) k_sym_b(SymArgs a) {
     extern __shared__ int32_t keys[];
     __shared__ int64_t s_scan[40];
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    constexpr int NW = THREADS_B / 32;
+    __shared__ ProdSmem psm;
     constexpr int MAXLG = 15;  // log2(TB_SYM)
     const unsigned n = *(volatile unsigned *)&a.ctl->nB;
     for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
@@ -355,12 +425,8 @@ __global__ void __launch_bounds__(THREADS_B) k_sym_b(SymArgs a) {
         for (int t = threadIdx.x; t < T; t += THREADS_B) keys[t] = EMPTY;
         __syncthreads();
         int cnt = 0;
-        const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
-        for (int64_t p = as + wid; p < ae; p += NW) {
-            const int32_t k = __ldg(&a.A.col[p]);
-            const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
-            for (int64_t q = bs + lane; q < be; q += 32) cnt += sym_insert(keys, __ldg(&a.B.col[q]), lg);
-        }
+        block_row_products<THREADS_B, false>(a.A, a.B, i, psm,
+                                             [&](int32_t c, double) { cnt += sym_insert(keys, c, lg); });
         int64_t tot;
         block_excl_scan<THREADS_B>(cnt, s_scan, &tot);
         if (threadIdx.x == 0) {
@@ -380,25 +446,18 @@ __global__ void __launch_bounds__(THREADS_B) k_sym_b(SymArgs a) {
 
 __global__ void __launch_bounds__(THREADS_G) k_sym_g(SymArgs a) {
     __shared__ int64_t s_scan[40];
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    constexpr int NW = THREADS_G / 32;
+    __shared__ ProdSmem psm;
     uint32_t *bm = a.gscratch + (int64_t)blockIdx.x * a.gstride;
     const unsigned n = *(volatile unsigned *)&a.ctl->nG;
     const int64_t nwords = (a.B.ncols + 31) / 32;
     for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
         const int64_t i = a.listG[idx];
         int cnt = 0;
-        const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
-        for (int64_t p = as + wid; p < ae; p += NW) {
-            const int32_t k = __ldg(&a.A.col[p]);
-            const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
-            for (int64_t q = bs + lane; q < be; q += 32) {
-                const int32_t c = __ldg(&a.B.col[q]);
-                const uint32_t bit = 1u << (c & 31);
-                const uint32_t old = atomicOr(&bm[c >> 5], bit);
-                cnt += (old & bit) ? 0 : 1;
-            }
-        }
+        block_row_products<THREADS_G, false>(a.A, a.B, i, psm, [&](int32_t c, double) {
+            const uint32_t bit = 1u << (c & 31);
+            const uint32_t old = atomicOr(&bm[c >> 5], bit);
+            cnt += (old & bit) ? 0 : 1;
+        });
         int64_t tot;
         block_excl_scan<THREADS_G>(cnt, s_scan, &tot);
         if (threadIdx.x == 0) {
@@ -409,11 +468,7 @@ __global__ void __launch_bounds__(THREADS_G) k_sym_g(SymArgs a) {
         }
         // clear (block_excl_scan ended with a barrier, so all atomics of this row are done)
         if (a.bnd[i] < nwords) {  // bnd = min(products, ncols): re-walk only when cheaper than a sweep
-            for (int64_t p = as + wid; p < ae; p += NW) {
-                const int32_t k = __ldg(&a.A.col[p]);
-                const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
-                for (int64_t q = bs + lane; q < be; q += 32) bm[__ldg(&a.B.col[q]) >> 5] = 0u;
-            }
+            block_row_products<THREADS_G, false>(a.A, a.B, i, psm, [&](int32_t c, double) { bm[c >> 5] = 0u; });
         } else {
             for (int64_t w = threadIdx.x; w < nwords; w += THREADS_G) bm[w] = 0u;
         }
@@ -585,14 +640,16 @@ __device__ __forceinline__ void reg_bitonic(K (&x)[E]) {
 // load n packed keys (column << SB | slot) from smem or global memory, sort them in registers and
 // write the row out in column order: col from the key, value gathered from its hash slot in
 // shared memory (S7, §II-B).  pk may alias ov: all loads complete before any store.
-template <typename K, int E, int SB = 9>
+// PK_G / V_G: keys / values live in global memory and are read at L2 (ld.cg): they were written
+// or atomically updated in this row, possibly through other SMs' stale L1 views.
+template <typename K, int E, int SB = 9, bool PK_G = false, bool V_G = false>
 __device__ __forceinline__ void sort_emit(const K *pk, int n, const double *vals, int32_t *oc, double *ov) {
     const int lane = threadIdx.x & 31;
     K x[E];
 #pragma unroll
     for (int r = 0; r < E; ++r) {
         const int e = (r << 5) | lane;
-        x[r] = e < n ? pk[e] : ~K(0);
+        x[r] = e < n ? (PK_G ? __ldcg(pk + e) : pk[e]) : ~K(0);
     }
     __syncwarp();
     reg_bitonic<K, E>(x);
@@ -601,8 +658,23 @@ __device__ __forceinline__ void sort_emit(const K *pk, int n, const double *vals
         const int e = (r << 5) | lane;
         if (e < n) {
             oc[e] = (int32_t)(x[r] >> SB);
-            ov[e] = vals[(int)(x[r] & ((1u << SB) - 1u))];
+            const int slot = (int)(x[r] & ((K(1) << SB) - 1u));
+            ov[e] = V_G ? __ldcg(vals + slot) : vals[slot];
         }
+    }
+}
+
+// one warp sorts and emits a bucket of m packed keys (E chosen from m <= 512)
+template <int SB, bool PK_G, bool V_G>
+__device__ __forceinline__ void sort_emit_any(const unsigned long long *pk, int m, const double *vals, int32_t *oc,
+                                              double *ov) {
+    const int E = pow2_at_least((m + 31) / 32, 1);
+    switch (E) {
+        case 1: sort_emit<unsigned long long, 1, SB, PK_G, V_G>(pk, m, vals, oc, ov); break;
+        case 2: sort_emit<unsigned long long, 2, SB, PK_G, V_G>(pk, m, vals, oc, ov); break;
+        case 4: sort_emit<unsigned long long, 4, SB, PK_G, V_G>(pk, m, vals, oc, ov); break;
+        case 8: sort_emit<unsigned long long, 8, SB, PK_G, V_G>(pk, m, vals, oc, ov); break;
+        default: sort_emit<unsigned long long, 16, SB, PK_G, V_G>(pk, m, vals, oc, ov); break;
     }
 }
 
@@ -631,7 +703,7 @@ __global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
             const int64_t n = a.crp[i + 1] - o;
             if (n == 0) continue;
             if (n > CAPW_NUM) {
-                if (lane == 0) push_long(i, n, CAPB_NUM, a.listB, a.listG, a.ctl);
+                if (lane == 0) push_long(i, n, CAPB_NUM, CAPH_NUM, a.hblocks > 0, a.listB, a.listH, a.listG, a.ctl);
                 continue;
             }
             const int lg = table_log2(n, MAXLG);
@@ -712,6 +784,7 @@ __global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
     double *vals = smem_d;
     int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);
     __shared__ int64_t s_scan[40];
+    __shared__ ProdSmem psm;
     __shared__ int s_cnt[64], s_cur[64], s_start[64], s_mm[3], s_occ[THREADS_B / 32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     constexpr int NW = THREADS_B / 32;
@@ -729,15 +802,8 @@ __global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
             vals[t] = 0.0;
         }
         __syncthreads();
-        const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
-        for (int64_t p = as + wid; p < ae; p += NW) {
-            const int32_t k = __ldg(&a.A.col[p]);
-            const double av = __ldg(&a.A.val[p]);
-            const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
-            for (int64_t q = bs + lane; q < be; q += 32)
-                num_insert(keys, vals, __ldg(&a.B.col[q]), av * __ldg(&a.B.val[q]), lg);
-        }
-        __syncthreads();
+        block_row_products<THREADS_B, true>(a.A, a.B, i, psm,
+                                            [&](int32_t c, double v) { num_insert(keys, vals, c, v, lg); });
         int32_t *oc = a.out_col + (o - off0);
         double *ov = a.out_val + (o - off0);
         // S7 for CTA rows: one MSD pass (bucket by column within the row's column range), the
@@ -812,15 +878,7 @@ __global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
             for (int b = wid; b < P; b += NW) {
                 const int st = s_start[b], m = s_cnt[b];
                 if (m == 0) continue;
-                const int E = pow2_at_least((m + 31) / 32, 1);
-                const unsigned long long *pk = stage + st;
-                switch (E) {
-                    case 1: sort_emit<unsigned long long, 1, 14>(pk, m, vals, oc + st, ov + st); break;
-                    case 2: sort_emit<unsigned long long, 2, 14>(pk, m, vals, oc + st, ov + st); break;
-                    case 4: sort_emit<unsigned long long, 4, 14>(pk, m, vals, oc + st, ov + st); break;
-                    case 8: sort_emit<unsigned long long, 8, 14>(pk, m, vals, oc + st, ov + st); break;
-                    default: sort_emit<unsigned long long, 16, 14>(pk, m, vals, oc + st, ov + st); break;
-                }
+                sort_emit_any<14, true, false>(stage + st, m, vals, oc + st, ov + st);
             }
             __syncthreads();
             continue;
@@ -853,6 +911,193 @@ __global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
     }
 }
 
+// ----------------------------------------------------------------- S4 / S6, global-hash tier H
+// CTA per row, open-addressing table (int32 keys, fp64 values) in this CTA's arena slice, sized
+// per row (load <= 3/4).  Rows of a few 10^4 .. 10^5 nonzeros keep their table in L2.  The numeric
+// pass sorts like the CTA tier: one MSD bucket pass over the row's column range, keys staged in
+// the row's own output, a register sort per bucket; a row whose buckets overflow (clustered
+// columns) is handed to the dense tier, which runs after this kernel.
+
+__device__ __forceinline__ int sym_insert_g(int32_t *keys, int32_t c, int lg) {
+    const uint32_t mask = (1u << lg) - 1;
+    uint32_t h = hslot(c, lg);
+    while (true) {
+        const int32_t k = __ldcg(keys + h);
+        if (k == c) return 0;
+        if (k == EMPTY) {
+            const int32_t old = atomicCAS(&keys[h], EMPTY, c);
+            if (old == EMPTY) return 1;
+            if (old == c) return 0;
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+__global__ void __launch_bounds__(THREADS_H) k_sym_h(SymArgs a) {
+    __shared__ int64_t s_scan[40];
+    __shared__ ProdSmem psm;
+    int32_t *keys = a.hkeys + (int64_t)blockIdx.x * a.hstride;
+    const unsigned nrows = *(volatile unsigned *)&a.ctl->nH;
+    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
+        const int64_t i = a.listH[idx];
+        const int lg = table_log2(a.bnd[i], 20);
+        const int T = 1 << lg;
+        int4 *k4 = reinterpret_cast<int4 *>(keys);
+        for (int t = threadIdx.x; t < (T >> 2); t += THREADS_H) k4[t] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
+        __syncthreads();
+        int cnt = 0;
+        block_row_products<THREADS_H, false>(a.A, a.B, i, psm,
+                                             [&](int32_t c, double) { cnt += sym_insert_g(keys, c, lg); });
+        int64_t tot;
+        block_excl_scan<THREADS_H>(cnt, s_scan, &tot);
+        if (threadIdx.x == 0) {
+            a.nnz[i] = (int32_t)tot;
+            atomicMax(&a.ctl->max_nnz, (unsigned long long)tot);
+            atomicMax(&a.ctl->pass_max, (unsigned long long)tot);
+            atomicAdd(&a.ctl->rows_g, 1ull);
+        }
+        __syncthreads();
+    }
+}
+
+__global__ void __launch_bounds__(THREADS_H) k_num_h(NumArgs a) {
+    __shared__ int64_t s_scan[40];
+    __shared__ ProdSmem psm;
+    // bucket counts and cursors; a bucket's start is its cursor minus its count after the scatter
+    __shared__ int s_cnt[HBUCKETS], s_cur[HBUCKETS], s_mm[3], s_occ[THREADS_H / 32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    constexpr int NW = THREADS_H / 32;
+    int32_t *keys = a.hkeys + (int64_t)blockIdx.x * a.hstride;
+    double *vals = a.hvals + (int64_t)blockIdx.x * a.hstride;
+    const unsigned nrows = *(volatile unsigned *)&a.ctl->nH;
+    const int64_t off0 = a.crp[a.r0];
+    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
+        const int64_t i = a.listH[idx];
+        const int64_t o = a.crp[i];
+        const int n = (int)(a.crp[i + 1] - o);
+        const int lg = table_log2(n, 19);
+        const int T = 1 << lg;
+        {
+            int4 *k4 = reinterpret_cast<int4 *>(keys);
+            double2 *v2 = reinterpret_cast<double2 *>(vals);
+            for (int t = threadIdx.x; t < (T >> 2); t += THREADS_H) k4[t] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
+            for (int t = threadIdx.x; t < (T >> 1); t += THREADS_H) v2[t] = make_double2(0.0, 0.0);
+        }
+        const int P = min(HBUCKETS, max(1, (n + 255) / 256));
+        for (int b = threadIdx.x; b < P; b += THREADS_H) s_cnt[b] = 0;
+        if (threadIdx.x == 0) {
+            s_mm[0] = INT_MAX;
+            s_mm[1] = -1;
+        }
+        __syncthreads();
+        block_row_products<THREADS_H, true>(a.A, a.B, i, psm, [&](int32_t c, double v) {
+            const uint32_t mask = (1u << lg) - 1;
+            uint32_t h = hslot(c, lg);
+            while (true) {
+                const int32_t kk = __ldcg(keys + h);
+                if (kk == c) break;
+                if (kk == EMPTY) {
+                    const int32_t old = atomicCAS(&keys[h], EMPTY, c);
+                    if (old == EMPTY || old == c) break;
+                }
+                h = (h + 1) & mask;
+            }
+            atomicAdd(&vals[h], v);
+        });
+        int32_t *oc = a.out_col + (o - off0);
+        double *ov = a.out_val + (o - off0);
+        {
+            int lmin = INT_MAX, lmax = -1, occ = 0;
+            for (int t = threadIdx.x; t < T; t += THREADS_H) {
+                const int32_t k = __ldcg(keys + t);
+                if (k != EMPTY) {
+                    lmin = min(lmin, k);
+                    lmax = max(lmax, k);
+                    ++occ;
+                }
+            }
+#pragma unroll
+            for (int d = 16; d > 0; d >>= 1) {
+                lmin = min(lmin, __shfl_xor_sync(FULLMASK, lmin, d));
+                lmax = max(lmax, __shfl_xor_sync(FULLMASK, lmax, d));
+                occ += __shfl_xor_sync(FULLMASK, occ, d);
+            }
+            if (lane == 0) {
+                atomicMin(&s_mm[0], lmin);
+                atomicMax(&s_mm[1], lmax);
+                s_occ[wid] = occ;
+            }
+        }
+        __syncthreads();
+        int occ_total = 0;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) occ_total += s_occ[w];
+        if (occ_total != n) {
+            if (threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
+            __syncthreads();
+            continue;
+        }
+        const int64_t lo = s_mm[0], span = (int64_t)s_mm[1] - lo + 1;
+        for (int t = threadIdx.x; t < T; t += THREADS_H) {
+            const int32_t k = __ldcg(keys + t);
+            if (k != EMPTY) atomicAdd(&s_cnt[(int)(((int64_t)k - lo) * P / span)], 1);
+        }
+        __syncthreads();
+        {   // bucket starts: block scan over P <= HBUCKETS counts, 4 per thread
+            constexpr int PER = HBUCKETS / THREADS_H;
+            int loc[PER], sum = 0;
+#pragma unroll
+            for (int k = 0; k < PER; ++k) {
+                const int b = threadIdx.x * PER + k;
+                loc[k] = b < P ? s_cnt[b] : 0;
+                sum += loc[k];
+            }
+            int64_t tot;
+            int run = (int)block_excl_scan<THREADS_H>(sum, s_scan, &tot);
+#pragma unroll
+            for (int k = 0; k < PER; ++k) {
+                const int b = threadIdx.x * PER + k;
+                if (b < P) s_cur[b] = run;
+                run += loc[k];
+            }
+        }
+        if (threadIdx.x == 0) s_mm[2] = 0;
+        __syncthreads();
+        {
+            int big = 0;
+            for (int b = threadIdx.x; b < P; b += THREADS_H) big = max(big, s_cnt[b]);
+#pragma unroll
+            for (int d = 16; d > 0; d >>= 1) big = max(big, __shfl_xor_sync(FULLMASK, big, d));
+            if (lane == 0) atomicMax(&s_mm[2], big);
+        }
+        __syncthreads();
+        if (s_mm[2] > 512) {
+            // clustered columns: the dense tier (launched after this kernel) takes the row
+            if (threadIdx.x == 0) {
+                const unsigned gi = atomicAdd(&a.ctl->nG, 1u);
+                a.listG[gi] = (int32_t)i;
+            }
+            __syncthreads();
+            continue;
+        }
+        unsigned long long *stage = reinterpret_cast<unsigned long long *>(ov);
+        for (int t = threadIdx.x; t < T; t += THREADS_H) {
+            const int32_t k = __ldcg(keys + t);
+            if (k != EMPTY) {
+                const int pos = atomicAdd(&s_cur[(int)(((int64_t)k - lo) * P / span)], 1);
+                stage[pos] = ((unsigned long long)(uint32_t)k << 20) | (unsigned)t;
+            }
+        }
+        __syncthreads();
+        for (int b = wid; b < P; b += NW) {
+            const int m = s_cnt[b], st = s_cur[b] - m;
+            if (m == 0) continue;
+            sort_emit_any<20, true, true>(stage + st, m, vals, oc + st, ov + st);
+        }
+        __syncthreads();
+    }
+}
+
 // ------------------------------------------------------------------------------ S6 numeric, G
 // Dense accumulation over all columns (§II-B): bitmap for structure (values may cancel to
 // 0.0 and must still be stored), fp64 array for values, in this CTA's arena slot.  Output is
@@ -860,8 +1105,7 @@ __global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
 
 __global__ void __launch_bounds__(THREADS_G) k_num_g(NumArgs a) {
     __shared__ int64_t s_scan[40];
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    constexpr int NW = THREADS_G / 32;
+    __shared__ ProdSmem psm;
     uint32_t *bm = a.gbits + (int64_t)blockIdx.x * a.gstride_bits;
     double *dv = a.gvals + (int64_t)blockIdx.x * a.gstride_vals;
     const unsigned nrows = *(volatile unsigned *)&a.ctl->nG;
@@ -871,18 +1115,10 @@ __global__ void __launch_bounds__(THREADS_G) k_num_g(NumArgs a) {
         const int64_t i = a.listG[idx];
         const int64_t o = a.crp[i];
         const int64_t n = a.crp[i + 1] - o;
-        const int64_t as = a.A.rp[i], ae = a.A.rp[i + 1];
-        for (int64_t p = as + wid; p < ae; p += NW) {
-            const int32_t k = __ldg(&a.A.col[p]);
-            const double av = __ldg(&a.A.val[p]);
-            const int64_t bs = __ldg(&a.B.rp[k]), be = __ldg(&a.B.rp[k + 1]);
-            for (int64_t q = bs + lane; q < be; q += 32) {
-                const int32_t c = __ldg(&a.B.col[q]);
-                atomicOr(&bm[c >> 5], 1u << (c & 31));
-                atomicAdd(&dv[c], av * __ldg(&a.B.val[q]));
-            }
-        }
-        __syncthreads();
+        block_row_products<THREADS_G, true>(a.A, a.B, i, psm, [&](int32_t c, double v) {
+            atomicOr(&bm[c >> 5], 1u << (c & 31));
+            atomicAdd(&dv[c], v);
+        });
         int32_t *oc = a.out_col + (o - off0);
         double *ov = a.out_val + (o - off0);
         int64_t cnt = 0;
@@ -1034,7 +1270,7 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
     int dev = 0;
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
-    cudaMemsetAsync(&a.ctl->row_ctr, 0, 24, s);  // row_ctr, nB, nG, pass_max
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);  // row_ctr, nB, nG, pass_max, nH
     SymArgs aw = a;
     aw.batch = batch_for(rows, g.symw_blocks);
     const int wblocks = grid_for(rows, WARPS_W * aw.batch, g.symw_blocks);
@@ -1051,7 +1287,11 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
         LAUNCHED(1);
     }
     rec(ev, 2, s);
-    if ((a.tiers & 2) && a.gblocks > 0) {
+    if ((a.tiers & 4) && a.hblocks > 0) {
+        k_sym_h<<<a.hblocks, THREADS_H, 0, s>>>(a);
+        LAUNCHED(1);
+    }
+    if (((a.tiers & 2) || ((a.tiers & 4) && a.hblocks == 0)) && a.gblocks > 0) {
         k_sym_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
         LAUNCHED(1);
     }
@@ -1067,7 +1307,7 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
     int dev = 0;
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
-    cudaMemsetAsync(&a.ctl->row_ctr, 0, 24, s);
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);
     NumArgs aw = a;
     aw.batch = batch_for(rows, g.numw_blocks);
     const int wblocks = grid_for(rows, WARPS_W * aw.batch, g.numw_blocks);
@@ -1084,7 +1324,14 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
         LAUNCHED(1);
     }
     rec(ev, 2, s);
-    if ((a.tiers & 2) && a.gblocks > 0) {
+    const bool h = (a.tiers & 4) && a.hblocks > 0;
+    if (h) {
+        k_num_h<<<a.hblocks, THREADS_H, 0, s>>>(a);
+        LAUNCHED(1);
+    }
+    // the dense tier also takes H rows whose buckets overflowed, and every long row when the
+    // H tier has no scratch
+    if (((a.tiers & 2) || (a.tiers & 4)) && a.gblocks > 0) {
         k_num_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
         LAUNCHED(1);
     }

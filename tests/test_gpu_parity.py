@@ -150,6 +150,35 @@ def test_tiers_warp_block_global():
     assert_parity(A, B, rp, col, val)
 
 
+def _csr_from_rows(rows, ncols, rng):
+    rp = np.zeros(len(rows) + 1, np.int64)
+    np.cumsum([len(r) for r in rows], out=rp[1:])
+    col = np.concatenate(rows).astype(np.int32) if rows else np.zeros(0, np.int32)
+    return W.CSR(len(rows), ncols, rp, col, rng.uniform(-1, 1, len(col)))
+
+
+@pytest.mark.parametrize("fused", [False, True])
+def test_global_hash_tier_fallback_and_dense_tier(fused):
+    """Rows for the arena tiers: a clustered H-tier row (its MSD buckets overflow, so the dense tier
+    takes it), a scattered H-tier row, and a row beyond the H tier (dense tier directly)."""
+    rng = np.random.default_rng(17)
+    ncols = 1_000_000
+    brows = []
+    for k in range(30):                      # clustered in [0, 50000) + one far outlier
+        brows.append(np.append(np.sort(rng.choice(50_000, 1000, replace=False)), ncols - 1))
+    for k in range(40):                      # scattered
+        brows.append(np.sort(rng.choice(ncols, 1000, replace=False)))
+    for k in range(600):                     # long scattered rows for the dense tier
+        brows.append(np.sort(rng.choice(ncols, 1500, replace=False)))
+    B = _csr_from_rows(brows, ncols, rng)
+    arows = [np.arange(0, 30), np.arange(30, 70), np.arange(70, 670), np.array([3, 40, 100])]
+    A = _csr_from_rows(arows, B.nrows, rng)
+    r = run_fused(A, B) if fused else run(A, B)
+    info = r[3]
+    assert info["rows_global"] >= 3, info
+    assert_parity(A, B, r[0], r[1], r[2])
+
+
 @pytest.mark.parametrize("fused", [False, True])
 def test_wide_column_space(fused):
     """ncols > 2^23: the numeric sort switches to 64-bit packed keys (column << 9 | slot)."""

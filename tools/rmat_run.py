@@ -18,7 +18,10 @@ from paper_conf_ipps_xia0ar21_b200 import capi
 scale = int(os.environ.get("SCALE", "22"))
 frac = float(os.environ.get("ROWS_FRAC", "1"))
 t0 = time.perf_counter()
-A = W.rmat(scale, 16)
+if os.environ.get("GEN", "numpy") == "torch":
+    A = W.rmat_torch(scale, 16)
+else:
+    A = W.rmat(scale, 16)
 gen_s = time.perf_counter() - t0
 dev = torch.device("cuda", 0)
 

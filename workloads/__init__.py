@@ -199,8 +199,9 @@ def rmat_torch(scale: int, edge_factor: int = 16, a=0.45, b=0.20, c=0.20, seed: 
             q = (q << 1) | cbit.to(torch.int64)
         del u
     nr, nc = 1 << rs, 1 << cs
-    r = torch.randperm(nr, generator=g, device=device)[r]
-    q = torch.randperm(nc, generator=g, device=device)[q]
+    pr = torch.randperm(nr, generator=g, device=device)
+    pc = pr if rs == cs else torch.randperm(nc, generator=g, device=device)  # square: relabel vertices
+    r, q = pr[r], pc[q]
     if symmetric and rs == cs:
         keep = r != q
         r, q = r[keep], q[keep]
