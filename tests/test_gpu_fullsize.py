@@ -83,6 +83,55 @@ def test_c2_full_size_budget_2gib():
     assert oracle.compare(gp, col[idx], val[idx], E)["ok"]
 
 
+def _streamed_panel_check(A, B, r1, picks_per_chunk=2, chunk_nnz=300_000_000, seed=7):
+    """Stream rows [0, r1) of C = A*B through the sink (fused plan, ring 3), keep a few sampled rows
+    per chunk, and check them against the oracle in one call at the end."""
+    dev = torch.device("cuda", 0)
+    dA = _device_csr(A, dev)
+    dB = dA if B is A else _device_csr(B, dev)
+    rng = np.random.default_rng(seed)
+    kept = []
+    seen = {"rows": 0, "nnz": 0, "chunks": 0}
+
+    def sink(r0, r1_, rp, col, val):
+        seen["chunks"] += 1
+        seen["rows"] += r1_ - r0
+        seen["nnz"] += int(rp[-1])
+        for r in sorted({r0, r1_ - 1} | set(rng.integers(r0, r1_, picks_per_chunk).tolist())):
+            lr = r - r0
+            kept.append((r, col[rp[lr]:rp[lr + 1]].copy(), val[rp[lr]:rp[lr + 1]].copy()))
+
+    o = capi.opts(fused=True, ring=3, chunk_nnz=chunk_nnz, row_end=r1)
+    with capi.Plan(dA, dB, 0, o) as P:
+        P.execute_stream(sink)
+        info = P.info()
+    assert seen["rows"] == r1 and seen["nnz"] == info["nnz"] and seen["chunks"] == info["num_chunks"]
+    rows = np.array([k[0] for k in kept])
+    E = oracle.spgemm(A, B, rows=rows)
+    gp = np.concatenate([[0], np.cumsum([len(k[1]) for k in kept])])
+    res = oracle.compare(gp, np.concatenate([k[1] for k in kept]), np.concatenate([k[2] for k in kept]), E)
+    assert res["ok"], res
+    return info
+
+
+@pytest.mark.skipif(os.environ.get("SPGEMM_SKIP_C45") == "1", reason="C4/C5 panel runs disabled")
+def test_c4_rmat_s24_rank_panel():
+    """configs[3] (R-MAT s24 ef16, C several TB) -- the row panel one rank of an 8-GPU deal owns."""
+    A = W.rmat_torch(24, 16, seed=20210518)
+    info = _streamed_panel_check(A, A, A.nrows // 8)
+    assert info["rows_global"] > 0
+
+
+@pytest.mark.skipif(os.environ.get("SPGEMM_SKIP_C45") == "1", reason="C4/C5 panel runs disabled")
+def test_c5_rectangular_rank_panel():
+    """configs[4]: A = 2^24 x 2^22 power-law, B = 2^22 x 2^24 (2^28 generated edges each), rank 0's
+    panel of an 8-GPU deal."""
+    A = W.rmat_torch(24, col_scale=22, nedges=1 << 28, seed=11, symmetric=False)
+    B = W.rmat_torch(22, col_scale=24, nedges=1 << 28, seed=12, symmetric=False)
+    assert A.nnz + B.nnz > 4e8
+    _streamed_panel_check(A, B, A.nrows // 8)
+
+
 @pytest.mark.skipif(os.environ.get("SPGEMM_SKIP_C3") == "1", reason="C3 full-size run disabled")
 def test_c3_rmat_s22_streamed():
     """configs[2] at full size: ~2.9e10 products, C of ~0.3 TB streamed through the sink; in every

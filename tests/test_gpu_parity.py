@@ -298,6 +298,21 @@ def test_device_inputs_with_base_and_row_panels():
     assert np.array_equal(np.concatenate([p[0] for p in parts]), full[1])
 
 
+def test_no_leak_across_plans():
+    """Library-owned arenas, streams, events and pinned staging are released by spgemm_free."""
+    A = W.rmat(11, 8, seed=3)
+    torch.cuda.synchronize()
+    for _ in range(2):  # warm the process-wide caches
+        with capi.Plan(A, A, 256 << 20, capi.opts(fused=True, chunk_nnz=20000)) as P:
+            P.execute_stream(lambda *a: 0)
+    free0 = torch.cuda.mem_get_info()[0]
+    for k in range(12):
+        with capi.Plan(A, A, 256 << 20, capi.opts(fused=bool(k & 1), chunk_nnz=20000, ring=1 + k % 3)) as P:
+            P.execute_stream(lambda *a: 0)
+    torch.cuda.synchronize()
+    assert abs(torch.cuda.mem_get_info()[0] - free0) < (8 << 20)
+
+
 def test_workspace_from_torch():
     A = W.stencil_3d27(12)
     ws = torch.empty(64 << 20, dtype=torch.uint8, device="cuda")
