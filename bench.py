@@ -65,6 +65,8 @@ class Clocks:
         self.gpu, self.rows, self.p = gpu, [], None
 
     def __enter__(self):
+        if os.environ.get("BENCH_CLOCKS", "1") == "0":  # diagnostic: no sampler process
+            return self
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
                                        "--format=csv,noheader,nounits", "-lms", "100"],
@@ -102,6 +104,33 @@ class Clocks:
                         reasons.add(nm)
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
                 "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def probe_d2h(h_dst, dev, nbytes=1 << 30, reps=3):
+    """This box's pinned D2H rate (GB/s), measured in this process just before the timed region:
+    one cudaMemcpyAsync of up to 1 GiB from HBM into the bench's own pinned output buffer, best
+    of `reps` (CUDA events on a side stream).  The link bound of the step is judged against it."""
+    import torch
+    hb = h_dst.view(torch.uint8)
+    n = min(nbytes, hb.numel())
+    if n < (1 << 20):
+        return None
+    src = torch.empty(n, dtype=torch.uint8, device=dev)
+    src.fill_(7)
+    s = torch.cuda.Stream(device=dev)
+    best = None
+    for _ in range(reps):
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(s):
+            e0.record(s)
+            hb[:n].copy_(src, non_blocking=True)
+            e1.record(s)
+        s.synchronize()
+        t = e0.elapsed_time(e1) / 1e3
+        best = t if best is None else min(best, t)
+    del src
+    return n / best / 1e9
 
 
 def dist_env():
@@ -281,8 +310,14 @@ def main():
 
     chunk_table = {}
 
-    def step(profile=False):
+    host_ms = {"plan": [], "execute": [], "free": []}
+
+    def step(profile=False, keep=False):
+        """One multiply (plan + execute + free).  keep: return the plan unfreed, so that its
+        kernel times (CUDA events recorded inside the step) are read after the timed region."""
+        h0 = time.perf_counter()
         P = capi.Plan(dA, dB, wbytes, mk_opts(profile))
+        h1 = time.perf_counter()
         if fused:
             z = P.execute_capacity(h_rp, h_col, h_val, nnz_local)
             if world > 1:
@@ -293,12 +328,14 @@ def main():
                 b, _ = pdist.slice_bases(P.info()["nnz"], device=cdev)
                 P.set_row_ptr_base(b)
             P.execute_into(h_rp, h_col, h_val)
-        st = P.stats() if profile else None
-        if profile and "rows" not in chunk_table:
-            chunk_table["rows"], chunk_table["offs"] = P.chunks()
-            chunk_table["info"] = P.info()
+        h2 = time.perf_counter()
+        host_ms["plan"].append(1e3 * (h1 - h0))
+        host_ms["execute"].append(1e3 * (h2 - h1))
+        if keep:
+            return P
         P.free()
-        return st
+        host_ms["free"].append(1e3 * (time.perf_counter() - h2))
+        return None
 
     def barrier():
         if world > 1:
@@ -306,8 +343,11 @@ def main():
         torch.cuda.synchronize()
 
     for _ in range(args.warmup):
-        step()
+        step(profile=True)
     barrier()
+    for v in host_ms.values():
+        v.clear()
+    link_live = probe_d2h(h_val, dev)
     launches0 = capi.kernel_launches()
     stats = []
     with Clocks(local) as clk:
@@ -315,11 +355,17 @@ def main():
         e1 = torch.cuda.Event(enable_timing=True)
         w0 = time.perf_counter()
         e0.record(stream)
-        for _ in range(args.steps):
-            stats.append(step(profile=True))
+        for k in range(args.steps):
+            last = step(profile=True, keep=(k == args.steps - 1))
         e1.record(stream)
         barrier()
         wall = time.perf_counter() - w0
+    # kernel times of the last timed step (its events were recorded inside the timed region)
+    stats.append(last.stats())
+    chunk_table["rows"], chunk_table["offs"] = last.chunks()
+    chunk_table["info"] = last.info()
+    last.free()
+    nstat = len(stats)
     launches = capi.kernel_launches() - launches0
     ms = e0.elapsed_time(e1)
     t_max = ms
@@ -371,12 +417,12 @@ def main():
     if dom is not None:
         if dom.startswith("num"):
             per_launch = compulsory_bytes(A, B, chunk_table["rows"], chunk_table["offs"], r0)
-            byts = float(np.sum(per_launch)) * args.steps
+            byts = float(np.sum(per_launch)) * nstat
         elif dom.startswith("sym"):
             # symbolic: A panel + u + crp + touched B rows (col only) + crp writes
             bl = np.diff(B.row_ptr)
             touched = np.unique(A.col[A.row_ptr[r0]:A.row_ptr[r1]])
-            byts = args.steps * (24.0 * (r1 - r0) + 12.0 * (A.row_ptr[r1] - A.row_ptr[r0]) + 16.0 * len(touched)
+            byts = nstat * (24.0 * (r1 - r0) + 12.0 * (A.row_ptr[r1] - A.row_ptr[r0]) + 16.0 * len(touched)
                                  + 4.0 * float(bl[touched].sum()))
         else:
             byts = 0.0
@@ -385,8 +431,9 @@ def main():
         roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
                 "frac": ach / hbm_peak, "traffic": None, "peak_source": peak_src,
                 "avg_launch_ms": ms_dom / max(1, kern[dom]["launches"]),
-                "share_of_step": ms_dom / t_max if t_max else None,
-                "per_kernel_ms_per_step": {k: v["ms"] / args.steps for k, v in agg.items()}}
+                "share_of_step": (ms_dom / nstat) / (t_max / args.steps) if t_max else None,
+                "per_kernel_ms_per_step": {k: v["ms"] / nstat for k, v in agg.items()},
+                "kernel_times_from": "CUDA events of the last timed step (read after the timed region)"}
         tf = os.path.join(ROOT, "profiles", "traffic.json")
         if os.path.exists(tf):
             try:
@@ -470,7 +517,9 @@ def main():
         d2h_bytes = 12 * nnz_total + 8 * (A.nrows + 1)
         link = json.load(open(os.path.join(ROOT, "profiles", "hostlink.json"))) if os.path.exists(
             os.path.join(ROOT, "profiles", "hostlink.json")) else {}
-        link_gbs = float(link.get("d2h_GBps", 57.2))
+        link_gbs = float(link_live) if link_live else float(link.get("d2h_GBps", 57.2))
+        link_src = ("measured live in this run (1 GiB pinned D2H, best of 3)" if link_live
+                    else "profiles/hostlink.json (another box)")
         bound_ms = d2h_bytes / (link_gbs * world) / 1e6
         line = {
             "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
@@ -488,9 +537,10 @@ def main():
             "cpu_baseline": cpu,
             "e2e": e2e,
             "d2h": {"bytes_per_step": d2h_bytes, "achieved_GBps": d2h_bytes / (t_max / args.steps / 1e3) / 1e9,
-                    "host_link_GBps": link_gbs, "host_link_bound_ms": bound_ms,
+                    "host_link_GBps": link_gbs, "host_link_source": link_src, "host_link_bound_ms": bound_ms,
                     "frac_of_link_bound": bound_ms / (t_max / args.steps)},
-            "wall_s_timed": wall, "pinned_output_alloc_s": pin_s,
+            "wall_s_timed": wall,
+            "host_ms_per_step": {k: round(float(np.median(v)), 3) for k, v in host_ms.items() if v}, "pinned_output_alloc_s": pin_s,
             "parity": parity,
         }
         print(json.dumps(line), flush=True)

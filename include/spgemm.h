@@ -183,7 +183,9 @@ typedef struct {
     double bytes; /* algorithmic bytes moved by those launches */
 } spgemm_kernel_stat;
 
-/* Fills up to max entries; returns the number of classes in *n. */
+/* Fills up to max entries; returns the number of classes in *n.  With opts.profile = 1 the times
+ * of the last execution are read from its CUDA events on this call (not inside the execution, so
+ * profiling adds only event records to a timed step). */
 spgemm_status spgemm_stats(spgemm_plan_t plan, spgemm_kernel_stat *stats, int32_t max, int32_t *n);
 
 /* Timeline of the last execution with opts.profile = 1: 6 doubles per chunk, milliseconds from the
@@ -198,7 +200,9 @@ void spgemm_free(spgemm_plan_t plan);
 /* Process-wide number of CUDA kernels this library has launched (all plans, all devices). */
 int64_t spgemm_kernel_launches(void);
 
-/* Release the library's cached pinned staging memory. */
+/* Release the library's caches that no live plan holds: pinned staging memory, and the pooled
+ * streams and events that plans take at spgemm_plan and return at spgemm_free (reused so that a
+ * plan does not create or destroy CUDA objects; see api.cu "reusable CUDA objects"). */
 void spgemm_release_cache(void);
 
 const char *spgemm_status_string(spgemm_status s);

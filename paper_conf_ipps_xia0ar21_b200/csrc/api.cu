@@ -111,15 +111,64 @@ double elapsed(cudaEvent_t a, cudaEvent_t b) {
     return ms;
 }
 
-struct EvSet {  // timing events (profile mode only)
-    std::vector<cudaEvent_t> ev;
-    explicit EvSet(bool on, size_t n) {
-        if (!on) return;
-        ev.resize(n);
-        for (auto &e : ev) CK(cudaEventCreate(&e));
+// ------------------------------------------------ reusable CUDA objects (per device, pooled)
+// Streams and events are created on first use and handed from plan to plan: creating and
+// destroying ~100 events and 3 streams per multiply cost ~1-2 ms of host time per step, serial
+// with the pipeline.  A plan takes one Res at spgemm_plan and returns it at spgemm_free.
+struct Res {
+    int device = -1;
+    bool used = false;
+    cudaStream_t copy = nullptr, astream = nullptr, hstream = nullptr, own = nullptr;
+    enum { PLAIN = 0, TIMING = 1, PIECE = 2 };
+    std::vector<cudaEvent_t> pool[3];
+    // n events of pool `kind` starting at index `from`; grows the pool as needed
+    std::vector<cudaEvent_t> events(int kind, size_t from, size_t n) {
+        auto &v = pool[kind];
+        while (v.size() < from + n) {
+            cudaEvent_t e;
+            CK(cudaEventCreateWithFlags(&e, kind == TIMING ? cudaEventDefault : cudaEventDisableTiming));
+            v.push_back(e);
+        }
+        return std::vector<cudaEvent_t>(v.begin() + from, v.begin() + from + n);
     }
-    ~EvSet() {
-        for (auto e : ev) cudaEventDestroy(e);
+    cudaStream_t stream(cudaStream_t &slot) {
+        if (!slot) CK(cudaStreamCreateWithFlags(&slot, cudaStreamNonBlocking));
+        return slot;
+    }
+    void destroy() {
+        for (auto &v : pool)
+            for (auto e : v) cudaEventDestroy(e);
+        for (auto st : {copy, astream, hstream, own})
+            if (st) cudaStreamDestroy(st);
+    }
+};
+std::mutex g_res_mu;
+std::vector<Res *> g_res;
+
+Res *res_acquire(int device) {
+    std::lock_guard<std::mutex> lk(g_res_mu);
+    for (auto r : g_res)
+        if (!r->used && r->device == device) {
+            r->used = true;
+            return r;
+        }
+    Res *r = new Res();
+    r->device = device;
+    r->used = true;
+    g_res.push_back(r);
+    return r;
+}
+
+void res_release(Res *r) {
+    if (!r) return;
+    std::lock_guard<std::mutex> lk(g_res_mu);
+    r->used = false;
+}
+
+struct EvSet {  // timing events (profile mode only), borrowed from the plan's Res
+    std::vector<cudaEvent_t> ev;
+    EvSet(bool on, Res *r, size_t from, size_t n) {
+        if (on) ev = r->events(Res::TIMING, from, n);
     }
     cudaEvent_t *at(size_t k) { return ev.empty() ? nullptr : ev.data() + k; }
     void rec(size_t k, cudaStream_t s) {
@@ -131,8 +180,8 @@ struct EvSet {  // timing events (profile mode only)
 
 struct spgemm_plan_s {
     int device = 0, num_sms = 148;
+    Res *res = nullptr;  // pooled streams and events
     cudaStream_t stream = nullptr, copy = nullptr;
-    bool own_stream = false;
     std::vector<cudaEvent_t> ev_num, ev_d2h, ev_tot;
     cudaEvent_t ev_ready = nullptr;
 
@@ -149,7 +198,6 @@ struct spgemm_plan_s {
     int32_t *nnzr = nullptr, *listB = nullptr, *listG = nullptr;  // symbolic long-row lists
     int32_t *listBn = nullptr, *listGn = nullptr;                  // numeric long-row lists
     cudaStream_t astream = nullptr;  // fused plans: symbolic passes run here, ahead of the numeric
-    bool own_astream = false;
     cudaStream_t hstream = nullptr;         // host B: value pieces H2D
     std::vector<cudaEvent_t> ev_piece;      // one per value piece, in upload order
     std::vector<int64_t> bpiece_rows;       // B row boundaries of the pieces
@@ -187,6 +235,14 @@ struct spgemm_plan_s {
     double *h_val = nullptr;
 
     bool profile = false;
+    struct Pending {  // profile mode: events of the last execution, evaluated on demand
+        bool active = false;
+        std::vector<cudaEvent_t> ev;
+        int64_t nch = 0, total = 0;
+        size_t per = 0;
+        bool overflow = false;
+        std::vector<int64_t> offs;
+    } pend;
     std::vector<Stat> stats;
     std::vector<double> timeline;  // profile: 6 times (ms) per chunk of the last execution
     bool failed = false;
@@ -230,23 +286,9 @@ struct spgemm_plan_s {
     }
     int64_t num_chunks() const { return chunk_rows.empty() ? 0 : int64_t(chunk_rows.size()) - 1; }
     ~spgemm_plan_s() {
-        if (stream) cudaStreamSynchronize(stream);
-        if (copy) cudaStreamSynchronize(copy);
-        for (auto e : ev_num) cudaEventDestroy(e);
-        for (auto e : ev_d2h) cudaEventDestroy(e);
-        for (auto e : ev_tot) cudaEventDestroy(e);
-        if (ev_ready) cudaEventDestroy(ev_ready);
-        if (astream && own_astream) {
-            cudaStreamSynchronize(astream);
-            cudaStreamDestroy(astream);
-        }
-        if (hstream) {
-            cudaStreamSynchronize(hstream);
-            cudaStreamDestroy(hstream);
-        }
-        for (auto e : ev_piece) cudaEventDestroy(e);
-        if (copy) cudaStreamDestroy(copy);
-        if (own_stream && stream) cudaStreamDestroy(stream);
+        for (auto st : {stream, copy, astream, hstream})
+            if (st) cudaStreamSynchronize(st);
+        res_release(res);
         if (own_arena && arena) cudaFree(arena);
         if (h_rp) cudaFreeHost(h_rp);
         if (h_col) cudaFreeHost(h_col);
@@ -376,21 +418,18 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->nnzB = Bh->nnz;
     P->base_wanted = opts.row_ptr_base;
 
-    // streams and events (created at plan time: nothing is created inside execute)
-    if (opts.stream) {
-        P->stream = (cudaStream_t)opts.stream;
-    } else {
-        CK(cudaStreamCreateWithFlags(&P->stream, cudaStreamNonBlocking));
-        P->own_stream = true;
-    }
-    CK(cudaStreamCreateWithFlags(&P->copy, cudaStreamNonBlocking));
-    P->ev_num.resize(P->ring);
-    P->ev_d2h.resize(P->ring);
-    for (int r = 0; r < P->ring; ++r) {
-        CK(cudaEventCreateWithFlags(&P->ev_num[r], cudaEventDisableTiming));
-        CK(cudaEventCreateWithFlags(&P->ev_d2h[r], cudaEventDisableTiming));
-    }
-    CK(cudaEventCreateWithFlags(&P->ev_ready, cudaEventDisableTiming));
+    // streams and events: taken from the device's pool at plan time (nothing is created inside
+    // execute; plans after the first reuse the previous plans' objects)
+    P->res = res_acquire(P->device);
+    Res *rs = P->res;
+    P->stream = opts.stream ? (cudaStream_t)opts.stream : rs->stream(rs->own);
+    P->copy = rs->stream(rs->copy);
+    // plain-event layout in the pool: [0, ring) numeric done, [ring, 2 ring) copy done, 2 ring
+    // ready, then per-chunk totals, then value pieces
+    P->ev_num = rs->events(Res::PLAIN, 0, P->ring);
+    P->ev_d2h = rs->events(Res::PLAIN, P->ring, P->ring);
+    P->ev_ready = rs->events(Res::PLAIN, 2 * P->ring, 1)[0];
+    const size_t ev_base = 2 * size_t(P->ring) + 1;
     cudaStream_t s = P->stream;
 
     // S9 arena
@@ -412,7 +451,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         P->own_arena = true;
     }
 
-    EvSet pe(P->profile, 12);
+    EvSet pe(P->profile, rs, 0, 12);
     pe.rec(0, s);
 
     // S0 residency: B.  Host operands: row_ptr and col_idx now (the count and symbolic passes need
@@ -471,16 +510,15 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     }
     // start the B value pieces (host operands) on their own stream, one event per piece
     if (!bval_pieces.empty()) {
-        CK(cudaStreamCreateWithFlags(&P->hstream, cudaStreamNonBlocking));
+        P->hstream = rs->stream(rs->hstream);
         CK(cudaEventRecord(P->ev_ready, s));  // allocation order: after everything queued so far
         CK(cudaStreamWaitEvent(P->hstream, P->ev_ready, 0));
-        P->ev_piece.resize(bval_pieces.size());
+        P->ev_piece = rs->events(Res::PIECE, 0, bval_pieces.size());
         for (size_t k = 0; k < bval_pieces.size(); ++k) {
             const auto &pc = bval_pieces[k];
             if (pc.second)
                 CK(cudaMemcpyAsync(bval_dev + pc.first, Bh->values + pc.first, sizeof(double) * pc.second,
                                    cudaMemcpyHostToDevice, P->hstream));
-            CK(cudaEventCreateWithFlags(&P->ev_piece[k], cudaEventDisableTiming));
             CK(cudaEventRecord(P->ev_piece[k], P->hstream));
         }
     }
@@ -513,6 +551,14 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     launch_count(P->A, P->B, P->bnd, P->ctl, s);
     CKL("count");
     pe.rec(2, s);
+    // fused plans: the prefix of the row bounds (chunk boundaries) is scanned before the first
+    // host round trip, which then reads both the count totals and the prefix total
+    int64_t total_b = 0;
+    if (P->fused) {
+        launch_scan64(P->bnd, P->R, P->crp, P->tmp, s);
+        CKL("bound scan");
+        CK(cudaMemcpyAsync(&total_b, P->crp + P->R, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    }
     Ctl hc;
     CK(cudaMemcpyAsync(&hc, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
@@ -604,11 +650,6 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     } else {
         // fused: boundaries from the prefix of the row bounds; the symbolic pass runs per chunk
         // inside execute.  crp temporarily holds that prefix.
-        int64_t total_b = 0;
-        launch_scan64(P->bnd, R, P->crp, P->tmp, s);
-        CKL("bound scan");
-        CK(cudaMemcpyAsync(&total_b, P->crp + R, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-        CK(cudaStreamSynchronize(s));
         P->sum_bound = total_b;
         int64_t cap = ring_cap(P->max_bound);
         cap = std::max<int64_t>(std::min<int64_t>(cap, std::max<int64_t>(total_b, 1)), std::max<int64_t>(P->max_bound, 1));
@@ -634,17 +675,11 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
             CK(cudaStreamSynchronize(s));
             P->used = save;
         }
-        P->ev_tot.resize(nch);
-        for (auto &e : P->ev_tot) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        P->ev_tot = rs->events(Res::PLAIN, ev_base, nch);
         // the symbolic passes get their own stream so that chunk j+1's symbolic pass overlaps
         // chunk j's numeric pass (the two passes have separate lists and arena scratch)
         const char *ser = getenv("SPGEMM_SERIAL_ANALYSIS");  // ablation knob
-        if (ser && ser[0] == '1') {
-            P->astream = P->stream;
-        } else {
-            CK(cudaStreamCreateWithFlags(&P->astream, cudaStreamNonBlocking));
-            P->own_astream = true;
-        }
+        P->astream = (ser && ser[0] == '1') ? P->stream : rs->stream(rs->astream);
     }
     // host operands: the last value piece each chunk's numeric pass reads (largest B row touched;
     // with A aliasing B also the chunk's own rows)
@@ -743,6 +778,58 @@ void enqueue_analysis(spgemm_plan_s *P, int64_t j, cudaEvent_t *ev) {
     CK(cudaEventRecord(P->ev_tot[j], as));
 }
 
+// Per-kernel statistics and the timeline of the last execution, from its timing events.  Done
+// on demand (spgemm_stats / spgemm_timeline, or before the next execution reuses the events):
+// ~500 cudaEventElapsedTime calls cost ~2 ms of host time, which must not sit inside a timed step.
+void finalize_profile(spgemm_plan_s *P) {
+    if (!P->pend.active) return;
+    P->pend.active = false;
+    std::vector<cudaEvent_t> &ev = P->pend.ev;
+    auto ev_at = [&](size_t k) { return ev.data() + k; };
+    const int64_t nch = P->pend.nch;
+    const size_t per = P->pend.per;
+    const bool overflow = P->pend.overflow;
+    const std::vector<int64_t> &offs = P->pend.offs;
+    const int64_t total = P->pend.total;
+    P->clear_stats({"num_w", "num_b", "num_g", "d2h_span", "execute_total"});
+    if (P->fused) P->clear_stats({"sym_w", "sym_b", "sym_g", "scan"});
+    for (int64_t c = 0; c < nch; ++c) {
+        cudaEvent_t *e = ev_at(size_t(c) * per);
+        if (P->fused) {
+            P->add_stat("sym_w", elapsed(e[0], e[1]), 0);
+            P->add_stat("sym_b", elapsed(e[1], e[2]), 0);
+            P->add_stat("sym_g", elapsed(e[2], e[3]), 0);
+            P->add_stat("scan", elapsed(e[3], e[4]), 0);
+        }
+        if (!overflow) {
+            P->add_stat("num_w", elapsed(e[6], e[7]), 0);
+            P->add_stat("num_b", elapsed(e[7], e[8]), 0);
+            P->add_stat("num_g", elapsed(e[8], e[9]), 0);
+            cudaEvent_t end = (c + 1 < nch) ? ev[size_t(c + 1) * per + 10] : ev[size_t(nch) * per + 1];
+            P->add_stat("d2h_span", elapsed(e[10], end), double(offs[c + 1] - offs[c]) * 12);
+        }
+    }
+    P->add_stat("execute_total", elapsed(ev[size_t(nch) * per], ev[size_t(nch) * per + 1]),
+                double(total) * 12 + 8.0 * (P->R + 1));
+    // timeline: per chunk [analysis start, end, numeric start, end, copy start, end] in ms
+    P->timeline.assign(size_t(nch) * 6, -1.0);
+    cudaEvent_t t0 = ev[size_t(nch) * per];
+    for (int64_t c = 0; c < nch; ++c) {
+        cudaEvent_t *e = ev_at(size_t(c) * per);
+        double *t = &P->timeline[size_t(c) * 6];
+        if (P->fused) {
+            t[0] = elapsed(t0, e[0]);
+            t[1] = elapsed(t0, e[4]);
+        }
+        if (!overflow) {
+            t[2] = elapsed(t0, e[6]);
+            t[3] = elapsed(t0, e[9]);
+            t[4] = elapsed(t0, e[10]);
+            t[5] = elapsed(t0, e[11]);
+        }
+    }
+}
+
 struct Sink {
     spgemm_chunk_cb cb = nullptr;
     void *user = nullptr;
@@ -756,6 +843,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
                      const Sink *sink, bool *overflow) {
     if (P->failed) fail(SPGEMM_ERR_STATE, "plan is in a failed state");
     DeviceGuard g(P->device);
+    finalize_profile(P);  // the previous execution's events are about to be reused
     cudaStream_t s = P->stream, cp = P->copy;
     const int64_t nch = P->num_chunks();
     const int ring = P->ring;
@@ -801,7 +889,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
     };
 
     const int per = 12;
-    EvSet pe(P->profile, size_t(nch) * per + 4);
+    EvSet pe(P->profile, P->res, 12, size_t(nch) * per + 4);
     CK(cudaEventRecord(P->ev_ready, s));
     CK(cudaStreamWaitEvent(cp, P->ev_ready, 0));
     pe.rec(size_t(nch) * per, s);
@@ -897,44 +985,14 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         P->rows_b = (int64_t)hc.rows_b;
         P->rows_g = (int64_t)hc.rows_g;
     }
-    if (P->profile) {
-        P->clear_stats({"num_w", "num_b", "num_g", "d2h_span", "execute_total"});
-        if (P->fused) P->clear_stats({"sym_w", "sym_b", "sym_g", "scan"});
-        for (int64_t c = 0; c < nch; ++c) {
-            cudaEvent_t *e = pe.at(size_t(c) * per);
-            if (P->fused) {
-                P->add_stat("sym_w", elapsed(e[0], e[1]), 0);
-                P->add_stat("sym_b", elapsed(e[1], e[2]), 0);
-                P->add_stat("sym_g", elapsed(e[2], e[3]), 0);
-                P->add_stat("scan", elapsed(e[3], e[4]), 0);
-            }
-            if (!*overflow) {
-                P->add_stat("num_w", elapsed(e[6], e[7]), 0);
-                P->add_stat("num_b", elapsed(e[7], e[8]), 0);
-                P->add_stat("num_g", elapsed(e[8], e[9]), 0);
-                cudaEvent_t end = (c + 1 < nch) ? pe.ev[size_t(c + 1) * per + 10] : pe.ev[size_t(nch) * per + 1];
-                P->add_stat("d2h_span", elapsed(e[10], end), double(offs[c + 1] - offs[c]) * 12);
-            }
-        }
-        P->add_stat("execute_total", elapsed(pe.ev[size_t(nch) * per], pe.ev[size_t(nch) * per + 1]),
-                    double(total) * 12 + 8.0 * (P->R + 1));
-        // timeline: per chunk [analysis start, end, numeric start, end, copy start, end] in ms
-        P->timeline.assign(size_t(nch) * 6, -1.0);
-        cudaEvent_t t0 = pe.ev[size_t(nch) * per];
-        for (int64_t c = 0; c < nch; ++c) {
-            cudaEvent_t *e = pe.at(size_t(c) * per);
-            double *t = &P->timeline[size_t(c) * 6];
-            if (P->fused) {
-                t[0] = elapsed(t0, e[0]);
-                t[1] = elapsed(t0, e[4]);
-            }
-            if (!*overflow) {
-                t[2] = elapsed(t0, e[6]);
-                t[3] = elapsed(t0, e[9]);
-                t[4] = elapsed(t0, e[10]);
-                t[5] = elapsed(t0, e[11]);
-            }
-        }
+    if (P->profile) {  // per-kernel times are read from the events lazily (finalize_profile)
+        P->pend.active = true;
+        P->pend.ev = pe.ev;
+        P->pend.nch = nch;
+        P->pend.per = per;
+        P->pend.overflow = *overflow;
+        P->pend.offs = offs;
+        P->pend.total = total;
     }
     return total;
 }
@@ -1167,6 +1225,10 @@ spgemm_status spgemm_stats(spgemm_plan_t P, spgemm_kernel_stat *out, int32_t max
         g_err = "NULL argument";
         return SPGEMM_ERR_INVALID_ARGUMENT;
     }
+    {
+        DeviceGuard g(P->device);
+        finalize_profile(P);
+    }
     *n = (int32_t)P->stats.size();
     for (int32_t k = 0; k < max && k < *n && out; ++k) {
         std::memset(&out[k], 0, sizeof(out[k]));
@@ -1183,6 +1245,10 @@ spgemm_status spgemm_timeline(spgemm_plan_t P, double *out, int64_t max, int64_t
         g_err = "NULL argument";
         return SPGEMM_ERR_INVALID_ARGUMENT;
     }
+    {
+        DeviceGuard g(P->device);
+        finalize_profile(P);
+    }
     *n = (int64_t)P->timeline.size();
     for (int64_t k = 0; k < max && k < *n && out; ++k) out[k] = P->timeline[k];
     return SPGEMM_OK;
@@ -1198,13 +1264,30 @@ void spgemm_free(spgemm_plan_t P) {
 }
 
 void spgemm_release_cache(void) {
-    std::lock_guard<std::mutex> lk(g_pin_mu);
-    std::vector<PinnedBlock> keep;
-    for (auto &b : g_pins) {
-        if (b.used) keep.push_back(b);
-        else cudaFreeHost(b.p);
+    {
+        std::lock_guard<std::mutex> lk(g_pin_mu);
+        std::vector<PinnedBlock> keep;
+        for (auto &b : g_pins) {
+            if (b.used) keep.push_back(b);
+            else cudaFreeHost(b.p);
+        }
+        g_pins.swap(keep);
     }
-    g_pins.swap(keep);
+    std::lock_guard<std::mutex> lk(g_res_mu);
+    std::vector<Res *> keep;
+    int prev = -1;
+    cudaGetDevice(&prev);
+    for (auto r : g_res) {
+        if (r->used) {
+            keep.push_back(r);
+            continue;
+        }
+        cudaSetDevice(r->device);
+        r->destroy();
+        delete r;
+    }
+    if (prev >= 0) cudaSetDevice(prev);
+    g_res.swap(keep);
 }
 
 const char *spgemm_status_string(spgemm_status s) {
