@@ -735,7 +735,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
 }
 
 void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t max_row_nnz, cudaEvent_t *ev) {
-    NumArgs na;
+    NumArgs na{};
     na.A = P->A;
     na.B = P->B;
     na.crp = P->crp;

@@ -133,6 +133,7 @@ struct NumArgs {
     int group;
     int tiers;           // as in SymArgs
     int batch;
+    int tload;           // W tier table sizing: 0 -> >= 4n/3 slots, 1 -> >= 2n, 2 -> >= 4n (capped at TW_NUM)
 };
 // S6+S7: numeric pass over chunk rows [r0, r1); ev as in launch_symbolic
 void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);
@@ -145,7 +146,7 @@ int choose_group(const DevCSR &B, int64_t nnzB);
 
 // occupancy-derived grid sizes (queried once per device)
 struct Grids {
-    int count_blocks, symw_blocks, numw_blocks, symb_blocks, numb_blocks;
+    int count_blocks, symw_blocks, numw_blocks, numw3_blocks, symb_blocks, numb_blocks;
 };
 const Grids &grids(int device, int num_sms);
 

@@ -15,6 +15,7 @@
 // "dense accumulation" of §II-B L107 / §III-B, used here for the longest rows).
 #include <climits>
 #include <cstdio>
+#include <cstdlib>
 
 #include <atomic>
 
@@ -29,6 +30,10 @@ long long kernel_launches() { return g_launches.load(); }
 #define FULLMASK 0xffffffffu
 constexpr int32_t EMPTY = -1;
 
+// Home slot of column c in a table of 2^lg slots: multiplicative (Fibonacci) hashing.  (A variant
+// whose low 5 bits XOR-fold c's digits, so that a stencil row's columns fall in distinct shared
+// memory banks, cut bank conflicts by 22% but cost 8 more instructions per probe; the W kernels
+// are issue-bound, not LSU-bound, so it was slower -- profiles/r01/ncu_*_h1.md.)
 __device__ __forceinline__ uint32_t hslot(int32_t c, int lg) {
     return ((uint32_t)c * 0x9E3779B1u) >> (32 - lg);
 }
@@ -116,23 +121,33 @@ __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t *s, int64_
 // ------------------------------------------------------------------ warp product iterator (W tier)
 //
 // Visits every intermediate product A_ik * B_kj of row i with one warp (Alg. 1 lines 3-5).
-//  * A entries are fetched 32 at a time (one per lane) together with their B row bounds, so the
-//    A.col -> B.rp dependency is paid once per 32 entries; bounds are then broadcast by shuffle.
+//  * A entries are fetched 32 at a time (one per lane) together with their B row bounds and staged
+//    in the warp's shared-memory slot `st`, so the A.col -> B.rp dependency is paid once per 32
+//    entries; a round then reads its entry's bounds with one broadcast LDS.128 (+ one LDS.64 for
+//    the A value) -- shuffles would cost six LSU wavefronts per round, and the LSU data pipe
+//    (shared memory, shuffles, L1) is what bounds these kernels.
 //  * Lanes form 32/G subgroups; subgroup g takes one B row per round and its lanes take G
 //    consecutive entries of it (coalesced).  U rounds are loaded before any is consumed, so U
 //    independent B-row loads are in flight per warp (latency, not bandwidth, bounds this loop).
-//  * f(ok, col, value) is called once per round by every lane, followed by __syncwarp().  With
+//  * f(ok, col, value) is called once per round by every lane, followed by __syncwarp() when SYNC
+//    (the numeric pass: a round's value updates must land before the next round's; the symbolic
+//    pass only inserts keys with atomicCAS and needs no ordering between rounds).  With
 //    G == 32 all active lanes of a round hold entries of ONE B row, i.e. distinct columns
 //    (rows are sorted and unique), which lets the numeric pass update values without atomics.
-template <int G, int U, bool VALS, typename F>
-__device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR &B, int64_t i, F &&f) {
+struct AStage {
+    longlong2 be[32];  // [begin, end) of B row A.col[e] for the 32 staged A entries
+    double a[32];      // A values (numeric pass)
+};
+
+template <int G, int U, bool VALS, bool SYNC, typename F>
+__device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR &B, int64_t i, AStage *st, F &&f) {
     constexpr int R = 32 / G;  // B rows per round
     const int lane = threadIdx.x & 31;
     const int sub = lane / G, sl = lane % G;
     const int64_t as = A.rp[i], ae = A.rp[i + 1];
     for (int64_t pb = as; pb < ae; pb += 32) {
         const int64_t e = pb + lane;
-        int64_t bs = 0, be = 0;
+        long long bs = 0, be = 0;
         double av = 0.0;
         if (e < ae) {
             const int32_t k = __ldg(&A.col[e]);
@@ -140,8 +155,12 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
             be = __ldg(&B.rp[k + 1]);
             if (VALS) av = __ldg(&A.val[e]);
         }
+        __syncwarp();  // the previous batch's rounds have read their entries
+        st->be[lane] = make_longlong2(bs, be);  // lanes past the row's end stage empty ranges
+        if (VALS) st->a[lane] = av;
+        __syncwarp();
         const int nb = (int)(ae - pb < 32 ? ae - pb : 32);
-        for (int t = 0; t < nb; t += R * U) {
+        for (int t = 0; t < nb; t += R * U) {  // R * U divides 32, so src < 32
             int64_t s[U], en[U];
             double a[U], v[U];
             int32_t c[U];
@@ -149,21 +168,19 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const int src = t + u * R + sub;
-                int64_t ss = __shfl_sync(FULLMASK, bs, src & 31);
-                int64_t ee = __shfl_sync(FULLMASK, be, src & 31);
-                a[u] = VALS ? __shfl_sync(FULLMASK, av, src & 31) : 0.0;
-                if (src >= nb) ss = ee = 0;
-                s[u] = ss;
-                en[u] = ee;
-                const int64_t q = ss + sl;
-                ok[u] = q < ee;
+                const longlong2 r = st->be[src];
+                s[u] = r.x;
+                en[u] = r.y;
+                a[u] = VALS ? st->a[src] : 0.0;
+                const int64_t q = r.x + sl;
+                ok[u] = q < r.y;
                 c[u] = ok[u] ? __ldg(&B.col[q]) : 0;
                 v[u] = (VALS && ok[u]) ? __ldg(&B.val[q]) : 0.0;
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 f(ok[u], c[u], a[u] * v[u]);
-                __syncwarp();
+                if (SYNC) __syncwarp();
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
@@ -175,7 +192,7 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
                     const int32_t cc = okk ? __ldg(&B.col[q]) : 0;
                     const double vv = (VALS && okk) ? __ldg(&B.val[q]) : 0.0;
                     f(okk, cc, a[u] * vv);
-                    __syncwarp();
+                    if (SYNC) __syncwarp();
                 }
             }
         }
@@ -262,6 +279,36 @@ __device__ __forceinline__ uint32_t find_slot(int32_t *keys, int32_t c, int lg) 
         }
         h = (h + 1) & mask;
     }
+}
+
+// Warp-uniform find-or-insert (W tier): every lane of the warp calls it (inactive lanes with
+// ok = false); all lanes probe in lockstep -- one predicated LDS (+ predicated CAS on an empty
+// slot) per step and one uniform vote to leave -- instead of a divergent per-lane loop, whose
+// reconvergence barriers and branch resolution dominated the stalls of the W kernels (ncu).
+// Returns the slot (undefined for inactive lanes); *fresh = 1 if this lane inserted the key.
+__device__ __forceinline__ uint32_t warp_find_slot(int32_t *keys, int32_t c, int lg, bool ok, int *fresh) {
+    const uint32_t mask = (1u << lg) - 1;
+    uint32_t h = hslot(c, lg);
+    volatile int32_t *vk = keys;
+    bool done = !ok;
+    int ins = 0;
+    while (true) {
+        if (!done) {
+            int32_t k = vk[h];
+            if (k == EMPTY) {
+                k = atomicCAS(&keys[h], EMPTY, c);
+                if (k == EMPTY) {
+                    ins = 1;
+                    k = c;
+                }
+            }
+            if (k == c) done = true;
+            else h = (h + 1) & mask;
+        }
+        if (__all_sync(FULLMASK, done)) break;
+    }
+    *fresh = ins;
+    return h;
 }
 
 // vectorised fill of n (multiple of 4) int32 / n (even) doubles with a warp
@@ -357,9 +404,10 @@ __device__ __forceinline__ void push_long(int64_t i, int64_t bound, int64_t capB
 
 template <int G>
 __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
-    extern __shared__ int32_t smem_i[];
+    extern __shared__ __align__(16) int32_t smem_i[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     int32_t *keys = smem_i + wid * TW_SYM;
+    AStage *ast = reinterpret_cast<AStage *>(smem_i + WARPS_W * TW_SYM) + wid;
     const int64_t R = a.r1 - a.r0;
     unsigned long long lmax = 0, nw = 0, nlong = 0;
     constexpr int MAXLG = 10;  // log2(TW_SYM)
@@ -388,8 +436,10 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
             warp_fill_keys(keys, T);
             __syncwarp();
             int cnt = 0;
-            warp_row_products<G, (G == 32 ? 4 : 2), false>(a.A, a.B, i, [&](bool ok, int32_t c, double) {
-                if (ok) cnt += sym_insert(keys, c, lg);
+            warp_row_products<G, (G == 32 ? 4 : 2), false, false>(a.A, a.B, i, ast, [&](bool ok, int32_t c, double) {
+                int fresh;
+                warp_find_slot(keys, c, lg, ok, &fresh);
+                cnt += fresh;
             });
             cnt = warp_sum(cnt);
             if (lane == 0) {
@@ -678,15 +728,18 @@ __device__ __forceinline__ void sort_emit_any(const unsigned long long *pk, int 
     }
 }
 
-template <int G, bool WIDE>
-__global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
-    extern __shared__ double smem_d[];
+template <int G, bool WIDE, int MINB>
+__global__ void __launch_bounds__(WARPS_W * 32, MINB) k_num_w(NumArgs a) {
+    extern __shared__ __align__(16) double smem_d[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    double *vals = smem_d + wid * TW_NUM;
-    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + WARPS_W * TW_NUM) + wid * TW_NUM;
+    AStage *ast = reinterpret_cast<AStage *>(smem_d) + wid;  // A-entry staging first (16-B aligned)
+    double *vals = smem_d + WARPS_W * (sizeof(AStage) / sizeof(double)) + wid * TW_NUM;
+    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + WARPS_W * (sizeof(AStage) / sizeof(double)) +
+                                                WARPS_W * TW_NUM) + wid * TW_NUM;
     // WIDE (ncols > 2^23): 64-bit packed keys staged after the key tables
     unsigned long long *stage = reinterpret_cast<unsigned long long *>(
-                                    reinterpret_cast<int32_t *>(smem_d + WARPS_W * TW_NUM) + WARPS_W * TW_NUM) +
+                                    reinterpret_cast<int32_t *>(smem_d + WARPS_W * (sizeof(AStage) / sizeof(double)) +
+                                                                WARPS_W * TW_NUM) + WARPS_W * TW_NUM) +
                                 wid * TW_NUM;
     constexpr int MAXLG = 9;  // log2(TW_NUM)
     const int64_t R = a.r1 - a.r0;
@@ -706,18 +759,17 @@ __global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
                 if (lane == 0) push_long(i, n, CAPB_NUM, CAPH_NUM, a.hblocks > 0, a.listB, a.listH, a.listG, a.ctl);
                 continue;
             }
-            const int lg = table_log2(n, MAXLG);
+            const int lg = table_log2(a.tload == 0 ? n : a.tload == 1 ? (3 * n) / 2 : 3 * n, MAXLG);
             const int T = 1 << lg;
             warp_fill_keys(keys, T);
             warp_fill_zero(vals, T);
             __syncwarp();
-            warp_row_products<G, (G == 32 ? 4 : 2), true>(a.A, a.B, i, [&](bool ok, int32_t c, double v) {
+            warp_row_products<G, (G == 32 ? 4 : 2), true, true>(a.A, a.B, i, ast, [&](bool ok, int32_t c, double v) {
                 if (G == 32) {
                     // one B row per round: distinct columns -> distinct slots -> plain RMW
-                    if (ok) {
-                        const uint32_t h = find_slot(keys, c, lg);
-                        vals[h] += v;
-                    }
+                    int fresh;
+                    const uint32_t h = warp_find_slot(keys, c, lg, ok, &fresh);
+                    if (ok) vals[h] += v;
                 } else {
                     const unsigned act = __ballot_sync(FULLMASK, ok);
                     if (ok) {
@@ -1151,9 +1203,10 @@ __global__ void __launch_bounds__(THREADS_G) k_num_g(NumArgs a) {
 
 // ------------------------------------------------------------------------------------ launchers
 
-size_t symw_smem() { return size_t(WARPS_W) * TW_SYM * sizeof(int32_t); }
+size_t symw_smem() { return size_t(WARPS_W) * (TW_SYM * sizeof(int32_t) + sizeof(AStage)); }
 size_t numw_smem(bool wide) {
-    return size_t(WARPS_W) * TW_NUM * (sizeof(int32_t) + sizeof(double) + (wide ? sizeof(unsigned long long) : 0));
+    return size_t(WARPS_W) * (TW_NUM * (sizeof(int32_t) + sizeof(double) + (wide ? sizeof(unsigned long long) : 0)) +
+                              sizeof(AStage));
 }
 size_t symb_smem() { return size_t(TB_SYM) * sizeof(int32_t); }
 size_t numb_smem() { return size_t(TB_NUM) * (sizeof(int32_t) + sizeof(double)); }
@@ -1161,8 +1214,10 @@ size_t numb_smem() { return size_t(TB_NUM) * (sizeof(int32_t) + sizeof(double));
 template <int G>
 static void set_attrs_w() {
     cudaFuncSetAttribute(k_sym_w<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symw_smem());
-    cudaFuncSetAttribute(k_num_w<G, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(false));
-    cudaFuncSetAttribute(k_num_w<G, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(true));
+    cudaFuncSetAttribute(k_num_w<G, false, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(false));
+    cudaFuncSetAttribute(k_num_w<G, true, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(true));
+    cudaFuncSetAttribute(k_num_w<G, false, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(false));
+    cudaFuncSetAttribute(k_num_w<G, true, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(true));
 }
 
 const Grids &grids(int device, int num_sms) {
@@ -1182,8 +1237,10 @@ const Grids &grids(int device, int num_sms) {
         g.count_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_w<8>, WARPS_W * 32, symw_smem());
         g.symw_blocks = num_sms * (occ > 0 ? occ : 1);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false>, WARPS_W * 32, numw_smem(false));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false, 4>, WARPS_W * 32, numw_smem(false));
         g.numw_blocks = num_sms * (occ > 0 ? occ : 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false, 3>, WARPS_W * 32, numw_smem(false));
+        g.numw3_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b, THREADS_B, symb_smem());
         g.symb_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_b, THREADS_B, numb_smem());
@@ -1242,11 +1299,20 @@ static void sym_w(const SymArgs &a, int blocks, cudaStream_t s) {
     k_sym_w<G><<<blocks, WARPS_W * 32, symw_smem(), s>>>(a);
     LAUNCHED(1);
 }
-template <int G>
+template <int G, int MINB>
 static void num_w(const NumArgs &a, int blocks, cudaStream_t s) {
-    if (a.B.ncols > (int64_t(1) << 23)) k_num_w<G, true><<<blocks, WARPS_W * 32, numw_smem(true), s>>>(a);
-    else k_num_w<G, false><<<blocks, WARPS_W * 32, numw_smem(false), s>>>(a);
+    if (a.B.ncols > (int64_t(1) << 23)) k_num_w<G, true, MINB><<<blocks, WARPS_W * 32, numw_smem(true), s>>>(a);
+    else k_num_w<G, false, MINB><<<blocks, WARPS_W * 32, numw_smem(false), s>>>(a);
     LAUNCHED(1);
+}
+template <int G>
+static void num_w(const NumArgs &a, int blocks, int minb, cudaStream_t s) {
+    if (minb == 3) num_w<G, 3>(a, blocks, s);
+    else num_w<G, 4>(a, blocks, s);
+}
+static int env_int(const char *name, int dflt) {
+    const char *v = getenv(name);
+    return (v && *v) ? atoi(v) : dflt;
 }
 
 static int group_for(const DevCSR &B, int64_t nnzB) {
@@ -1309,14 +1375,18 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
     const Grids &g = grids(dev, num_sms);
     cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);
     NumArgs aw = a;
-    aw.batch = batch_for(rows, g.numw_blocks);
-    const int wblocks = grid_for(rows, WARPS_W * aw.batch, g.numw_blocks);
+    static const int minb = env_int("SPGEMM_NUMW_MINB", 4);  // tuning knobs
+    static const int tload = env_int("SPGEMM_NUMW_TLOAD", 2);
+    aw.tload = tload;
+    const int full = minb == 3 ? g.numw3_blocks : g.numw_blocks;
+    aw.batch = batch_for(rows, full);
+    const int wblocks = grid_for(rows, WARPS_W * aw.batch, full);
     rec(ev, 0, s);
     switch (a.group) {
-        case 4: num_w<4>(aw, wblocks, s); break;
-        case 8: num_w<8>(aw, wblocks, s); break;
-        case 16: num_w<16>(aw, wblocks, s); break;
-        default: num_w<32>(aw, wblocks, s); break;
+        case 4: num_w<4>(aw, wblocks, minb, s); break;
+        case 8: num_w<8>(aw, wblocks, minb, s); break;
+        case 16: num_w<16>(aw, wblocks, minb, s); break;
+        default: num_w<32>(aw, wblocks, minb, s); break;
     }
     rec(ev, 1, s);
     if (a.tiers & 1) {

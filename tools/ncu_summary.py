@@ -18,6 +18,8 @@ KEYS = [
     "sm__maximum_warps_per_active_cycle_pct", "launch__grid_size", "launch__block_size",
     "l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum", "smsp__average_warp_latency_issue_stalled",
     "lts__t_sector_hit_rate.pct", "l1tex__t_sector_hit_rate.pct",
+    "inst_executed", "l1tex__data_pipe_lsu_wavefronts.sum.pct_of_peak_sustained_elapsed",
+    "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "sass__inst_executed_register_spilling",
 ]
 STALLS = "smsp__average_warps_issue_stalled_"
 
