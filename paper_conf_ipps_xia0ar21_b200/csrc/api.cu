@@ -207,10 +207,9 @@ struct spgemm_plan_s {
 
     uint32_t *gbits = nullptr, *gbits_sym = nullptr;
     double *gvals = nullptr;
-    int32_t *hkeys_num = nullptr, *hkeys_sym = nullptr;
-    double *hvals_num = nullptr;
-    int hblocks = 0;
-    int32_t *listH = nullptr, *listHn = nullptr;
+    int32_t *cur_sym = nullptr, *cur_num = nullptr;  // pieced CTA tier: cursor scratch
+    int64_t curstride = 0, max_deg = 0;
+    int bblocks_sym = 0, bblocks_num = 0;
     int64_t gstride_bits = 0, gstride_vals = 0;
     int gblocks = 0;
 
@@ -366,7 +365,7 @@ void cut_chunks(spgemm_plan_s *P, const int64_t *pre, int64_t total, int64_t cap
 }
 
 SymArgs sym_args(spgemm_plan_s *P, int64_t r0, int64_t r1, int tiers) {
-    SymArgs sa;
+    SymArgs sa{};
     sa.A = P->A;
     sa.B = P->B;
     sa.bnd = P->bnd;
@@ -375,14 +374,13 @@ SymArgs sym_args(spgemm_plan_s *P, int64_t r0, int64_t r1, int tiers) {
     sa.r1 = r1;
     sa.listB = P->listB;
     sa.listG = P->listG;
-    sa.listH = P->listH;
     sa.ctl = P->ctl;
     sa.gscratch = P->gbits_sym;
     sa.gstride = P->gstride_bits;
     sa.gblocks = P->gblocks;
-    sa.hkeys = P->hkeys_sym;
-    sa.hstride = TH_SYM;
-    sa.hblocks = P->hblocks;
+    sa.cursor = P->cur_sym;
+    sa.curstride = P->curstride;
+    sa.bblocks = P->bblocks_sym;
     sa.group = P->group;
     sa.tiers = tiers;
     return sa;
@@ -533,8 +531,6 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->listG = P->alloc<int32_t>(R, "listG");
     P->listBn = P->alloc<int32_t>(R, "numeric listB");
     P->listGn = P->alloc<int32_t>(R, "numeric listG");
-    P->listH = P->alloc<int32_t>(R, "listH");
-    P->listHn = P->alloc<int32_t>(R, "numeric listH");
     P->ctl = P->alloc<Ctl>(2, "ctl");
     P->tmp = P->alloc<int64_t>((R + SCAN_TILE - 1) / SCAN_TILE + 64, "scan scratch");
     CK(cudaMemsetAsync(P->ctl, 0, 2 * sizeof(Ctl), s));
@@ -567,27 +563,29 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->products = (int64_t)hc.sum_u;
     P->max_u = (int64_t)hc.max_u;
     P->max_bound = (int64_t)hc.max_bound;
+    P->max_deg = (int64_t)hc.max_deg;
 
-    // arena-resident accumulator scratch, sized only if a row can exceed the CTA tier:
-    //   H (global hash, per CTA: TH_NUM keys + values for the numeric pass, TH_SYM keys for the
-    //   symbolic pass -- separate, so both passes may run concurrently on two streams) and
+    // arena-resident accumulator scratch, sized only if a row can exceed one CTA-tier piece:
+    //   cursors of the pieced CTA tier (per CTA: 2 x curstride int32 for each pass -- separate,
+    //   so both passes may run concurrently on two streams) and
     //   G (dense, per CTA: a bitmap for each pass + fp64 [ncols] for the numeric pass).
-    //   Together at most 1/4 of what is left after the smallest ring.
+    //   The dense scratch takes at most 1/4 of what is left after the smallest ring.
     if (P->max_bound > CAPB_NUM) {
+        const Grids &gr = grids(P->device, P->num_sms);
+        P->curstride = (std::min<int64_t>(std::max<int64_t>(P->max_deg, 1), CURSOR_MAX) + 31) & ~int64_t(31);
+        P->bblocks_sym = gr.symb_blocks;
+        P->bblocks_num = gr.numb_blocks;
+        P->cur_sym = P->alloc<int32_t>(int64_t(P->bblocks_sym) * 2 * P->curstride, "CTA-tier cursors (symbolic)");
+        P->cur_num = P->alloc<int32_t>(int64_t(P->bblocks_num) * 2 * P->curstride, "CTA-tier cursors (numeric)");
         const int64_t nwords = (P->ncols + 31) / 32;
         const size_t ring_min = size_t(P->ring) * size_t(P->max_bound) * 12 + 4096;
         const size_t freeb = P->arena_bytes > P->used ? P->arena_bytes - P->used : 0;
         const size_t avail = freeb > ring_min ? (freeb - ring_min) / 4 : 0;
-        // H
-        const size_t hper = size_t(TH_NUM) * 12 + size_t(TH_SYM) * 4;
-        int64_t nh = std::min<int64_t>(2 * P->num_sms, int64_t((avail / 2) / hper));
-        // G (always some: the H pass hands clustered rows to it)
         P->gstride_bits = (nwords + 63) & ~int64_t(63);
         P->gstride_vals = (P->ncols + 31) & ~int64_t(31);
         const size_t gper = size_t(P->gstride_bits) * 8 + size_t(P->gstride_vals) * 8;
-        const size_t gavail = avail - size_t(std::max<int64_t>(nh, 0)) * hper;
-        const int64_t gwant = P->max_bound > CAPH_NUM ? P->num_sms : 8;
-        int64_t ng = std::min<int64_t>(gwant, int64_t(gavail / gper));
+        const int64_t gwant = (P->max_bound > CAPS_NUM || P->max_deg > CURSOR_MAX) ? P->num_sms : 8;
+        int64_t ng = std::min<int64_t>(gwant, int64_t(avail / gper));
         if (ng < 1) {
             const size_t fb = P->arena_bytes > P->used + ring_min ? P->arena_bytes - P->used - ring_min : 0;
             ng = fb >= gper ? 1 : 0;
@@ -600,12 +598,6 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         CK(cudaMemsetAsync(P->gbits, 0, size_t(P->gstride_bits) * ng * 4, s));
         CK(cudaMemsetAsync(P->gbits_sym, 0, size_t(P->gstride_bits) * ng * 4, s));
         CK(cudaMemsetAsync(P->gvals, 0, size_t(P->gstride_vals) * ng * 8, s));
-        if (nh > 0) {
-            P->hblocks = (int)nh;
-            P->hkeys_num = P->alloc<int32_t>(TH_NUM * nh, "global-hash keys (numeric)");
-            P->hvals_num = P->alloc<double>(TH_NUM * nh, "global-hash values (numeric)");
-            P->hkeys_sym = P->alloc<int32_t>(TH_SYM * nh, "global-hash keys (symbolic)");
-        }
     }
 
     // ring capacity from what is left: each slot holds `cap` nonzeros (val fp64 + col int32)
@@ -745,17 +737,15 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t max_row_nnz, cu
     na.out_val = P->ring_val[b];
     na.listB = P->listBn;
     na.listG = P->listGn;
-    na.listH = P->listHn;
     na.ctl = P->ctl + 1;
     na.gbits = P->gbits;
     na.gvals = P->gvals;
     na.gstride_bits = P->gstride_bits;
     na.gstride_vals = P->gstride_vals;
     na.gblocks = P->gblocks;
-    na.hkeys = P->hkeys_num;
-    na.hvals = P->hvals_num;
-    na.hstride = TH_NUM;
-    na.hblocks = P->hblocks;
+    na.cursor = P->cur_num;
+    na.curstride = P->curstride;
+    na.bblocks = P->bblocks_num;
     na.group = P->group;
     na.tiers = num_tiers(max_row_nnz);
     launch_numeric(na, P->num_sms, P->stream, ev);

@@ -17,21 +17,27 @@ struct DevCSR {
 
 // Accumulator tiers.  A row is handled by
 //   W: one warp, shared-memory hash table of TW_* slots   (bound <= CAPW_*)
-//   B: one CTA,  shared-memory hash table of TB_* slots   (bound <= CAPB_*)
-//   G: one CTA,  dense bitmap (+ fp64 array) over all columns in arena scratch (any bound)
+//   B: one CTA,  shared-memory hash table of TB_* slots.  A row with bound <= CAPB_* is one piece;
+//      a longer one (bound <= CAPS_*) is cut into column pieces [lo, hi) processed one after the
+//      other in the same table, each A entry's B row resumed from a per-entry cursor -- the paper's
+//      column panels with its col_offset cursors (§III-D), applied per row, so every
+//      accumulation stays in shared memory.  Pieces are written in column order at a running
+//      offset, so the numeric pass needs no per-piece counts from the symbolic pass.
+//   G: one CTA,  dense bitmap (+ fp64 array) over all columns in arena scratch (the rest: very
+//      long rows, where density makes dense accumulation the cheaper one, §III-B)
 // where bound = min(products, ncols) in the symbolic pass and the exact nnz in the numeric pass.
 constexpr int WARPS_W = 8;                 // warps per CTA in the W kernels
+// hash tables are at most half full (CAP = T / 2; table_log2 in kernels.cu), except the W symbolic
+// table whose bound (products) over-estimates nnz (C2: 729 products, 125 nnz per row)
 constexpr int TW_SYM = 1024, CAPW_SYM = 768;
-constexpr int TW_NUM = 512, CAPW_NUM = 384;
-constexpr int THREADS_B = 512;
-constexpr int TB_SYM = 32768, CAPB_SYM = 24576;
-constexpr int TB_NUM = 16384, CAPB_NUM = 12288;
+constexpr int TW_NUM = 512, CAPW_NUM = 256;
+constexpr int THREADS_B = 512;             // 2 CTAs per SM (96 KB / 64 KB of table + 13 KB)
+constexpr int TB_SYM = 16384, CAPB_SYM = 8192;
+constexpr int TB_NUM = 8192, CAPB_NUM = 4096;
+constexpr int PIECE_SYM = 8192, PIECE_NUM = 4096;   // target bound / nnz per column piece
+constexpr int64_t CAPS_SYM = 32 * int64_t(PIECE_SYM), CAPS_NUM = 32 * int64_t(PIECE_NUM);  // <= 32 pieces
+constexpr int CURSOR_MAX = 32768;          // longest A row a pieced row may have (cursor scratch)
 constexpr int THREADS_G = 512;
-// H: one CTA, hash table in this CTA's arena slice (L2-resident for typical rows), same bucket sort
-constexpr int64_t TH_SYM = int64_t(1) << 20, CAPH_SYM = (TH_SYM / 4) * 3;
-constexpr int64_t TH_NUM = int64_t(1) << 19, CAPH_NUM = (TH_NUM / 4) * 3;
-constexpr int THREADS_H = 512;
-constexpr int HBUCKETS = 2048;             // max MSD buckets of an H row (<= 512 entries each)
 constexpr int ROW_BATCH = 16;              // rows a warp claims per atomic in the W kernels
 
 // Per-pass control block in the arena (zeroed with cudaMemsetAsync before each pass).
@@ -39,7 +45,7 @@ struct Ctl {
     unsigned long long row_ctr;   // W kernels: next row batch                      } reset before
     unsigned int nB, nG;          // long-row list lengths                          } every pass
     unsigned long long pass_max;  // symbolic: max nnz of a row in this pass        } (32 bytes)
-    unsigned int nH, pad0;        // global-hash list length                        }
+    unsigned int pad1, pad0;      //                                                }
     unsigned int err;             // bit 0: numeric count mismatch; bit 1: invalid input; bit 2: table overflow
     unsigned int pad;
     unsigned long long sum_u;     // count pass: sum of products
@@ -47,7 +53,8 @@ struct Ctl {
     unsigned long long max_bound; // count pass: max min(products, ncols)
     unsigned long long max_nnz;   // symbolic pass: max nnz in a row
     unsigned long long rows_w, rows_b, rows_g;
-    unsigned long long pad2[6];
+    unsigned long long max_deg;   // count pass: longest row of A (cursor scratch of pieced rows)
+    unsigned long long pad2[5];
 };
 
 // --- launchers (all asynchronous on `s`) ---------------------------------------------------
@@ -66,27 +73,23 @@ struct SymArgs {
     const int64_t *bnd;  // per-row bound min(products, ncols) from the count pass
     int32_t *nnz;        // out: nnz of every row in [r0, r1)
     int64_t r0, r1;      // rows of this pass
-    int32_t *listB, *listG, *listH;
+    int32_t *listB, *listG;
     Ctl *ctl;
     uint32_t *gscratch;  // G tier: per-CTA bitmap of ceil(ncols/32) words, zero on entry and exit
     int64_t gstride;     // words per CTA slot
     int gblocks;         // CTAs in the G kernel
-    int32_t *hkeys;      // H tier: per-CTA key table of hstride slots
-    int64_t hstride;
-    int hblocks;
+    int32_t *cursor;     // B tier, pieced rows: per-CTA 2 x curstride int32 cursors (NULL: none)
+    int64_t curstride;
+    int bblocks;         // CTAs in the B kernel (the cursor scratch holds that many slots)
     int group;           // lanes per A entry in the W kernel (4, 8, 16, 32)
-    int tiers;           // bit 0: launch the CTA tier, bit 1: the dense tier, bit 2: the global-hash
-                         // tier (host knows when a pass cannot have such rows and skips launches)
+    int tiers;           // bit 0: launch the CTA tier, bit 1: the dense tier (the host knows when a
+                         // pass cannot have such rows and skips launches)
     int batch;           // rows per claim in the W kernel (set by the launcher)
 };
 
 // tier bits for a pass whose rows have bound <= maxb
-inline int sym_tiers(int64_t maxb) {
-    return (maxb > CAPW_SYM ? 1 : 0) | (maxb > CAPH_SYM ? 2 : 0) | (maxb > CAPB_SYM ? 4 : 0);
-}
-inline int num_tiers(int64_t maxnnz) {
-    return (maxnnz > CAPW_NUM ? 1 : 0) | (maxnnz > CAPH_NUM ? 2 : 0) | (maxnnz > CAPB_NUM ? 4 : 0);
-}
+inline int sym_tiers(int64_t maxb) { return (maxb > CAPW_SYM ? 1 : 0) | (maxb > CAPS_SYM ? 2 : 0); }
+inline int num_tiers(int64_t maxnnz) { return (maxnnz > CAPW_NUM ? 1 : 0) | (maxnnz > CAPS_NUM ? 2 : 0); }
 
 // host2[0] = *end (a chunk's end offset), host2[1] = ctl->pass_max -- zero-copy stores into mapped
 // pinned memory, so no small D2H copy queues behind the big ones on the copy engine
@@ -120,20 +123,19 @@ struct NumArgs {
     int64_t r0, r1;      // chunk rows
     int32_t *out_col;    // ring slot: nnz of the chunk
     double *out_val;
-    int32_t *listB, *listG, *listH;
+    int32_t *listB, *listG;
     Ctl *ctl;
     uint32_t *gbits;     // G tier scratch: per CTA gstride_bits words of bitmap ...
     double *gvals;       // ... and gstride_vals doubles, all zero on entry and exit
     int64_t gstride_bits, gstride_vals;
     int gblocks;
-    int32_t *hkeys;      // H tier: per-CTA table of hstride slots (keys + values)
-    double *hvals;
-    int64_t hstride;
-    int hblocks;
+    int32_t *cursor;     // as in SymArgs (a separate scratch: both passes may run concurrently)
+    int64_t curstride;
+    int bblocks;
     int group;
     int tiers;           // as in SymArgs
     int batch;
-    int tload;           // W tier table sizing: 0 -> >= 4n/3 slots, 1 -> >= 2n, 2 -> >= 4n (capped at TW_NUM)
+    int tload;           // W tier table sizing: 0 -> >= 2n slots, 1 -> >= 3n, 2 -> >= 4n (capped at TW_NUM)
 };
 // S6+S7: numeric pass over chunk rows [r0, r1); ev as in launch_symbolic
 void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);
@@ -146,7 +148,7 @@ int choose_group(const DevCSR &B, int64_t nnzB);
 
 // occupancy-derived grid sizes (queried once per device)
 struct Grids {
-    int count_blocks, symw_blocks, numw_blocks, numw3_blocks, symb_blocks, numb_blocks;
+    int count_blocks, symw_blocks, numw_blocks, symb_blocks, numb_blocks;
 };
 const Grids &grids(int device, int num_sms);
 

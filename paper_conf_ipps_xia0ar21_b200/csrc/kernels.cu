@@ -38,9 +38,11 @@ __device__ __forceinline__ uint32_t hslot(int32_t c, int lg) {
     return ((uint32_t)c * 0x9E3779B1u) >> (32 - lg);
 }
 
-// log2 of the table size for a row with `bound` distinct keys: load factor <= 3/4, >= 32 slots
+// log2 of the table size for a row with `bound` distinct keys: load factor <= 1/2, >= 32 slots.
+// (At load 3/4 linear probing's unsuccessful searches average 8.5 probes and a warp waits for its
+// slowest lane; with CR ~ 1 -- R-MAT, C3 -- nearly every product is an unsuccessful search.)
 __device__ __forceinline__ int table_log2(int64_t bound, int maxlg) {
-    int64_t need = bound + bound / 3 + 1;
+    const int64_t need = 2 * bound;
     int lg = 5;
     while (lg < maxlg && (int64_t(1) << lg) < need) ++lg;
     return lg;
@@ -199,14 +201,16 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
     }
 }
 
-// ------------------------------------------------------------------ CTA product iterator (B/H/G)
+// ------------------------------------------------------------------ CTA product iterator (B/G)
 //
-// Visits every product of row i with a whole CTA, load-balanced: A entries are taken BATCH at a
-// time, a block scan of their B-row lengths flattens the products, and thread t handles products
-// t, t + NT, ...  (coalesced B loads), locating its A entry by binary search in shared memory.
-// One warp per A entry would leave the CTA waiting on the longest B row -- a hub row of a
-// power-law graph holds thousands of entries.
-constexpr int PBATCH = 1024;
+// Visits every product of row i with a whole CTA, load-balanced: A entries are taken PBATCH at a
+// time, a block scan of their B-row segment lengths flattens the products, and thread t handles
+// products t, t + NT, ...  (coalesced B loads), locating its A entry by binary search in shared
+// memory.  One warp per A entry would leave the CTA waiting on the longest B row -- a hub row of a
+// power-law graph holds thousands of entries.  seg(e, k, s0, e0, s, en) picks the segment [s, en)
+// of B row k = [s0, e0) that entry e (its index within the row) contributes: the whole row, or
+// one column piece of it (PieceSeg).
+constexpr int PBATCH = 512;
 struct ProdSmem {
     int64_t off[PBATCH + 1];
     int64_t bs[PBATCH];
@@ -214,9 +218,38 @@ struct ProdSmem {
     int64_t scan[40];
 };
 
-template <int NT, bool VALS, typename F>
+struct WholeSeg {
+    __device__ __forceinline__ void operator()(int, int32_t, int64_t s0, int64_t e0, int64_t &s, int64_t &en) const {
+        s = s0;
+        en = e0;
+    }
+};
+
+// Column piece [.., hi) of every B row, resumed at the entry's cursor (offset within the B row
+// of the first column not yet consumed by earlier pieces); the end of the segment -- the first
+// column >= hi, by binary search -- is left in nxt[e] for the next piece (the paper's col_offset,
+// P:L182).  cur / nxt live in this CTA's global scratch slot.
+struct PieceSeg {
+    const int32_t *bcol;
+    const int32_t *cur;
+    int32_t *nxt;
+    int32_t hi;
+    __device__ __forceinline__ void operator()(int e, int32_t, int64_t s0, int64_t e0, int64_t &s, int64_t &en) const {
+        s = s0 + cur[e];
+        int64_t lo = s, h = e0;
+        while (lo < h) {
+            const int64_t m = (lo + h) >> 1;
+            if (__ldg(&bcol[m]) < hi) lo = m + 1;
+            else h = m;
+        }
+        en = lo;
+        nxt[e] = (int32_t)(lo - s0);
+    }
+};
+
+template <int NT, bool VALS, typename SEG, typename F>
 __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmem &sm,
-                                                   F &&f) {
+                                                   const SEG &seg, F &&f) {
     constexpr int PER = PBATCH / NT;
     const int64_t as = A.rp[i], ae = A.rp[i + 1];
     for (int64_t pb = as; pb < ae; pb += PBATCH) {
@@ -230,8 +263,10 @@ __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR
             double av = 0.0;
             if (e < nb) {
                 const int32_t k = __ldg(&A.col[pb + e]);
-                bs = __ldg(&B.rp[k]);
-                len = __ldg(&B.rp[k + 1]) - bs;
+                int64_t s, en;
+                seg((int)(pb - as) + e, k, __ldg(&B.rp[k]), __ldg(&B.rp[k + 1]), s, en);
+                bs = s;
+                len = en - s;
                 if (VALS) av = __ldg(&A.val[pb + e]);
             }
             if (e < PBATCH) {
@@ -263,6 +298,11 @@ __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR
         }
         __syncthreads();
     }
+}
+
+template <int NT, bool VALS, typename F>
+__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmem &sm, F &&f) {
+    block_row_products<NT, VALS>(A, B, i, sm, WholeSeg{}, f);
 }
 
 // find-or-insert of a column in a warp-private table; returns the slot
@@ -328,9 +368,10 @@ __device__ __forceinline__ void warp_fill_zero(double *v, int n) {
 __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__restrict__ u, Ctl *ctl) {
     const int lane = threadIdx.x & 31;
     const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
-    unsigned long long lsum = 0, lmax = 0, lmaxb = 0;
+    unsigned long long lsum = 0, lmax = 0, lmaxb = 0, ldeg = 0;
     for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < A.nrows; i += nw) {
         const int64_t s = A.rp[i], e = A.rp[i + 1];
+        ldeg = max(ldeg, (unsigned long long)(e - s));
         int64_t acc = 0;
         for (int64_t p = s + lane; p < e; p += 32) {
             const int32_t k = __ldg(&A.col[p]);
@@ -349,6 +390,7 @@ __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__re
         atomicMax(&ctl->max_u, lmax);
         atomicMax(&ctl->max_bound, lmaxb);
     }
+    if (lane == 0 && ldeg) atomicMax(&ctl->max_deg, ldeg);
 }
 
 // --------------------------------------------------------------------------------- validation
@@ -380,16 +422,15 @@ __global__ void k_add(int64_t *rp, int64_t n, int64_t d) {
 
 // ------------------------------------------------------------------------ tier classification
 
-// rows too long for a warp: CTA tier (shared-memory hash) up to capB, global-hash tier up to capH
-// (when that tier has scratch), dense tier beyond
-__device__ __forceinline__ void push_long(int64_t i, int64_t bound, int64_t capB, int64_t capH, bool have_h,
-                                          int32_t *listB, int32_t *listH, int32_t *listG, Ctl *ctl) {
-    if (bound <= capB) {
+// rows too long for a warp: the CTA tier (one piece up to capB; column pieces up to capS when the
+// pass has cursor scratch and the row's A entries fit it), the dense tier beyond
+__device__ __forceinline__ void push_long(int64_t i, int64_t bound, const DevCSR &A, int64_t capB, int64_t capS,
+                                          const int32_t *cursor, int64_t curstride, int32_t *listB, int32_t *listG,
+                                          Ctl *ctl) {
+    const bool pieces_ok = cursor != nullptr && bound <= capS && A.rp[i + 1] - A.rp[i] <= curstride;
+    if (bound <= capB || pieces_ok) {
         unsigned idx = atomicAdd(&ctl->nB, 1u);
         listB[idx] = (int32_t)i;
-    } else if (have_h && bound <= capH) {
-        unsigned idx = atomicAdd(&ctl->nH, 1u);
-        listH[idx] = (int32_t)i;
     } else {
         unsigned idx = atomicAdd(&ctl->nG, 1u);
         listG[idx] = (int32_t)i;
@@ -426,7 +467,7 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
             }
             if (bound > CAPW_SYM) {
                 if (lane == 0) {
-                    push_long(i, bound, CAPB_SYM, CAPH_SYM, a.hblocks > 0, a.listB, a.listH, a.listG, a.ctl);
+                    push_long(i, bound, a.A, CAPB_SYM, CAPS_SYM, a.cursor, a.curstride, a.listB, a.listG, a.ctl);
                     nlong++;
                 }
                 continue;
@@ -461,28 +502,128 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
 
 // ----------------------------------------------------------------------------- S4 symbolic, B
 
-__global__ void __launch_bounds__(THREADS_B) k_sym_b(SymArgs a) {
-    extern __shared__ int32_t keys[];
-    __shared__ int64_t s_scan[40];
+// Insert with an occupancy count (CTA tables): *ins counts fresh keys; past `limit` the piece is
+// abandoned (*ovf = 1) and later inserts are skipped, so a table never fills beyond
+// limit + (threads in flight) and probing always ends.  Returns the slot, or -1 if skipped.
+__device__ __forceinline__ int insert_counted(int32_t *keys, int32_t c, int lg, int *ins, int limit,
+                                              volatile int *ovf) {
+    if (*ovf) return -1;
+    const uint32_t mask = (1u << lg) - 1;
+    uint32_t h = hslot(c, lg);
+    volatile int32_t *vk = keys;
+    while (true) {
+        const int32_t k = vk[h];
+        if (k == c) return (int)h;
+        if (k == EMPTY) {
+            const int32_t old = atomicCAS(&keys[h], EMPTY, c);
+            if (old == EMPTY) {
+                if (atomicAdd(ins, 1) >= limit) *ovf = 1;
+                return (int)h;
+            }
+            if (old == c) return (int)h;
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+// [cmin, cmax] of row i's columns: the first and last column of every B row it touches
+template <int NT>
+__device__ __forceinline__ void row_col_span(const DevCSR &A, const DevCSR &B, int64_t i, int *s_span) {
+    if (threadIdx.x == 0) {
+        s_span[0] = INT_MAX;
+        s_span[1] = -1;
+    }
+    __syncthreads();
+    int mn = INT_MAX, mx = -1;
+    for (int64_t p = A.rp[i] + threadIdx.x; p < A.rp[i + 1]; p += NT) {
+        const int32_t k = __ldg(&A.col[p]);
+        const int64_t s0 = __ldg(&B.rp[k]), e0 = __ldg(&B.rp[k + 1]);
+        if (e0 > s0) {
+            mn = min(mn, __ldg(&B.col[s0]));
+            mx = max(mx, __ldg(&B.col[e0 - 1]));
+        }
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) {
+        mn = min(mn, __shfl_xor_sync(FULLMASK, mn, d));
+        mx = max(mx, __shfl_xor_sync(FULLMASK, mx, d));
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicMin(&s_span[0], mn);
+        atomicMax(&s_span[1], mx);
+    }
+    __syncthreads();
+}
+
+// Column pieces of a long row (both passes): P = ceil(bound / target) pieces of equal width over
+// the row's column span, processed in column order; a piece whose table passes its limit is
+// halved and redone (the cursors advance only when a piece succeeds).  piece(lo, hi) runs the
+// products of the piece and returns false on overflow; done(lo, hi) consumes a successful piece.
+template <int NT, typename PIECE, typename DONE>
+__device__ __forceinline__ void row_pieces(const DevCSR &A, const DevCSR &B, int64_t i, int64_t bound, int target,
+                                           int32_t *cur, const int32_t *nxt, int *s_span, PIECE &&piece,
+                                           DONE &&done) {
+    row_col_span<NT>(A, B, i, s_span);
+    const int64_t cmin = s_span[0], cmax = s_span[1];
+    const int64_t deg = A.rp[i + 1] - A.rp[i];
+    for (int64_t e = threadIdx.x; e < deg; e += NT) cur[e] = 0;
+    __syncthreads();
+    if (cmax < cmin) return;  // no products
+    const int64_t P = (bound + target - 1) / target;
+    const int64_t width = (cmax - cmin + P) / P;
+    for (int64_t lo = cmin; lo <= cmax;) {
+        int64_t hi = min(lo + width, cmax + 1);
+        while (!piece((int32_t)lo, (int32_t)hi)) {
+            __syncthreads();
+            hi = lo + ((hi - lo) / 2 > 1 ? (hi - lo) / 2 : 1);
+        }
+        done();
+        for (int64_t e = threadIdx.x; e < deg; e += NT) cur[e] = nxt[e];
+        __syncthreads();
+        lo = hi;
+    }
+}
+
+__global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
+    extern __shared__ __align__(16) int32_t keys[];
     __shared__ ProdSmem psm;
-    constexpr int MAXLG = 15;  // log2(TB_SYM)
+    __shared__ int s_ins, s_ovf, s_span[2];
+    constexpr int MAXLG = 14;  // log2(TB_SYM)
+    constexpr int LIMIT = (TB_SYM / 4) * 3;
+    int32_t *cur = a.cursor ? a.cursor + (int64_t)blockIdx.x * 2 * a.curstride : nullptr;
+    int32_t *nxt = cur ? cur + a.curstride : nullptr;
     const unsigned n = *(volatile unsigned *)&a.ctl->nB;
     for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
         const int64_t i = a.listB[idx];
         const int64_t bound = a.bnd[i];
-        const int lg = table_log2(bound, MAXLG);
-        const int T = 1 << lg;
-        for (int t = threadIdx.x; t < T; t += THREADS_B) keys[t] = EMPTY;
-        __syncthreads();
-        int cnt = 0;
-        block_row_products<THREADS_B, false>(a.A, a.B, i, psm,
-                                             [&](int32_t c, double) { cnt += sym_insert(keys, c, lg); });
-        int64_t tot;
-        block_excl_scan<THREADS_B>(cnt, s_scan, &tot);
+        int64_t total = 0;
+        // one table pass over the products of [lo, hi) (whole row: seg = WholeSeg)
+        auto pass = [&](int lg, const auto &seg, int limit) {
+            const int T = 1 << lg;
+            for (int t = threadIdx.x; t < T; t += THREADS_B) keys[t] = EMPTY;
+            if (threadIdx.x == 0) {
+                s_ins = 0;
+                s_ovf = 0;
+            }
+            __syncthreads();
+            block_row_products<THREADS_B, false>(a.A, a.B, i, psm, seg, [&](int32_t c, double) {
+                insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
+            });  // ends with a barrier
+            return s_ovf == 0;
+        };
+        if (bound <= CAPB_SYM) {
+            pass(table_log2(bound, MAXLG), WholeSeg{}, INT_MAX);
+            total = s_ins;
+        } else {
+            row_pieces<THREADS_B>(
+                a.A, a.B, i, bound, PIECE_SYM, cur, nxt, s_span,
+                [&](int32_t lo, int32_t hi) { return pass(MAXLG, PieceSeg{a.B.col, cur, nxt, hi}, LIMIT); },
+                [&]() { total += s_ins; });
+        }
         if (threadIdx.x == 0) {
-            a.nnz[i] = (int32_t)tot;
-            atomicMax(&a.ctl->max_nnz, (unsigned long long)tot);
-            atomicMax(&a.ctl->pass_max, (unsigned long long)tot);
+            a.nnz[i] = (int32_t)total;
+            atomicMax(&a.ctl->max_nnz, (unsigned long long)total);
+            atomicMax(&a.ctl->pass_max, (unsigned long long)total);
             atomicAdd(&a.ctl->rows_b, 1ull);
         }
         __syncthreads();
@@ -728,8 +869,8 @@ __device__ __forceinline__ void sort_emit_any(const unsigned long long *pk, int 
     }
 }
 
-template <int G, bool WIDE, int MINB>
-__global__ void __launch_bounds__(WARPS_W * 32, MINB) k_num_w(NumArgs a) {
+template <int G, bool WIDE>
+__global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
     extern __shared__ __align__(16) double smem_d[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     AStage *ast = reinterpret_cast<AStage *>(smem_d) + wid;  // A-entry staging first (16-B aligned)
@@ -756,10 +897,10 @@ __global__ void __launch_bounds__(WARPS_W * 32, MINB) k_num_w(NumArgs a) {
             const int64_t n = a.crp[i + 1] - o;
             if (n == 0) continue;
             if (n > CAPW_NUM) {
-                if (lane == 0) push_long(i, n, CAPB_NUM, CAPH_NUM, a.hblocks > 0, a.listB, a.listH, a.listG, a.ctl);
+                if (lane == 0) push_long(i, n, a.A, CAPB_NUM, CAPS_NUM, a.cursor, a.curstride, a.listB, a.listG, a.ctl);
                 continue;
             }
-            const int lg = table_log2(a.tload == 0 ? n : a.tload == 1 ? (3 * n) / 2 : 3 * n, MAXLG);
+            const int lg = table_log2(a.tload == 0 ? n : a.tload == 1 ? (3 * n) / 2 : 2 * n, MAXLG);
             const int T = 1 << lg;
             warp_fill_keys(keys, T);
             warp_fill_zero(vals, T);
@@ -831,321 +972,189 @@ __global__ void __launch_bounds__(WARPS_W * 32, MINB) k_num_w(NumArgs a) {
 
 // ------------------------------------------------------------------------------ S6 numeric, B
 
-__global__ void __launch_bounds__(THREADS_B) k_num_b(NumArgs a) {
-    extern __shared__ double smem_d[];
-    double *vals = smem_d;
-    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);
-    __shared__ int64_t s_scan[40];
-    __shared__ ProdSmem psm;
-    __shared__ int s_cnt[64], s_cur[64], s_start[64], s_mm[3], s_occ[THREADS_B / 32];
+struct CtaSortSmem {
+    int cnt[64], cur[64], start[64], mm[3], occ[THREADS_B / 32];
+    int64_t scan[40];
+};
+
+template <typename T>
+__device__ __forceinline__ T warp_incl_scan(T x) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const T y = __shfl_up_sync(FULLMASK, x, d);
+        if (lane >= d) x += y;
+    }
+    return x;
+}
+
+// S7 for a CTA table of T slots holding n keys (+ values): one MSD pass (bucket by column within
+// the table's column range), the packed keys (column << SB | slot) staged in the output value
+// area, then each bucket sorted by one warp in registers.  A bucket over 512 entries (very
+// clustered columns) takes the general path: compaction + shared-memory bitonic.  Writes oc/ov
+// [0, n); returns false (nothing written) if the table does not hold exactly n keys.  All
+// threads call; ends with a barrier.
+template <int SB>
+__device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int32_t *oc, double *ov,
+                              CtaSortSmem &ss) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     constexpr int NW = THREADS_B / 32;
-    constexpr int MAXLG = 14;  // log2(TB_NUM)
+    const int P = min(64, max(1, (int)((n + 255) / 256)));
+    if (threadIdx.x < 64) ss.cnt[threadIdx.x] = 0;
+    if (threadIdx.x == 0) {
+        ss.mm[0] = INT_MAX;
+        ss.mm[1] = -1;
+    }
+    __syncthreads();
+    {
+        int lmin = INT_MAX, lmax = -1, occ = 0;
+        for (int t = threadIdx.x; t < T; t += THREADS_B) {
+            const int32_t k = keys[t];
+            if (k != EMPTY) {
+                lmin = min(lmin, k);
+                lmax = max(lmax, k);
+                ++occ;
+            }
+        }
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) {
+            lmin = min(lmin, __shfl_xor_sync(FULLMASK, lmin, d));
+            lmax = max(lmax, __shfl_xor_sync(FULLMASK, lmax, d));
+            occ += __shfl_xor_sync(FULLMASK, occ, d);
+        }
+        if (lane == 0) {
+            atomicMin(&ss.mm[0], lmin);
+            atomicMax(&ss.mm[1], lmax);
+            ss.occ[wid] = occ;
+        }
+    }
+    __syncthreads();
+    int occ_total = 0;
+#pragma unroll
+    for (int w = 0; w < NW; ++w) occ_total += ss.occ[w];
+    if (occ_total != n || n == 0) {
+        __syncthreads();
+        return occ_total == n;
+    }
+    const int64_t lo = ss.mm[0], span = (int64_t)ss.mm[1] - lo + 1;
+    for (int t = threadIdx.x; t < T; t += THREADS_B) {
+        const int32_t k = keys[t];
+        if (k != EMPTY) atomicAdd(&ss.cnt[(int)(((int64_t)k - lo) * P / span)], 1);
+    }
+    __syncthreads();
+    if (wid == 0) {  // bucket starts (lane l owns buckets l and l + 32) and the largest bucket
+        const int c0 = lane < P ? ss.cnt[lane] : 0, c1 = lane + 32 < P ? ss.cnt[lane + 32] : 0;
+        const int i0 = warp_incl_scan(c0), i1 = warp_incl_scan(c1);
+        const int tot0 = __shfl_sync(FULLMASK, i0, 31);
+        if (lane < P) ss.start[lane] = ss.cur[lane] = i0 - c0;
+        if (lane + 32 < P) ss.start[lane + 32] = ss.cur[lane + 32] = tot0 + i1 - c1;
+        int big = max(c0, c1);
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) big = max(big, __shfl_xor_sync(FULLMASK, big, d));
+        if (lane == 0) ss.mm[2] = big;
+    }
+    __syncthreads();
+    if (ss.mm[2] <= 512) {
+        unsigned long long *stage = reinterpret_cast<unsigned long long *>(ov);
+        for (int t = threadIdx.x; t < T; t += THREADS_B) {
+            const int32_t k = keys[t];
+            if (k != EMPTY) {
+                const int pos = atomicAdd(&ss.cur[(int)(((int64_t)k - lo) * P / span)], 1);
+                stage[pos] = ((unsigned long long)(uint32_t)k << SB) | (unsigned)t;
+            }
+        }
+        __syncthreads();  // staged keys (global) visible to the block
+        for (int b = wid; b < P; b += NW) {
+            const int st = ss.start[b], m = ss.cnt[b];
+            if (m == 0) continue;
+            sort_emit_any<SB, true, false>(stage + st, m, vals, oc + st, ov + st);
+        }
+        __syncthreads();
+        return true;
+    }
+    // general path: in-place compaction + shared-memory bitonic sort
+    int64_t cnt = 0;
+    for (int t0 = 0; t0 < T; t0 += THREADS_B) {
+        const int t = t0 + threadIdx.x;
+        const int32_t k = t < T ? keys[t] : EMPTY;
+        const double v = t < T ? vals[t] : 0.0;
+        const int occ = k != EMPTY;
+        int64_t tot;
+        const int64_t ex = block_excl_scan<THREADS_B>(occ, ss.scan, &tot);  // ends with a barrier
+        if (occ) {
+            keys[cnt + ex] = k;
+            vals[cnt + ex] = v;
+        }
+        cnt += tot;
+        __syncthreads();
+    }
+    const int N = pow2_at_least(n, 32);
+    for (int t = (int)n + threadIdx.x; t < N; t += THREADS_B) keys[t] = INT_MAX;
+    __syncthreads();
+    block_bitonic<THREADS_B>(keys, vals, N);
+    for (int t = threadIdx.x; t < n; t += THREADS_B) {
+        oc[t] = keys[t];
+        ov[t] = vals[t];
+    }
+    __syncthreads();
+    return true;
+}
+
+__global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
+    extern __shared__ __align__(16) double smem_d[];
+    double *vals = smem_d;
+    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);
+    __shared__ ProdSmem psm;
+    __shared__ CtaSortSmem ss;
+    __shared__ int s_ins, s_ovf, s_span[2];
+    constexpr int MAXLG = 13;  // log2(TB_NUM)
+    constexpr int LIMIT = (TB_NUM / 4) * 3;
+    int32_t *cur = a.cursor ? a.cursor + (int64_t)blockIdx.x * 2 * a.curstride : nullptr;
+    int32_t *nxt = cur ? cur + a.curstride : nullptr;
     const unsigned nrows = *(volatile unsigned *)&a.ctl->nB;
     const int64_t off0 = a.crp[a.r0];
     for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
         const int64_t i = a.listB[idx];
         const int64_t o = a.crp[i];
         const int64_t n = a.crp[i + 1] - o;
-        const int lg = table_log2(n, MAXLG);
-        const int T = 1 << lg;
-        for (int t = threadIdx.x; t < T; t += THREADS_B) {
-            keys[t] = EMPTY;
-            vals[t] = 0.0;
-        }
-        __syncthreads();
-        block_row_products<THREADS_B, true>(a.A, a.B, i, psm,
-                                            [&](int32_t c, double v) { num_insert(keys, vals, c, v, lg); });
         int32_t *oc = a.out_col + (o - off0);
         double *ov = a.out_val + (o - off0);
-        // S7 for CTA rows: one MSD pass (bucket by column within the row's column range), the
-        // packed keys (column << 14 | slot) staged in the row's own output value area, then each
-        // bucket sorted by one warp in registers.  A bucket over 512 entries (very clustered
-        // columns) sends the row to the general path: compaction + shared-memory bitonic.
-        const int P = min(64, max(1, (int)((n + 255) / 256)));
-        if (threadIdx.x < 64) s_cnt[threadIdx.x] = 0;
-        if (threadIdx.x == 0) {
-            s_mm[0] = INT_MAX;
-            s_mm[1] = -1;
-        }
-        __syncthreads();
-        {
-            int lmin = INT_MAX, lmax = -1, occ = 0;
+        auto pass = [&](int lg, const auto &seg, int limit) {
+            const int T = 1 << lg;
             for (int t = threadIdx.x; t < T; t += THREADS_B) {
-                const int32_t k = keys[t];
-                if (k != EMPTY) {
-                    lmin = min(lmin, k);
-                    lmax = max(lmax, k);
-                    ++occ;
-                }
+                keys[t] = EMPTY;
+                vals[t] = 0.0;
             }
-#pragma unroll
-            for (int d = 16; d > 0; d >>= 1) {
-                lmin = min(lmin, __shfl_xor_sync(FULLMASK, lmin, d));
-                lmax = max(lmax, __shfl_xor_sync(FULLMASK, lmax, d));
-                occ += __shfl_xor_sync(FULLMASK, occ, d);
-            }
-            if (lane == 0) {
-                atomicMin(&s_mm[0], lmin);
-                atomicMax(&s_mm[1], lmax);
-                s_occ[wid] = occ;
-            }
-        }
-        __syncthreads();
-        int occ_total = 0;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) occ_total += s_occ[w];
-        if (occ_total != n) {
-            if (threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
-            __syncthreads();
-            continue;
-        }
-        const int64_t lo = s_mm[0], span = (int64_t)s_mm[1] - lo + 1;
-        for (int t = threadIdx.x; t < T; t += THREADS_B) {
-            const int32_t k = keys[t];
-            if (k != EMPTY) atomicAdd(&s_cnt[(int)(((int64_t)k - lo) * P / span)], 1);
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            int run = 0, big = 0;
-            for (int b = 0; b < P; ++b) {
-                s_start[b] = run;
-                s_cur[b] = run;
-                run += s_cnt[b];
-                big = max(big, s_cnt[b]);
-            }
-            s_mm[2] = big;
-        }
-        __syncthreads();
-        if (s_mm[2] <= 512) {
-            unsigned long long *stage = reinterpret_cast<unsigned long long *>(ov);
-            for (int t = threadIdx.x; t < T; t += THREADS_B) {
-                const int32_t k = keys[t];
-                if (k != EMPTY) {
-                    const int pos = atomicAdd(&s_cur[(int)(((int64_t)k - lo) * P / span)], 1);
-                    stage[pos] = ((unsigned long long)(uint32_t)k << 14) | (unsigned)t;
-                }
-            }
-            __syncthreads();  // staged keys (global) visible to the block
-            for (int b = wid; b < P; b += NW) {
-                const int st = s_start[b], m = s_cnt[b];
-                if (m == 0) continue;
-                sort_emit_any<14, true, false>(stage + st, m, vals, oc + st, ov + st);
-            }
-            __syncthreads();
-            continue;
-        }
-        // general path: in-place compaction + shared-memory bitonic sort
-        int64_t cnt = 0;
-        for (int t0 = 0; t0 < T; t0 += THREADS_B) {
-            const int t = t0 + threadIdx.x;
-            const int32_t k = t < T ? keys[t] : EMPTY;
-            const double v = t < T ? vals[t] : 0.0;
-            const int occ = k != EMPTY;
-            int64_t tot;
-            const int64_t ex = block_excl_scan<THREADS_B>(occ, s_scan, &tot);  // ends with a barrier
-            if (occ) {
-                keys[cnt + ex] = k;
-                vals[cnt + ex] = v;
-            }
-            cnt += tot;
-            __syncthreads();
-        }
-        const int N = pow2_at_least(n, 32);
-        for (int t = (int)n + threadIdx.x; t < N; t += THREADS_B) keys[t] = INT_MAX;
-        __syncthreads();
-        block_bitonic<THREADS_B>(keys, vals, N);
-        for (int t = threadIdx.x; t < n; t += THREADS_B) {
-            oc[t] = keys[t];
-            ov[t] = vals[t];
-        }
-        __syncthreads();
-    }
-}
-
-// ----------------------------------------------------------------- S4 / S6, global-hash tier H
-// CTA per row, open-addressing table (int32 keys, fp64 values) in this CTA's arena slice, sized
-// per row (load <= 3/4).  Rows of a few 10^4 .. 10^5 nonzeros keep their table in L2.  The numeric
-// pass sorts like the CTA tier: one MSD bucket pass over the row's column range, keys staged in
-// the row's own output, a register sort per bucket; a row whose buckets overflow (clustered
-// columns) is handed to the dense tier, which runs after this kernel.
-
-__device__ __forceinline__ int sym_insert_g(int32_t *keys, int32_t c, int lg) {
-    const uint32_t mask = (1u << lg) - 1;
-    uint32_t h = hslot(c, lg);
-    while (true) {
-        const int32_t k = __ldcg(keys + h);
-        if (k == c) return 0;
-        if (k == EMPTY) {
-            const int32_t old = atomicCAS(&keys[h], EMPTY, c);
-            if (old == EMPTY) return 1;
-            if (old == c) return 0;
-        }
-        h = (h + 1) & mask;
-    }
-}
-
-__global__ void __launch_bounds__(THREADS_H) k_sym_h(SymArgs a) {
-    __shared__ int64_t s_scan[40];
-    __shared__ ProdSmem psm;
-    int32_t *keys = a.hkeys + (int64_t)blockIdx.x * a.hstride;
-    const unsigned nrows = *(volatile unsigned *)&a.ctl->nH;
-    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
-        const int64_t i = a.listH[idx];
-        const int lg = table_log2(a.bnd[i], 20);
-        const int T = 1 << lg;
-        int4 *k4 = reinterpret_cast<int4 *>(keys);
-        for (int t = threadIdx.x; t < (T >> 2); t += THREADS_H) k4[t] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
-        __syncthreads();
-        int cnt = 0;
-        block_row_products<THREADS_H, false>(a.A, a.B, i, psm,
-                                             [&](int32_t c, double) { cnt += sym_insert_g(keys, c, lg); });
-        int64_t tot;
-        block_excl_scan<THREADS_H>(cnt, s_scan, &tot);
-        if (threadIdx.x == 0) {
-            a.nnz[i] = (int32_t)tot;
-            atomicMax(&a.ctl->max_nnz, (unsigned long long)tot);
-            atomicMax(&a.ctl->pass_max, (unsigned long long)tot);
-            atomicAdd(&a.ctl->rows_g, 1ull);
-        }
-        __syncthreads();
-    }
-}
-
-__global__ void __launch_bounds__(THREADS_H) k_num_h(NumArgs a) {
-    __shared__ int64_t s_scan[40];
-    __shared__ ProdSmem psm;
-    // bucket counts and cursors; a bucket's start is its cursor minus its count after the scatter
-    __shared__ int s_cnt[HBUCKETS], s_cur[HBUCKETS], s_mm[3], s_occ[THREADS_H / 32];
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    constexpr int NW = THREADS_H / 32;
-    int32_t *keys = a.hkeys + (int64_t)blockIdx.x * a.hstride;
-    double *vals = a.hvals + (int64_t)blockIdx.x * a.hstride;
-    const unsigned nrows = *(volatile unsigned *)&a.ctl->nH;
-    const int64_t off0 = a.crp[a.r0];
-    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
-        const int64_t i = a.listH[idx];
-        const int64_t o = a.crp[i];
-        const int n = (int)(a.crp[i + 1] - o);
-        const int lg = table_log2(n, 19);
-        const int T = 1 << lg;
-        {
-            int4 *k4 = reinterpret_cast<int4 *>(keys);
-            double2 *v2 = reinterpret_cast<double2 *>(vals);
-            for (int t = threadIdx.x; t < (T >> 2); t += THREADS_H) k4[t] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
-            for (int t = threadIdx.x; t < (T >> 1); t += THREADS_H) v2[t] = make_double2(0.0, 0.0);
-        }
-        const int P = min(HBUCKETS, max(1, (n + 255) / 256));
-        for (int b = threadIdx.x; b < P; b += THREADS_H) s_cnt[b] = 0;
-        if (threadIdx.x == 0) {
-            s_mm[0] = INT_MAX;
-            s_mm[1] = -1;
-        }
-        __syncthreads();
-        block_row_products<THREADS_H, true>(a.A, a.B, i, psm, [&](int32_t c, double v) {
-            const uint32_t mask = (1u << lg) - 1;
-            uint32_t h = hslot(c, lg);
-            while (true) {
-                const int32_t kk = __ldcg(keys + h);
-                if (kk == c) break;
-                if (kk == EMPTY) {
-                    const int32_t old = atomicCAS(&keys[h], EMPTY, c);
-                    if (old == EMPTY || old == c) break;
-                }
-                h = (h + 1) & mask;
-            }
-            atomicAdd(&vals[h], v);
-        });
-        int32_t *oc = a.out_col + (o - off0);
-        double *ov = a.out_val + (o - off0);
-        {
-            int lmin = INT_MAX, lmax = -1, occ = 0;
-            for (int t = threadIdx.x; t < T; t += THREADS_H) {
-                const int32_t k = __ldcg(keys + t);
-                if (k != EMPTY) {
-                    lmin = min(lmin, k);
-                    lmax = max(lmax, k);
-                    ++occ;
-                }
-            }
-#pragma unroll
-            for (int d = 16; d > 0; d >>= 1) {
-                lmin = min(lmin, __shfl_xor_sync(FULLMASK, lmin, d));
-                lmax = max(lmax, __shfl_xor_sync(FULLMASK, lmax, d));
-                occ += __shfl_xor_sync(FULLMASK, occ, d);
-            }
-            if (lane == 0) {
-                atomicMin(&s_mm[0], lmin);
-                atomicMax(&s_mm[1], lmax);
-                s_occ[wid] = occ;
-            }
-        }
-        __syncthreads();
-        int occ_total = 0;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) occ_total += s_occ[w];
-        if (occ_total != n) {
-            if (threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
-            __syncthreads();
-            continue;
-        }
-        const int64_t lo = s_mm[0], span = (int64_t)s_mm[1] - lo + 1;
-        for (int t = threadIdx.x; t < T; t += THREADS_H) {
-            const int32_t k = __ldcg(keys + t);
-            if (k != EMPTY) atomicAdd(&s_cnt[(int)(((int64_t)k - lo) * P / span)], 1);
-        }
-        __syncthreads();
-        {   // bucket starts: block scan over P <= HBUCKETS counts, 4 per thread
-            constexpr int PER = HBUCKETS / THREADS_H;
-            int loc[PER], sum = 0;
-#pragma unroll
-            for (int k = 0; k < PER; ++k) {
-                const int b = threadIdx.x * PER + k;
-                loc[k] = b < P ? s_cnt[b] : 0;
-                sum += loc[k];
-            }
-            int64_t tot;
-            int run = (int)block_excl_scan<THREADS_H>(sum, s_scan, &tot);
-#pragma unroll
-            for (int k = 0; k < PER; ++k) {
-                const int b = threadIdx.x * PER + k;
-                if (b < P) s_cur[b] = run;
-                run += loc[k];
-            }
-        }
-        if (threadIdx.x == 0) s_mm[2] = 0;
-        __syncthreads();
-        {
-            int big = 0;
-            for (int b = threadIdx.x; b < P; b += THREADS_H) big = max(big, s_cnt[b]);
-#pragma unroll
-            for (int d = 16; d > 0; d >>= 1) big = max(big, __shfl_xor_sync(FULLMASK, big, d));
-            if (lane == 0) atomicMax(&s_mm[2], big);
-        }
-        __syncthreads();
-        if (s_mm[2] > 512) {
-            // clustered columns: the dense tier (launched after this kernel) takes the row
             if (threadIdx.x == 0) {
-                const unsigned gi = atomicAdd(&a.ctl->nG, 1u);
-                a.listG[gi] = (int32_t)i;
+                s_ins = 0;
+                s_ovf = 0;
             }
             __syncthreads();
-            continue;
+            block_row_products<THREADS_B, true>(a.A, a.B, i, psm, seg, [&](int32_t c, double v) {
+                const int h = insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
+                if (h >= 0) atomicAdd(&vals[h], v);
+            });  // ends with a barrier
+            return s_ovf == 0;
+        };
+        bool ok = true;
+        if (n <= CAPB_NUM) {
+            const int lg = table_log2(n, MAXLG);
+            pass(lg, WholeSeg{}, INT_MAX);
+            ok = cta_sort_emit<MAXLG>(keys, vals, 1 << lg, n, oc, ov, ss);
+        } else {
+            int64_t written = 0;
+            row_pieces<THREADS_B>(
+                a.A, a.B, i, n, PIECE_NUM, cur, nxt, s_span,
+                [&](int32_t lo, int32_t hi) { return pass(MAXLG, PieceSeg{a.B.col, cur, nxt, hi}, LIMIT); },
+                [&]() {
+                    const int m = s_ins;
+                    if (written + m <= n) ok &= cta_sort_emit<MAXLG>(keys, vals, TB_NUM, m, oc + written, ov + written, ss);
+                    else ok = false;
+                    written += m;
+                });
+            ok &= written == n;
         }
-        unsigned long long *stage = reinterpret_cast<unsigned long long *>(ov);
-        for (int t = threadIdx.x; t < T; t += THREADS_H) {
-            const int32_t k = __ldcg(keys + t);
-            if (k != EMPTY) {
-                const int pos = atomicAdd(&s_cur[(int)(((int64_t)k - lo) * P / span)], 1);
-                stage[pos] = ((unsigned long long)(uint32_t)k << 20) | (unsigned)t;
-            }
-        }
-        __syncthreads();
-        for (int b = wid; b < P; b += NW) {
-            const int m = s_cnt[b], st = s_cur[b] - m;
-            if (m == 0) continue;
-            sort_emit_any<20, true, true>(stage + st, m, vals, oc + st, ov + st);
-        }
+        if (!ok && threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
         __syncthreads();
     }
 }
@@ -1214,10 +1223,8 @@ size_t numb_smem() { return size_t(TB_NUM) * (sizeof(int32_t) + sizeof(double));
 template <int G>
 static void set_attrs_w() {
     cudaFuncSetAttribute(k_sym_w<G>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symw_smem());
-    cudaFuncSetAttribute(k_num_w<G, false, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(false));
-    cudaFuncSetAttribute(k_num_w<G, true, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(true));
-    cudaFuncSetAttribute(k_num_w<G, false, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(false));
-    cudaFuncSetAttribute(k_num_w<G, true, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(true));
+    cudaFuncSetAttribute(k_num_w<G, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(false));
+    cudaFuncSetAttribute(k_num_w<G, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numw_smem(true));
 }
 
 const Grids &grids(int device, int num_sms) {
@@ -1237,10 +1244,8 @@ const Grids &grids(int device, int num_sms) {
         g.count_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_w<8>, WARPS_W * 32, symw_smem());
         g.symw_blocks = num_sms * (occ > 0 ? occ : 1);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false, 4>, WARPS_W * 32, numw_smem(false));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false>, WARPS_W * 32, numw_smem(false));
         g.numw_blocks = num_sms * (occ > 0 ? occ : 1);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false, 3>, WARPS_W * 32, numw_smem(false));
-        g.numw3_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b, THREADS_B, symb_smem());
         g.symb_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_b, THREADS_B, numb_smem());
@@ -1299,16 +1304,11 @@ static void sym_w(const SymArgs &a, int blocks, cudaStream_t s) {
     k_sym_w<G><<<blocks, WARPS_W * 32, symw_smem(), s>>>(a);
     LAUNCHED(1);
 }
-template <int G, int MINB>
-static void num_w(const NumArgs &a, int blocks, cudaStream_t s) {
-    if (a.B.ncols > (int64_t(1) << 23)) k_num_w<G, true, MINB><<<blocks, WARPS_W * 32, numw_smem(true), s>>>(a);
-    else k_num_w<G, false, MINB><<<blocks, WARPS_W * 32, numw_smem(false), s>>>(a);
-    LAUNCHED(1);
-}
 template <int G>
-static void num_w(const NumArgs &a, int blocks, int minb, cudaStream_t s) {
-    if (minb == 3) num_w<G, 3>(a, blocks, s);
-    else num_w<G, 4>(a, blocks, s);
+static void num_w(const NumArgs &a, int blocks, cudaStream_t s) {
+    if (a.B.ncols > (int64_t(1) << 23)) k_num_w<G, true><<<blocks, WARPS_W * 32, numw_smem(true), s>>>(a);
+    else k_num_w<G, false><<<blocks, WARPS_W * 32, numw_smem(false), s>>>(a);
+    LAUNCHED(1);
 }
 static int env_int(const char *name, int dflt) {
     const char *v = getenv(name);
@@ -1349,15 +1349,14 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
     }
     rec(ev, 1, s);
     if (a.tiers & 1) {
-        k_sym_b<<<g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
+        k_sym_b<<<a.cursor ? a.bblocks : g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
         LAUNCHED(1);
     }
     rec(ev, 2, s);
-    if ((a.tiers & 4) && a.hblocks > 0) {
-        k_sym_h<<<a.hblocks, THREADS_H, 0, s>>>(a);
-        LAUNCHED(1);
-    }
-    if (((a.tiers & 2) || ((a.tiers & 4) && a.hblocks == 0)) && a.gblocks > 0) {
+    // the dense tier: rows beyond the pieced CTA tier, and rows whose A entries do not fit the
+    // cursor scratch (possible whenever the pass has CTA-tier rows; the kernel exits at once
+    // when its list is empty)
+    if ((a.tiers & 3) && a.gblocks > 0) {
         k_sym_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
         LAUNCHED(1);
     }
@@ -1375,33 +1374,24 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
     const Grids &g = grids(dev, num_sms);
     cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);
     NumArgs aw = a;
-    static const int minb = env_int("SPGEMM_NUMW_MINB", 4);  // tuning knobs
-    static const int tload = env_int("SPGEMM_NUMW_TLOAD", 2);
+    static const int tload = env_int("SPGEMM_NUMW_TLOAD", 2);  // tuning knob
     aw.tload = tload;
-    const int full = minb == 3 ? g.numw3_blocks : g.numw_blocks;
-    aw.batch = batch_for(rows, full);
-    const int wblocks = grid_for(rows, WARPS_W * aw.batch, full);
+    aw.batch = batch_for(rows, g.numw_blocks);
+    const int wblocks = grid_for(rows, WARPS_W * aw.batch, g.numw_blocks);
     rec(ev, 0, s);
     switch (a.group) {
-        case 4: num_w<4>(aw, wblocks, minb, s); break;
-        case 8: num_w<8>(aw, wblocks, minb, s); break;
-        case 16: num_w<16>(aw, wblocks, minb, s); break;
-        default: num_w<32>(aw, wblocks, minb, s); break;
+        case 4: num_w<4>(aw, wblocks, s); break;
+        case 8: num_w<8>(aw, wblocks, s); break;
+        case 16: num_w<16>(aw, wblocks, s); break;
+        default: num_w<32>(aw, wblocks, s); break;
     }
     rec(ev, 1, s);
     if (a.tiers & 1) {
-        k_num_b<<<g.numb_blocks, THREADS_B, numb_smem(), s>>>(a);
+        k_num_b<<<a.cursor ? a.bblocks : g.numb_blocks, THREADS_B, numb_smem(), s>>>(a);
         LAUNCHED(1);
     }
     rec(ev, 2, s);
-    const bool h = (a.tiers & 4) && a.hblocks > 0;
-    if (h) {
-        k_num_h<<<a.hblocks, THREADS_H, 0, s>>>(a);
-        LAUNCHED(1);
-    }
-    // the dense tier also takes H rows whose buckets overflowed, and every long row when the
-    // H tier has no scratch
-    if (((a.tiers & 2) || (a.tiers & 4)) && a.gblocks > 0) {
+    if ((a.tiers & 3) && a.gblocks > 0) {
         k_num_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
         LAUNCHED(1);
     }

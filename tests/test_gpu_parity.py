@@ -123,14 +123,14 @@ def test_empty_b_rows_and_explicit_zeros():
 # ------------------------------------------------------------------------------------- tiers
 
 def _long_rows_case(seed=0, wide=60000, deg=240):
-    """A few rows whose products/nnz exceed the warp and CTA tiers (forces tiers B and G)."""
+    """A few rows whose products/nnz exceed the warp tier and one CTA-tier piece."""
     rng = np.random.default_rng(seed)
     k = 800
     B = W.random_csr_sparse(k, wide, deg, seed=seed + 1)
     rows = []
     for i in range(300):
         if i % 100 == 0:
-            d = 300            # ~300 * 240 = 72k products over 60k columns -> G tier
+            d = 300            # ~300 * 240 = 72k products over 60k columns -> pieced CTA tier
         elif i % 10 == 0:
             d = 12             # ~2.9k products -> B tier
         else:
@@ -143,10 +143,11 @@ def _long_rows_case(seed=0, wide=60000, deg=240):
     return A, B
 
 
-def test_tiers_warp_block_global():
+def test_tiers_warp_block_pieced():
+    """Warp rows, one-piece CTA rows and (72k products over 60k columns) pieced CTA rows."""
     A, B = _long_rows_case()
     rp, col, val, info, _ = run(A, B)
-    assert info["rows_block"] > 0 and info["rows_global"] > 0 and info["rows_warp"] > 0, info
+    assert info["rows_block"] > 0 and info["rows_warp"] > 0, info
     assert_parity(A, B, rp, col, val)
 
 
@@ -158,9 +159,9 @@ def _csr_from_rows(rows, ncols, rng):
 
 
 @pytest.mark.parametrize("fused", [False, True])
-def test_global_hash_tier_fallback_and_dense_tier(fused):
-    """Rows for the arena tiers: a clustered H-tier row (its MSD buckets overflow, so the dense tier
-    takes it), a scattered H-tier row, and a row beyond the H tier (dense tier directly)."""
+def test_pieced_cta_tier_and_dense_tier(fused):
+    """Long rows: a clustered row (its column pieces overflow the CTA table and are halved until
+    they fit), a scattered row (plain column pieces), and a row beyond the pieced tier (dense)."""
     rng = np.random.default_rng(17)
     ncols = 1_000_000
     brows = []
@@ -175,7 +176,26 @@ def test_global_hash_tier_fallback_and_dense_tier(fused):
     A = _csr_from_rows(arows, B.nrows, rng)
     r = run_fused(A, B) if fused else run(A, B)
     info = r[3]
-    assert info["rows_global"] >= 3, info
+    assert info["rows_global"] >= 1 and info["rows_block"] >= 2, info
+    assert_parity(A, B, r[0], r[1], r[2])
+
+
+@pytest.mark.parametrize("fused", [False, True])
+def test_pieced_rows_many_entries_and_dense_fallback(fused):
+    """Pieced rows whose A rows hold many entries (cursor scratch per entry), one A row longer than
+    the cursor scratch (CURSOR_MAX = 32768 entries: the dense tier takes it), empty B rows among
+    the entries, and pieces whose column ranges hold no product at all."""
+    rng = np.random.default_rng(23)
+    ncols = 3_000_000
+    brows = [np.sort(rng.choice(ncols, int(rng.integers(0, 4)), replace=False)) for _ in range(50_000)]
+    brows += [np.sort(rng.choice(ncols, 400, replace=False)) for _ in range(100)]
+    B = _csr_from_rows(brows, ncols, rng)
+    arows = [np.sort(rng.choice(50_000, 12_000, replace=False)),            # ~18k products, pieced
+             np.arange(50_000, 50_100),                                    # 40k products, pieced
+             np.sort(rng.choice(50_000, 40_000, replace=False)),           # > CURSOR_MAX entries
+             np.array([0, 1, 2]), np.array([], dtype=np.int64)]
+    A = _csr_from_rows(arows, B.nrows, rng)
+    r = run_fused(A, B) if fused else run(A, B)
     assert_parity(A, B, r[0], r[1], r[2])
 
 

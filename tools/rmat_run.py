@@ -37,12 +37,16 @@ d.col = torch.from_numpy(A.col).to(dev)
 d.val = torch.from_numpy(A.val).to(dev)
 r1 = int(A.nrows * frac)
 res = {"scale": scale, "nnz_A": int(A.nnz), "rows": r1, "gen_s": gen_s}
-for rep in range(2):
+for rep in range(int(os.environ.get("REPS", "2"))):
     got = {"nnz": 0, "chunks": 0}
+
+    rownnz = np.zeros(r1, dtype=np.int64) if os.environ.get("TIERS") else None
 
     def sink(r0_, r1_, rp, col, val):
         got["nnz"] += int(rp[-1])
         got["chunks"] += 1
+        if rownnz is not None:
+            rownnz[r0_:r1_] = np.diff(rp)
 
     torch.cuda.synchronize()
     t0 = time.perf_counter()
@@ -61,4 +65,17 @@ for rep in range(2):
                 "rows_block": info["rows_block"], "rows_global": info["rows_global"],
                 "max_row_nnz": info["max_row_nnz"], "max_row_products": info["max_row_products"],
                 "stats_ms": {k: round(v["ms"], 2) for k, v in st.items()}})
+if rownnz is not None:
+    # products and nnz per accumulator tier (numeric thresholds of internal.h: W <= 384, B <= 12288,
+    # H <= 393216, G beyond)
+    deg = np.diff(A.row_ptr)
+    prod = np.add.reduceat(deg[A.col].astype(np.int64), A.row_ptr[:-1].clip(max=max(A.nnz - 1, 0)))
+    prod[deg == 0] = 0
+    prod = prod[:r1]
+    tiers = {}
+    for name, lo, hi in (("W", 1, 384), ("B", 385, 12288), ("H", 12289, 393216), ("G", 393217, 1 << 62)):
+        m = (rownnz >= lo) & (rownnz <= hi)
+        tiers[name] = {"rows": int(m.sum()), "products": int(prod[m].sum()), "nnz": int(rownnz[m].sum()),
+                       "max_products": int(prod[m].max()) if m.any() else 0}
+    res["tiers"] = tiers
 print(json.dumps(res), flush=True)
