@@ -133,6 +133,23 @@ def probe_d2h(h_dst, dev, nbytes=1 << 30, reps=3):
     return n / best / 1e9
 
 
+def d2h_detail(tl, d2h_bytes):
+    """Copy-engine view of the last timed step from its chunk timeline: when the first copy
+    starts, how long the copy stream is busy vs idle between the first and last copy, and the
+    rate while busy (separates a slow link from a starved one)."""
+    if tl is None or len(tl) == 0:
+        return None
+    tl = tl[tl[:, 4] >= 0]  # copies are recorded on the last unit of each output chunk
+    if len(tl) == 0:
+        return None
+    c0, c1 = tl[:, 4], tl[:, 5]
+    busy = float(np.sum(c1 - c0))
+    span = float(c1[-1] - c0[0])
+    return {"first_copy_start_ms": float(c0[0]), "copy_span_ms": span, "copy_busy_ms": busy,
+            "copy_idle_ms": span - busy, "rate_while_busy_GBps": d2h_bytes / (busy / 1e3) / 1e9 if busy > 0 else None,
+            "copies": int(len(tl))}
+
+
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -362,6 +379,7 @@ def main():
         wall = time.perf_counter() - w0
     # kernel times of the last timed step (its events were recorded inside the timed region)
     stats.append(last.stats())
+    tl = capi.timeline(last)  # [chunk, 6] ms: analysis, numeric and copy start/end
     chunk_table["rows"], chunk_table["offs"] = last.chunks()
     chunk_table["info"] = last.info()
     last.free()
@@ -527,7 +545,8 @@ def main():
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": name, "budget_bytes": budget, "m": A.nrows, "nnz_A": A.nnz,
                        "products": products_total, "nnz_C": nnz_total, "C_host_bytes": d2h_bytes,
-                       "chunks": chunk_table["info"]["num_chunks"], "ring": args.ring,
+                       "chunks": chunk_table["info"]["num_chunks"], "output_copies": chunk_table["info"]["num_copies"],
+                       "ring": args.ring,
                        "plan": "fused (per-chunk symbolic overlapped with D2H)" if fused else "two-phase",
                        "l2": "inputs (686 MB) and output (3.07 GB) larger than L2; no flush needed",
                        "parallelism": f"row panels x{world}"},
@@ -539,6 +558,7 @@ def main():
             "d2h": {"bytes_per_step": d2h_bytes, "achieved_GBps": d2h_bytes / (t_max / args.steps / 1e3) / 1e9,
                     "host_link_GBps": link_gbs, "host_link_source": link_src, "host_link_bound_ms": bound_ms,
                     "frac_of_link_bound": bound_ms / (t_max / args.steps)},
+            "d2h_detail": d2h_detail(tl, d2h_bytes),
             "wall_s_timed": wall,
             "host_ms_per_step": {k: round(float(np.median(v)), 3) for k, v in host_ms.items() if v}, "pinned_output_alloc_s": pin_s,
             "parity": parity,

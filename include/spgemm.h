@@ -122,7 +122,9 @@ typedef struct {
     int64_t arena_bytes, arena_used, ring_bytes;
     int64_t rows_warp, rows_block, rows_global; /* rows per accumulator tier in the symbolic pass   */
     int32_t fused;              /* 1 if the plan is fused (nnz, max_row_nnz = -1 until executed)    */
-    int32_t reserved;
+    int32_t num_copies;         /* output chunks of the last execution: runs of consecutive chunks  */
+                                /* (num_chunks = symbolic/numeric units) that share one ring slot   */
+                                /* and leave in one copy per array (0 before the first execution)  */
 } spgemm_info;
 
 spgemm_status spgemm_plan_info(spgemm_plan_t plan, spgemm_info *info);
@@ -131,8 +133,10 @@ spgemm_status spgemm_plan_info(spgemm_plan_t plan, spgemm_info *info);
  * (offsets relative to the slice).  Arrays of num_chunks+1 entries, caller-allocated. */
 spgemm_status spgemm_plan_chunks(spgemm_plan_t plan, int64_t *rows, int64_t *offs);
 
-/* Execute = steps S6-S8: numeric hash accumulate + sort per chunk into a ring buffer, each
- * chunk D2H-copied into host memory while the next is computed.  Synchronises before return.
+/* Execute = steps S6-S8: numeric hash accumulate + sort per chunk into a ring buffer; runs of
+ * consecutive chunks share a ring slot and leave as one output chunk (one D2H copy per array,
+ * spgemm_info.num_copies), copied into host memory while the next is computed.  Synchronises
+ * before return.
  * spgemm_execute_into writes into caller memory: row_ptr [nrows+1] (may be NULL), col_idx and
  * values [nnz]; page-locked memory (cudaHostAlloc / torch pin_memory) gives asynchronous copies,
  * pageable memory is correct but slow.  Repeatable on the same plan.  On a fused plan it needs
@@ -150,8 +154,9 @@ spgemm_status spgemm_execute_capacity(spgemm_plan_t plan, int64_t *row_ptr, int3
  * (kept until free). */
 spgemm_status spgemm_execute(spgemm_plan_t plan, spgemm_csr_out *C_out);
 
-/* Sink mode for C larger than host memory: every chunk is copied into a pinned staging ring and
- * handed to cb (on the calling thread) while the GPU computes the next chunks.  row_ptr holds
+/* Sink mode for C larger than host memory: every output chunk (num_copies of them, consecutive
+ * row ranges in order) is copied into a pinned staging ring and handed to cb (on the calling
+ * thread) while the GPU computes the next chunks.  row_ptr holds
  * rows+1 offsets relative to the start of the chunk; the pointers are valid only during the call.
  * A non-zero return from cb stops execution with SPGEMM_ERR_CALLBACK. */
 typedef int (*spgemm_chunk_cb)(void *user, int64_t row0, int64_t row1, const int64_t *row_ptr,
@@ -190,8 +195,9 @@ spgemm_status spgemm_stats(spgemm_plan_t plan, spgemm_kernel_stat *stats, int32_
 
 /* Timeline of the last execution with opts.profile = 1: 6 doubles per chunk, milliseconds from the
  * start of the execution -- symbolic start, symbolic end (fused plans; -1 otherwise), numeric
- * start, numeric end (compute stream), copy start, copy end (copy stream).  *n = 6 x chunks; up to
- * max values are written. */
+ * start, numeric end (compute stream), copy start, copy end (copy stream; set on the last chunk
+ * of each output chunk, whose copies carry all of its chunks, -1 on the others).  *n = 6 x chunks;
+ * up to max values are written. */
 spgemm_status spgemm_timeline(spgemm_plan_t plan, double *out, int64_t max, int64_t *n);
 
 /* NULL-safe; frees the arena (if library-owned), streams, events and plan-owned host memory. */

@@ -54,7 +54,7 @@ class spgemm_info(ctypes.Structure):
                 ("num_chunks", ctypes.c_int32), ("ring", ctypes.c_int32), ("chunk_capacity", ctypes.c_int64),
                 ("arena_bytes", ctypes.c_int64), ("arena_used", ctypes.c_int64), ("ring_bytes", ctypes.c_int64),
                 ("rows_warp", ctypes.c_int64), ("rows_block", ctypes.c_int64), ("rows_global", ctypes.c_int64),
-                ("fused", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("fused", ctypes.c_int32), ("num_copies", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

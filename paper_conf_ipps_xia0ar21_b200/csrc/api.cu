@@ -224,6 +224,7 @@ struct spgemm_plan_s {
                                       // plan for two-phase plans, after an execution for fused)
     int64_t nnz = -1, products = 0, max_nnz = 0, max_u = 0, max_bound = 0, sum_bound = 0;
     int64_t rows_w = 0, rows_b = 0, rows_g = 0;
+    int64_t num_groups = 0;  // output chunks (copies) of the last execution
     int64_t base_applied = 0, base_wanted = 0;
     int64_t *h_small = nullptr;  // pinned + mapped: [0] base; chunk j: [1 + 2j] end offset,
     int64_t *d_small = nullptr;  //   [2 + 2j] max row nnz (fused; written by k_publish)
@@ -241,6 +242,7 @@ struct spgemm_plan_s {
         size_t per = 0;
         bool overflow = false;
         std::vector<int64_t> offs;
+        std::vector<int64_t> group_last;  // last unit of every output chunk (copy events live there)
     } pend;
     std::vector<Stat> stats;
     std::vector<double> timeline;  // profile: 6 times (ms) per chunk of the last execution
@@ -726,15 +728,15 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     }
 }
 
-void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t max_row_nnz, cudaEvent_t *ev) {
+void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t slot_off, int64_t max_row_nnz, cudaEvent_t *ev) {
     NumArgs na{};
     na.A = P->A;
     na.B = P->B;
     na.crp = P->crp;
     na.r0 = P->chunk_rows[c];
     na.r1 = P->chunk_rows[c + 1];
-    na.out_col = P->ring_col[b];
-    na.out_val = P->ring_val[b];
+    na.out_col = P->ring_col[b] + slot_off;
+    na.out_val = P->ring_val[b] + slot_off;
     na.listB = P->listBn;
     na.listG = P->listGn;
     na.ctl = P->ctl + 1;
@@ -795,9 +797,14 @@ void finalize_profile(spgemm_plan_s *P) {
             P->add_stat("num_w", elapsed(e[6], e[7]), 0);
             P->add_stat("num_b", elapsed(e[7], e[8]), 0);
             P->add_stat("num_g", elapsed(e[8], e[9]), 0);
-            cudaEvent_t end = (c + 1 < nch) ? ev[size_t(c + 1) * per + 10] : ev[size_t(nch) * per + 1];
-            P->add_stat("d2h_span", elapsed(e[10], end), double(offs[c + 1] - offs[c]) * 12);
         }
+    }
+    const std::vector<int64_t> &gl = P->pend.group_last;
+    for (size_t g = 0; g < gl.size() && !overflow; ++g) {
+        const int64_t c = gl[g];
+        cudaEvent_t end = g + 1 < gl.size() ? ev[size_t(gl[g + 1]) * per + 10] : ev[size_t(nch) * per + 1];
+        const int64_t c0 = g == 0 ? 0 : gl[g - 1] + 1;
+        P->add_stat("d2h_span", elapsed(ev[size_t(c) * per + 10], end), double(offs[c + 1] - offs[c0]) * 12);
     }
     P->add_stat("execute_total", elapsed(ev[size_t(nch) * per], ev[size_t(nch) * per + 1]),
                 double(total) * 12 + 8.0 * (P->R + 1));
@@ -814,9 +821,12 @@ void finalize_profile(spgemm_plan_s *P) {
         if (!overflow) {
             t[2] = elapsed(t0, e[6]);
             t[3] = elapsed(t0, e[9]);
-            t[4] = elapsed(t0, e[10]);
-            t[5] = elapsed(t0, e[11]);
         }
+    }
+    for (size_t g = 0; g < gl.size() && !overflow; ++g) {  // copies: on each output chunk's last unit
+        const size_t c = size_t(gl[g]);
+        P->timeline[c * 6 + 4] = elapsed(t0, ev[c * per + 10]);
+        P->timeline[c * 6 + 5] = elapsed(t0, ev[c * per + 11]);
     }
 }
 
@@ -868,7 +878,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         }
     } rel{stage};
     int64_t maxn = 0, maxr = 0;
-    for (int64_t c = 0; c < nch; ++c) maxr = std::max(maxr, P->chunk_rows[c + 1] - P->chunk_rows[c]);
+    maxr = P->R;  // an output chunk (group of units) may span any number of rows
     maxn = P->cap;
     if (sink)
         for (int r = 0; r < ring; ++r) stage[r] = pin_acquire(size_t(maxn) * 12 + size_t(maxr + 1) * 8 + 64);
@@ -897,66 +907,110 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
     std::vector<int64_t> offs(nch + 1, 0);  // chunk offsets relative to the slice
     if (!P->fused && nch > 0)
         for (int64_t c = 0; c <= nch; ++c) offs[c] = P->chunk_offs[c] - off0;
+    // Output chunks ("groups") are runs of consecutive analysis units sharing one ring slot: the
+    // copy engine moves few large pieces (a 60 MB copy runs ~8% slower than a 1 GB one on the
+    // host link) while the units stay small for a quick pipeline start.  A group closes when the
+    // next unit would not fit the slot, when it reaches its target (the first group: one unit;
+    // each later target: twice the previous group), or when the previous group's copy has
+    // finished (so the copy engine never waits for a large group to fill).
+    struct Group {
+        int b;
+        int64_t u0, u1, r0, r1, off, nnz;
+    };
+    std::vector<Group> groups;
     int64_t done_cb = 0;
-    auto consume = [&](int64_t c) {  // sink: wait for chunk c's copy and hand it over
-        const int b = int(c % ring);
-        CK(cudaEventSynchronize(P->ev_d2h[b]));
-        const int64_t r0 = P->chunk_rows[c], r1 = P->chunk_rows[c + 1];
-        int64_t *rp = st_rp(b);
+    auto consume = [&](int64_t g) {  // sink: wait for group g's copy and hand it over
+        const Group &G = groups[g];
+        CK(cudaEventSynchronize(P->ev_d2h[G.b]));
+        int64_t *rp = st_rp(G.b);
         const int64_t first = rp[0];
-        for (int64_t k = 0; k <= r1 - r0; ++k) rp[k] -= first;
-        const int rc = sink->cb(sink->user, P->row_begin + r0, P->row_begin + r1, rp, st_col(b), st_val(b), rp[r1 - r0]);
+        for (int64_t k = 0; k <= G.r1 - G.r0; ++k) rp[k] -= first;
+        const int rc = sink->cb(sink->user, P->row_begin + G.r0, P->row_begin + G.r1, rp, st_col(G.b), st_val(G.b),
+                                rp[G.r1 - G.r0]);
         if (rc != 0) {
             CK(cudaStreamSynchronize(cp));
             CK(cudaStreamSynchronize(s));
             fail(SPGEMM_ERR_CALLBACK, "chunk sink returned " + std::to_string(rc));
         }
-        done_cb = c + 1;
+        done_cb = g + 1;
+    };
+    auto close_group = [&](Group &G) {  // enqueue the group's copies after its numeric passes
+        CK(cudaEventRecord(P->ev_num[G.b], s));
+        CK(cudaStreamWaitEvent(cp, P->ev_num[G.b], 0));
+        pe.rec(size_t(G.u1 - 1) * per + 10, cp);
+        int32_t *dcol = sink ? st_col(G.b) : col_out + G.off;
+        double *dval = sink ? st_val(G.b) : val_out + G.off;
+        if (G.nnz > 0) {
+            CK(cudaMemcpyAsync(dcol, P->ring_col[G.b], sizeof(int32_t) * G.nnz, cudaMemcpyDeviceToHost, cp));
+            CK(cudaMemcpyAsync(dval, P->ring_val[G.b], sizeof(double) * G.nnz, cudaMemcpyDeviceToHost, cp));
+        }
+        if (sink) {
+            CK(cudaMemcpyAsync(st_rp(G.b), P->crp + G.r0, sizeof(int64_t) * (G.r1 - G.r0 + 1), cudaMemcpyDeviceToHost, cp));
+        } else if (rp_out && P->fused && G.r1 > G.r0) {
+            CK(cudaMemcpyAsync(rp_out + G.r0 + 1, P->crp + G.r0 + 1, sizeof(int64_t) * (G.r1 - G.r0),
+                               cudaMemcpyDeviceToHost, cp));
+        }
+        pe.rec(size_t(G.u1 - 1) * per + 11, cp);
+        CK(cudaEventRecord(P->ev_d2h[G.b], cp));
     };
 
+    Group cur{-1, 0, 0, 0, 0, 0, 0};
+    int64_t target = 0;
+    static const bool one_per_unit = [] {  // ablation knob: one output chunk per unit
+        const char *v = getenv("SPGEMM_NO_GROUPS");
+        return v && v[0] == '1';
+    }();
     for (int64_t j = 0; j < nch; ++j) {
-        const int b = int(j % ring);
         const int64_t r0 = P->chunk_rows[j], r1 = P->chunk_rows[j + 1];
         int64_t mx = P->max_nnz;
         if (P->fused) {
-            // chunk j's symbolic pass was enqueued one iteration ago; its total decides where the
-            // chunk lands on the host and its max row nnz which numeric tiers to launch
+            // unit j's symbolic pass was enqueued one iteration ago; its total decides where the
+            // unit lands on the host and its max row nnz which numeric tiers to launch
             CK(cudaEventSynchronize(P->ev_tot[j]));
             offs[j + 1] = P->h_small[1 + 2 * j] - base;
             mx = P->h_small[2 + 2 * j];
         }
         const int64_t o = offs[j], n = offs[j + 1] - offs[j];
         if (!sink && o + n > capacity) *overflow = true;
-        if (j >= ring) CK(cudaStreamWaitEvent(s, P->ev_d2h[b], 0));
+        if (*overflow) {
+            if (P->fused && j + 1 < nch) enqueue_analysis(P, j + 1, pe.at(size_t(j + 1) * per));
+            continue;
+        }
+        if (cur.b >= 0) {
+            bool close = one_per_unit || cur.nnz + n > P->cap || cur.nnz >= target;
+            if (!close && !groups.empty()) close = cudaEventQuery(P->ev_d2h[groups.back().b]) == cudaSuccess;
+            if (close) {
+                close_group(cur);
+                groups.push_back(cur);
+                target = std::min<int64_t>(P->cap, 2 * cur.nnz);
+                cur.b = -1;
+            }
+        }
+        if (cur.b < 0) {  // open a group in the next ring slot
+            const int64_t g = int64_t(groups.size());
+            cur = Group{int(g % ring), j, j, r0, r0, o, 0};
+            if (g >= ring) {
+                CK(cudaStreamWaitEvent(s, P->ev_d2h[cur.b], 0));
+                if (sink) consume(g - ring);  // frees staging slot cur.b
+            }
+        }
         if (P->fused) CK(cudaStreamWaitEvent(s, P->ev_tot[j], 0));  // (already complete: host waited)
         if (!P->chunk_wait.empty() && P->chunk_wait[j] >= 0)       // host operands: value pieces
             CK(cudaStreamWaitEvent(s, P->ev_piece[P->chunk_wait[j]], 0));
-        if (!*overflow) {
-            pe.rec(size_t(j) * per + 5, s);
-            enqueue_numeric(P, j, b, mx, pe.at(size_t(j) * per + 6));
-            CK(cudaEventRecord(P->ev_num[b], s));
-        }
+        pe.rec(size_t(j) * per + 5, s);
+        enqueue_numeric(P, j, cur.b, cur.nnz, mx, pe.at(size_t(j) * per + 6));
+        cur.nnz += n;
+        cur.u1 = j + 1;
+        cur.r1 = r1;
         if (P->fused && j + 1 < nch) enqueue_analysis(P, j + 1, pe.at(size_t(j + 1) * per));
-        if (*overflow) continue;
-        if (sink && j >= ring) consume(j - ring);  // frees staging slot b
-        CK(cudaStreamWaitEvent(cp, P->ev_num[b], 0));
-        pe.rec(size_t(j) * per + 10, cp);
-        int32_t *dcol = sink ? st_col(b) : col_out + o;
-        double *dval = sink ? st_val(b) : val_out + o;
-        if (n > 0) {
-            CK(cudaMemcpyAsync(dcol, P->ring_col[b], sizeof(int32_t) * n, cudaMemcpyDeviceToHost, cp));
-            CK(cudaMemcpyAsync(dval, P->ring_val[b], sizeof(double) * n, cudaMemcpyDeviceToHost, cp));
-        }
-        if (sink) {
-            CK(cudaMemcpyAsync(st_rp(b), P->crp + r0, sizeof(int64_t) * (r1 - r0 + 1), cudaMemcpyDeviceToHost, cp));
-        } else if (rp_out && P->fused && r1 > r0) {
-            CK(cudaMemcpyAsync(rp_out + r0 + 1, P->crp + r0 + 1, sizeof(int64_t) * (r1 - r0), cudaMemcpyDeviceToHost, cp));
-        }
-        pe.rec(size_t(j) * per + 11, cp);
-        CK(cudaEventRecord(P->ev_d2h[b], cp));
+    }
+    if (cur.b >= 0) {
+        close_group(cur);
+        groups.push_back(cur);
     }
     if (sink)
-        for (int64_t c = done_cb; c < nch; ++c) consume(c);
+        for (int64_t g = done_cb; g < int64_t(groups.size()); ++g) consume(g);
+    P->num_groups = int64_t(groups.size());
     pe.rec(size_t(nch) * per + 1, cp);
     CK(cudaStreamSynchronize(cp));
     CK(cudaStreamSynchronize(s));
@@ -983,6 +1037,8 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         P->pend.overflow = *overflow;
         P->pend.offs = offs;
         P->pend.total = total;
+        P->pend.group_last.clear();
+        for (const auto &G : groups) P->pend.group_last.push_back(G.u1 - 1);
     }
     return total;
 }
@@ -1066,6 +1122,7 @@ spgemm_status spgemm_plan_info(spgemm_plan_t P, spgemm_info *info) {
     info->rows_block = P->rows_b;
     info->rows_global = P->rows_g;
     info->fused = P->fused ? 1 : 0;
+    info->num_copies = (int32_t)P->num_groups;
     return SPGEMM_OK;
 }
 

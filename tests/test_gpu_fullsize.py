@@ -105,7 +105,7 @@ def _streamed_panel_check(A, B, r1, picks_per_chunk=2, chunk_nnz=300_000_000, se
     with capi.Plan(dA, dB, 0, o) as P:
         P.execute_stream(sink)
         info = P.info()
-    assert seen["rows"] == r1 and seen["nnz"] == info["nnz"] and seen["chunks"] == info["num_chunks"]
+    assert seen["rows"] == r1 and seen["nnz"] == info["nnz"] and seen["chunks"] == info["num_copies"]
     rows = np.array([k[0] for k in kept])
     E = oracle.spgemm(A, B, rows=rows)
     gp = np.concatenate([[0], np.cumsum([len(k[1]) for k in kept])])
@@ -161,5 +161,5 @@ def test_c3_rmat_s22_streamed():
         P.execute_stream(sink)
         info = P.info()
     assert seen["rows"] == A.nrows and seen["nnz"] == info["nnz"] and info["products"] == int(u.sum())
-    assert seen["chunks"] == info["num_chunks"] and seen["checked"] >= 2 * seen["chunks"]
+    assert seen["chunks"] == info["num_copies"] and seen["checked"] >= 2 * seen["chunks"]
     assert info["rows_global"] + info["rows_block"] > 0  # the skewed tiers were exercised

