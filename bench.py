@@ -165,20 +165,31 @@ def load_config(args):
     return A, B, budget or 0, name
 
 
-def compulsory_bytes(A, B, rows, offs, r0):
-    """Algorithmic bytes of each numeric launch: the A panel (row_ptr + col +
-    val), the C row offsets, every B row the panel touches read once (row_ptr pair + col + val),
-    and the chunk of C written once (col + val)."""
-    out = []
+def launch_bytes(A, B, rows, offs, r0, kind):
+    """Bytes of each numeric ("num") or symbolic ("sym") launch (one per analysis unit), two ways
+    (DESIGN.md §7 "Roofline"):
+      algorithmic  SURVEY §8(a) S4/S6's per-unit figures, i.e. what Gustavson's row-by-row
+                   formulation (Alg. 1) reads and writes: the A panel (row_ptr + col
+                   [+ val]), one B entry per intermediate product (col [+ val]: 4 or 12 B), the
+                   B row_ptr pair per A entry, and the unit's output (C col + val, or nnz per row);
+      compulsory   every byte touched once: the A panel, each B row the panel touches read ONCE,
+                   the output once -- the floor the L2 (126 MB) makes reachable.
+    Returns (algorithmic list, compulsory list)."""
     bl = np.diff(B.row_ptr)
+    vb = 12.0 if kind == "num" else 4.0
+    alg, comp = [], []
     for c in range(len(rows) - 1):
         a0, a1 = r0 + rows[c], r0 + rows[c + 1]
         p0, p1 = int(A.row_ptr[a0]), int(A.row_ptr[a1])
-        touched = np.unique(A.col[p0:p1])
-        nr = a1 - a0
-        out.append(16.0 * (nr + 1) + 12.0 * (p1 - p0) + 16.0 * len(touched) + 12.0 * float(bl[touched].sum())
-                   + 12.0 * float(offs[c + 1] - offs[c]))
-    return out
+        cols = A.col[p0:p1]
+        touched = np.unique(cols)
+        nr, na = a1 - a0, p1 - p0
+        prods = float(bl[cols].sum())
+        out = 12.0 * float(offs[c + 1] - offs[c]) if kind == "num" else 4.0 * nr
+        a_b = 8.0 * (nr + 1) + (12.0 if kind == "num" else 4.0) * na + 8.0 * nr  # + C row offsets / bounds
+        alg.append(a_b + 16.0 * na + vb * prods + out)
+        comp.append(a_b + 16.0 * len(touched) + vb * float(bl[touched].sum()) + out)
+    return alg, comp
 
 
 # ---------------------------------------------------------------------------------------- reference
@@ -433,21 +444,21 @@ def main():
     peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s"
     roof = None
     if dom is not None:
-        if dom.startswith("num"):
-            per_launch = compulsory_bytes(A, B, chunk_table["rows"], chunk_table["offs"], r0)
-            byts = float(np.sum(per_launch)) * nstat
-        elif dom.startswith("sym"):
-            # symbolic: A panel + u + crp + touched B rows (col only) + crp writes
-            bl = np.diff(B.row_ptr)
-            touched = np.unique(A.col[A.row_ptr[r0]:A.row_ptr[r1]])
-            byts = nstat * (24.0 * (r1 - r0) + 12.0 * (A.row_ptr[r1] - A.row_ptr[r0]) + 16.0 * len(touched)
-                                 + 4.0 * float(bl[touched].sum()))
-        else:
-            byts = 0.0
+        byts = byts_c = 0.0
+        if dom[:3] in ("num", "sym"):
+            alg, comp = launch_bytes(A, B, chunk_table["rows"], chunk_table["offs"], r0, dom[:3])
+            byts, byts_c = float(np.sum(alg)) * nstat, float(np.sum(comp)) * nstat
         ms_dom = kern[dom]["ms"]
         ach = byts / (ms_dom / 1e3) / 1e9 if ms_dom > 0 else 0.0
+        ach_c = byts_c / (ms_dom / 1e3) / 1e9 if ms_dom > 0 else 0.0
+        nl = max(1, kern[dom]["launches"])
         roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
                 "frac": ach / hbm_peak, "traffic": None, "peak_source": peak_src,
+                "bytes_per_launch": byts / nl,
+                "bytes_rule": "algorithmic: SURVEY S6/S4 per-unit figures (A panel, 12 B (num) / 4 B (sym) of B "
+                              "per intermediate product, B row_ptr pair per A entry, C out) -- DESIGN.md §7",
+                "achieved_compulsory": ach_c, "frac_compulsory": ach_c / hbm_peak,
+                "bytes_per_launch_compulsory": byts_c / nl,
                 "avg_launch_ms": ms_dom / max(1, kern[dom]["launches"]),
                 "share_of_step": (ms_dom / nstat) / (t_max / args.steps) if t_max else None,
                 "per_kernel_ms_per_step": {k: v["ms"] / nstat for k, v in agg.items()},

@@ -38,7 +38,7 @@
 extern "C" {
 #endif
 
-#define SPGEMM_ABI_VERSION 1
+#define SPGEMM_ABI_VERSION 2
 
 typedef enum {
     SPGEMM_OK = 0,
@@ -95,7 +95,19 @@ typedef struct {
                            /* 1 = fused: spgemm_plan only counts products and cuts chunks from the  */
                            /*   row bounds min(products, ncols); each chunk's symbolic pass + scan  */
                            /*   run inside execute, overlapped with the previous chunk's D2H        */
-    int32_t reserved;
+    int32_t col_panels;    /* column panels of B (Alg. 3 line 4, §III-D):                   */
+                           /*   0 = automatic: B is used whole when it fits the budget; if it does  */
+                           /*       not (SPGEMM_ERR_BUDGET), the plan is retried with B cut into the */
+                           /*       fewest column panels that fit ("column-panel mode", below);     */
+                           /*   1 = never cut B (a B too large for the budget is SPGEMM_ERR_BUDGET); */
+                           /*   >= 2 = column-panel mode with exactly this many panels.              */
+                           /* Column-panel mode: A and B stream through the device (neither needs  */
+                           /* to be resident), each chunk C[i][j] = A[i] x B[j] is computed by the   */
+                           /* same kernels, and its row pieces are stored straight into their final */
+                           /* place in host C by the GPU (zero-copy stores over the host link).     */
+                           /* Plans are two-phase (fused is ignored); sink mode is not available;   */
+                           /* output buffers should be page-locked (pageable ones are registered   */
+                           /* for the duration of the call).                                         */
 } spgemm_opts;
 
 typedef struct spgemm_plan_s *spgemm_plan_t;
@@ -125,12 +137,15 @@ typedef struct {
     int32_t num_copies;         /* output chunks of the last execution: runs of consecutive chunks  */
                                 /* (num_chunks = symbolic/numeric units) that share one ring slot   */
                                 /* and leave in one copy per array (0 before the first execution)  */
+    int32_t col_panels;         /* column panels of B (1 = B used whole)                            */
+    int32_t reserved;
 } spgemm_info;
 
 spgemm_status spgemm_plan_info(spgemm_plan_t plan, spgemm_info *info);
 
 /* Chunk table: chunk c covers C rows [rows[c], rows[c+1]) and nonzeros [offs[c], offs[c+1])
- * (offsets relative to the slice).  Arrays of num_chunks+1 entries, caller-allocated. */
+ * (offsets relative to the slice).  Arrays of num_chunks+1 entries, caller-allocated.
+ * SPGEMM_ERR_STATE for a column-panel plan (its chunks are (row unit, column panel) pairs). */
 spgemm_status spgemm_plan_chunks(spgemm_plan_t plan, int64_t *rows, int64_t *offs);
 
 /* Execute = steps S6-S8: numeric hash accumulate + sort per chunk into a ring buffer; runs of

@@ -160,4 +160,17 @@ size_t numw_smem(bool wide);
 size_t symb_smem();
 size_t numb_smem();
 
+// --- column panels of B (NEXT-1; kernels.cu "column panels") ---------------------------------
+// hist[col >> shift] += 1 over n column ids (nbins <= 4096)
+void launch_col_hist(const int32_t *col, int64_t n, int shift, int nbins, unsigned long long *hist, cudaStream_t s);
+// len[k] = entries of piece row k with lo <= col < hi
+void launch_panel_len(const DevCSR &Bp, int32_t lo, int32_t hi, int32_t *len, cudaStream_t s);
+// copy those entries to col/val at rp[k] (rp: the panel's offsets of the piece's rows)
+void launch_panel_fill(const DevCSR &Bp, int32_t lo, const int64_t *rp, int32_t *col, double *val, cudaStream_t s);
+// y[r] += x[r] for r < n; atomicMax(mx, max_r y[r]) (mx may be NULL)
+void launch_acc_i32(const int32_t *x, int32_t *y, int64_t n, unsigned long long *mx, cudaStream_t s);
+// rows [0, n) of chunk C[i][j] from a ring slot to mapped host memory at crpt[r] + pre[r] (k_scatter)
+void launch_scatter(const int32_t *scol, const double *sval, const int64_t *crpj, const int32_t *pre,
+                    const int64_t *crpt, int64_t n, int32_t *hcol, double *hval, int num_sms, cudaStream_t s);
+
 }  // namespace spg

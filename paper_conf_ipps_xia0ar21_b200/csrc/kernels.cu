@@ -1496,4 +1496,128 @@ void launch_gather(const int64_t *crp, const int64_t *idx, int64_t n, int64_t *o
     }
 }
 
+// ------------------------------------------------------------- column panels of B (NEXT-1)
+//
+// When B does not fit the device budget, B is cut into column panels B[j] = B restricted to
+// columns [lo_j, hi_j) (Alg. 3 line 4, §III-A, §III-D) and every chunk of C is
+// A[i] x B[j].  The paper partitions B on the host in two stages (count per panel, then fill,
+// L173) with a col_offset cursor per row (L182).  Here B streams through the device in row
+// pieces: a histogram of column ids picks balanced panel boundaries, and each panel is built on
+// the device by k_panel_len (two binary searches per row -- the cursor's job, without a
+// sequential scan) + the chained scan + k_panel_fill.  Column ids stay global.
+
+// hist[c >> shift] += 1 for the n column ids (nbins <= 4096; privatised in shared memory)
+__global__ void __launch_bounds__(256) k_col_hist(const int32_t *__restrict__ col, int64_t n, int shift, int nbins,
+                                                  unsigned long long *__restrict__ hist) {
+    __shared__ unsigned int h[4096];
+    for (int b = threadIdx.x; b < nbins; b += blockDim.x) h[b] = 0;
+    __syncthreads();
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(&h[__ldg(&col[i]) >> shift], 1u);
+    __syncthreads();
+    for (int b = threadIdx.x; b < nbins; b += blockDim.x)
+        if (h[b]) atomicAdd(&hist[b], (unsigned long long)h[b]);
+}
+
+// first position p in [s, e) with col[p] >= c (e if none)
+__device__ __forceinline__ int64_t lower_col(const int32_t *col, int64_t s, int64_t e, int32_t c) {
+    while (s < e) {
+        const int64_t m = (s + e) >> 1;
+        if (__ldg(&col[m]) < c) s = m + 1;
+        else e = m;
+    }
+    return s;
+}
+
+// len[k] = entries of row k of the piece with lo <= col < hi
+__global__ void k_panel_len(DevCSR Bp, int32_t lo, int32_t hi, int32_t *__restrict__ len) {
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < Bp.nrows; k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t s = Bp.rp[k], e = Bp.rp[k + 1];
+        const int64_t a = lower_col(Bp.col, s, e, lo);
+        const int64_t b = lower_col(Bp.col, a, e, hi);
+        len[k] = (int32_t)(b - a);
+    }
+}
+
+// copy the panel's entries of every row of the piece to B[j] (rp = B[j]'s offsets of these rows);
+// one warp per row, coalesced
+__global__ void k_panel_fill(DevCSR Bp, int32_t lo, const int64_t *__restrict__ rp, int32_t *__restrict__ ocol,
+                             double *__restrict__ oval) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t k = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); k < Bp.nrows; k += nw) {
+        const int64_t o = rp[k], n = rp[k + 1] - o;
+        if (n == 0) continue;
+        const int64_t a = lower_col(Bp.col, Bp.rp[k], Bp.rp[k + 1], lo);
+        for (int64_t t = lane; t < n; t += 32) {
+            ocol[o + t] = __ldg(&Bp.col[a + t]);
+            oval[o + t] = __ldg(&Bp.val[a + t]);
+        }
+    }
+}
+
+// y[r] += x[r] (row totals accumulated over the panels); *mx = max over rows of the new y
+__global__ void k_acc_i32(const int32_t *__restrict__ x, int32_t *__restrict__ y, int64_t n, unsigned long long *mx) {
+    unsigned long long m = 0;
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t t = y[r] + x[r];
+        y[r] = t;
+        m = max(m, (unsigned long long)t);
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) m = max(m, __shfl_xor_sync(FULLMASK, m, d));
+    if ((threadIdx.x & 31) == 0 && m && mx) atomicMax(mx, m);
+}
+
+// Chunk C[i][j] (rows [0, n) of a unit, packed in a ring slot at offsets crpj - crpj[0]) to its
+// final place in host C: row r's piece lands after the pieces of panels j' < j of the same row,
+// at crpt[r] + pre[r] (pre = sum of the row's earlier pieces).  The stores go straight into mapped pinned host memory
+// over the host link (zero-copy), one warp per row -- a row's pieces are not contiguous in host
+// C, so one copy-engine transfer per chunk cannot place them.
+__global__ void k_scatter(const int32_t *__restrict__ scol, const double *__restrict__ sval,
+                          const int64_t *__restrict__ crpj, const int32_t *__restrict__ pre,
+                          const int64_t *__restrict__ crpt, int64_t n, int32_t *hcol, double *hval) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+    const int64_t base = crpj[0];
+    for (int64_t r = blockIdx.x * (int64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); r < n; r += nw) {
+        const int64_t o = crpj[r] - base, len = crpj[r + 1] - crpj[r];
+        if (len == 0) continue;
+        const int64_t d = crpt[r] + pre[r];
+        for (int64_t t = lane; t < len; t += 32) hcol[d + t] = scol[o + t];
+        for (int64_t t = lane; t < len; t += 32) hval[d + t] = sval[o + t];
+    }
+}
+
+void launch_col_hist(const int32_t *col, int64_t n, int shift, int nbins, unsigned long long *hist, cudaStream_t s) {
+    if (n <= 0) return;
+    k_col_hist<<<grid_for(n, 256 * 16, 148 * 4), 256, 0, s>>>(col, n, shift, nbins, hist);
+    LAUNCHED(1);
+}
+
+void launch_panel_len(const DevCSR &Bp, int32_t lo, int32_t hi, int32_t *len, cudaStream_t s) {
+    if (Bp.nrows <= 0) return;
+    k_panel_len<<<grid_for(Bp.nrows, 256, 148 * 8), 256, 0, s>>>(Bp, lo, hi, len);
+    LAUNCHED(1);
+}
+
+void launch_panel_fill(const DevCSR &Bp, int32_t lo, const int64_t *rp, int32_t *col, double *val, cudaStream_t s) {
+    if (Bp.nrows <= 0) return;
+    k_panel_fill<<<grid_for(Bp.nrows, 8, 148 * 16), 256, 0, s>>>(Bp, lo, rp, col, val);
+    LAUNCHED(1);
+}
+
+void launch_acc_i32(const int32_t *x, int32_t *y, int64_t n, unsigned long long *mx, cudaStream_t s) {
+    if (n <= 0) return;
+    k_acc_i32<<<grid_for(n, 256, 148 * 8), 256, 0, s>>>(x, y, n, mx);
+    LAUNCHED(1);
+}
+
+void launch_scatter(const int32_t *scol, const double *sval, const int64_t *crpj, const int32_t *pre,
+                    const int64_t *crpt, int64_t n, int32_t *hcol, double *hval, int num_sms, cudaStream_t s) {
+    if (n <= 0) return;
+    k_scatter<<<grid_for(n, 8, num_sms * 4), 256, 0, s>>>(scol, sval, crpj, pre, crpt, n, hcol, hval);
+    LAUNCHED(1);
+}
+
 }  // namespace spg
