@@ -43,9 +43,8 @@ __device__ __forceinline__ uint32_t hslot(int32_t c, int lg) {
 // slowest lane; with CR ~ 1 -- R-MAT, C3 -- nearly every product is an unsuccessful search.)
 __device__ __forceinline__ int table_log2(int64_t bound, int maxlg) {
     const int64_t need = 2 * bound;
-    int lg = 5;
-    while (lg < maxlg && (int64_t(1) << lg) < need) ++lg;
-    return lg;
+    if (need <= 32) return 5;
+    return need >= (int64_t(1) << maxlg) ? maxlg : 64 - __clzll(need - 1);
 }
 
 // symbolic insert: returns 1 if `c` was not yet in the table
@@ -137,8 +136,10 @@ __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t *s, int64_
 //    G == 32 all active lanes of a round hold entries of ONE B row, i.e. distinct columns
 //    (rows are sorted and unique), which lets the numeric pass update values without atomics.
 struct AStage {
-    longlong2 be[32];  // [begin, end) of B row A.col[e] for the 32 staged A entries
-    double a[32];      // A values (numeric pass)
+    const int32_t *pc[32];  // &B.col[first entry of B row A.col[e]] for the 32 staged A entries
+    const double *pv[32];   // &B.val[...] (numeric pass)
+    int32_t len[32];        // length of that B row
+    double a[32];           // A values (numeric pass)
 };
 
 template <int G, int U, bool VALS, bool SYNC, typename F>
@@ -149,52 +150,68 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
     const int64_t as = A.rp[i], ae = A.rp[i + 1];
     for (int64_t pb = as; pb < ae; pb += 32) {
         const int64_t e = pb + lane;
-        long long bs = 0, be = 0;
+        int32_t len = 0;
+        const int32_t *pc = B.col;
+        const double *pv = B.val;
         double av = 0.0;
         if (e < ae) {
             const int32_t k = __ldg(&A.col[e]);
-            bs = __ldg(&B.rp[k]);
-            be = __ldg(&B.rp[k + 1]);
-            if (VALS) av = __ldg(&A.val[e]);
+            const int64_t bs = __ldg(&B.rp[k]);
+            len = (int32_t)(__ldg(&B.rp[k + 1]) - bs);
+            pc += bs;
+            if (VALS) {
+                pv += bs;
+                av = __ldg(&A.val[e]);
+            }
         }
+        // rows longer than a group need the remainder loop below (never on the stencils)
+        const bool any_long = __any_sync(FULLMASK, len > G);
         __syncwarp();  // the previous batch's rounds have read their entries
-        st->be[lane] = make_longlong2(bs, be);  // lanes past the row's end stage empty ranges
-        if (VALS) st->a[lane] = av;
+        st->pc[lane] = pc;  // lanes past the row's end stage empty rows
+        st->len[lane] = len;
+        if (VALS) {
+            st->pv[lane] = pv;
+            st->a[lane] = av;
+        }
         __syncwarp();
         const int nb = (int)(ae - pb < 32 ? ae - pb : 32);
         for (int t = 0; t < nb; t += R * U) {  // R * U divides 32, so src < 32
-            int64_t s[U], en[U];
-            double a[U], v[U];
             int32_t c[U];
+            double a[U], v[U];
             bool ok[U];
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const int src = t + u * R + sub;
-                const longlong2 r = st->be[src];
-                s[u] = r.x;
-                en[u] = r.y;
-                a[u] = VALS ? st->a[src] : 0.0;
-                const int64_t q = r.x + sl;
-                ok[u] = q < r.y;
-                c[u] = ok[u] ? __ldg(&B.col[q]) : 0;
-                v[u] = (VALS && ok[u]) ? __ldg(&B.val[q]) : 0.0;
+                ok[u] = sl < st->len[src];
+                c[u] = ok[u] ? __ldg(st->pc[src] + sl) : 0;
+                if (VALS) {
+                    a[u] = st->a[src];
+                    v[u] = ok[u] ? __ldg(st->pv[src] + sl) : 0.0;
+                }
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
-                f(ok[u], c[u], a[u] * v[u]);
+                f(ok[u], c[u], VALS ? a[u] * v[u] : 0.0);
                 if (SYNC) __syncwarp();
             }
-#pragma unroll
-            for (int u = 0; u < U; ++u) {
-                // remainder of B rows longer than G (uniform trip count across the warp)
-                for (int64_t q0 = s[u] + G;; q0 += G) {
-                    if (!__any_sync(FULLMASK, q0 < en[u])) break;
-                    const int64_t q = q0 + sl;
-                    const bool okk = q < en[u];
-                    const int32_t cc = okk ? __ldg(&B.col[q]) : 0;
-                    const double vv = (VALS && okk) ? __ldg(&B.val[q]) : 0.0;
-                    f(okk, cc, a[u] * vv);
-                    if (SYNC) __syncwarp();
+            if (any_long) {
+#pragma unroll 1
+                for (int u = 0; u < U; ++u) {
+                    // remainder of B rows longer than G (uniform trip count across the warp)
+                    const int src = t + u * R + sub;
+                    const int32_t *pc2 = st->pc[src];
+                    const double *pv2 = VALS ? st->pv[src] : nullptr;
+                    const int32_t ln2 = st->len[src];
+                    const double a2 = VALS ? st->a[src] : 0.0;
+                    for (int o = G;; o += G) {
+                        if (!__any_sync(FULLMASK, o < ln2)) break;
+                        const int q = o + sl;
+                        const bool okk = q < ln2;
+                        const int32_t cc = okk ? __ldg(pc2 + q) : 0;
+                        const double vv = (VALS && okk) ? __ldg(pv2 + q) : 0.0;
+                        f(okk, cc, VALS ? a2 * vv : 0.0);
+                        if (SYNC) __syncwarp();
+                    }
                 }
             }
         }
@@ -786,9 +803,8 @@ __device__ __forceinline__ void block_bitonic(int32_t *keys, double *vals, int N
 }
 
 __device__ __forceinline__ int pow2_at_least(int64_t n, int lo) {
-    int v = lo;
-    while (v < n) v <<= 1;
-    return v;
+    const int v = n <= 1 ? 1 : 1 << (64 - __clzll(n - 1));
+    return v < lo ? lo : v;
 }
 
 // ------------------------------------------------------------------------------ S6 numeric, W
@@ -927,18 +943,42 @@ __global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
             // any of it is written), into the warp's staging array for 64-bit keys.  Values stay
             // in their slots and are gathered by slot after the sort.
             int cnt = 0;
-            for (int t0 = 0; t0 < T; t0 += 32) {
-                const int32_t k = keys[t0 + lane];
-                const bool occ = k != EMPTY;
-                const unsigned bal = __ballot_sync(FULLMASK, occ);
-                const int dst = cnt + __popc(bal & ((1u << lane) - 1u));
-                __syncwarp();
-                if (occ) {
-                    if (WIDE) stage[dst] = ((unsigned long long)(uint32_t)k << 9) | (unsigned)(t0 + lane);
-                    else reinterpret_cast<uint32_t *>(keys)[dst] = ((uint32_t)k << 9) | (uint32_t)(t0 + lane);
+            const unsigned lt = (1u << lane) - 1u;
+            if (T >= 128) {
+                // 128 slots per step, 4 per lane (one LDS.128); the order of the packed keys is
+                // free (they are sorted next), so each of the 4 sub-slots is compacted by its own ballot
+                for (int t0 = 0; t0 < T; t0 += 128) {
+                    const int4 k4 = reinterpret_cast<const int4 *>(keys + t0)[lane];
+                    const int32_t kk[4] = {k4.x, k4.y, k4.z, k4.w};
+                    __syncwarp();  // the whole window is read before any write (dst < t0 + 128)
+#pragma unroll
+                    for (int r = 0; r < 4; ++r) {
+                        const bool occ = kk[r] != EMPTY;
+                        const unsigned bal = __ballot_sync(FULLMASK, occ);
+                        if (occ) {
+                            const int dst = cnt + __popc(bal & lt);
+                            const unsigned slot = (unsigned)(t0 + 4 * lane + r);
+                            if (WIDE) stage[dst] = ((unsigned long long)(uint32_t)kk[r] << 9) | slot;
+                            else reinterpret_cast<uint32_t *>(keys)[dst] = ((uint32_t)kk[r] << 9) | slot;
+                        }
+                        cnt += __popc(bal);
+                    }
+                    __syncwarp();
                 }
-                cnt += __popc(bal);
-                __syncwarp();
+            } else {
+                for (int t0 = 0; t0 < T; t0 += 32) {
+                    const int32_t k = keys[t0 + lane];
+                    const bool occ = k != EMPTY;
+                    const unsigned bal = __ballot_sync(FULLMASK, occ);
+                    const int dst = cnt + __popc(bal & lt);
+                    __syncwarp();
+                    if (occ) {
+                        if (WIDE) stage[dst] = ((unsigned long long)(uint32_t)k << 9) | (unsigned)(t0 + lane);
+                        else reinterpret_cast<uint32_t *>(keys)[dst] = ((uint32_t)k << 9) | (uint32_t)(t0 + lane);
+                    }
+                    cnt += __popc(bal);
+                    __syncwarp();
+                }
             }
             if (cnt != n) {
                 if (lane == 0) atomicOr(&a.ctl->err, 1u);
