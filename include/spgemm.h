@@ -108,6 +108,12 @@ typedef struct {
                            /* Plans are two-phase (fused is ignored); sink mode is not available;   */
                            /* output buffers should be page-locked (pageable ones are registered   */
                            /* for the duration of the call).                                         */
+    int32_t order;         /* order in which the chunks are computed and transferred (two-phase     */
+                           /*   plans; §IV-C): 0 = row order (default: consecutive chunks   */
+                           /*   then share ring slots and leave in few large copies); 1 = the       */
+                           /*   paper's schedule, decreasing number of flops (products) per chunk,  */
+                           /*   every chunk its own copy.  Fused plans and sink mode need 0.        */
+    int32_t reserved;
 } spgemm_opts;
 
 typedef struct spgemm_plan_s *spgemm_plan_t;

@@ -45,7 +45,7 @@ class spgemm_opts(ctypes.Structure):
                 ("profile", ctypes.c_int32), ("row_begin", ctypes.c_int64), ("row_end", ctypes.c_int64),
                 ("workspace", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("chunk_nnz", ctypes.c_int64),
                 ("row_ptr_base", ctypes.c_int64), ("min_chunks", ctypes.c_int64), ("fused", ctypes.c_int32),
-                ("col_panels", ctypes.c_int32)]
+                ("col_panels", ctypes.c_int32), ("order", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 class spgemm_info(ctypes.Structure):
@@ -157,7 +157,7 @@ def make_csr(M) -> tuple:
 
 def opts(device: int = -1, validate: bool = False, ring: int = 2, profile: bool = False, row_begin: int = 0,
          row_end: int = -1, workspace=None, stream=None, chunk_nnz: int = 0, row_ptr_base: int = 0,
-         min_chunks: int = 0, fused: bool = False, col_panels: int = 0) -> spgemm_opts:
+         min_chunks: int = 0, fused: bool = False, col_panels: int = 0, order: int = 0) -> spgemm_opts:
     o = spgemm_opts()
     _lib.spgemm_opts_default(ctypes.byref(o))
     o.device, o.validate, o.ring, o.profile = device, int(validate), ring, int(profile)
@@ -167,6 +167,7 @@ def opts(device: int = -1, validate: bool = False, ring: int = 2, profile: bool 
     o.chunk_nnz, o.row_ptr_base, o.min_chunks = chunk_nnz, row_ptr_base, min_chunks
     o.fused = int(fused)
     o.col_panels = int(col_panels)
+    o.order = int(order)
     o._keep = workspace  # the caller's workspace tensor must outlive the plan
     return o
 

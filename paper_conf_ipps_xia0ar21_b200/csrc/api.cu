@@ -229,6 +229,7 @@ struct spgemm_plan_s {
     int64_t rows_w = 0, rows_b = 0, rows_g = 0;
     int64_t num_groups = 0;  // output chunks (copies) of the last execution
     int64_t panel_units = 0; // column-panel plans: numeric units (chunks C[i][j]) over all panels
+    std::vector<int64_t> unit_order;  // order = 1: units by decreasing flops (empty: row order)
     int64_t base_applied = 0, base_wanted = 0;
     int64_t *h_small = nullptr;  // pinned + mapped: [0] base; chunk j: [1 + 2j] end offset,
     int64_t *d_small = nullptr;  //   [2 + 2j] max row nnz (fused; written by k_publish)
@@ -247,6 +248,7 @@ struct spgemm_plan_s {
         bool overflow = false;
         std::vector<int64_t> offs;
         std::vector<int64_t> group_last;  // last unit of every output chunk (copy events live there)
+        std::vector<int64_t> group_nnz;   // nonzeros of every output chunk
     } pend;
     std::vector<Stat> stats;
     std::vector<double> timeline;  // profile: 6 times (ms) per chunk of the last execution
@@ -407,6 +409,10 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     if (rb < 0 || re < rb || re > Ah->nrows) fail(SPGEMM_ERR_SHAPE, "row range outside A");
     if (re - rb > INT32_MAX) fail(SPGEMM_ERR_INDEX_OVERFLOW, "more than INT32_MAX rows in one plan");
     if (opts.ring < 1 || opts.ring > 64) fail(SPGEMM_ERR_INVALID_ARGUMENT, "ring must be in [1, 64]");
+    if (opts.order < 0 || opts.order > 1) fail(SPGEMM_ERR_INVALID_ARGUMENT, "order must be 0 or 1");
+    if (opts.order && opts.fused)
+        fail(SPGEMM_ERR_INVALID_ARGUMENT, "order = 1 needs a two-phase plan (a fused plan learns a chunk's host offset "
+                                          "only after the chunks before it)");
 
     if (opts.device >= 0) {
         CK(cudaSetDevice(opts.device));
@@ -647,6 +653,25 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         if (minc > 1) capp = std::min<int64_t>(capp, std::max<int64_t>(1, (total + minc - 1) / minc));
         if (opts.chunk_nnz > 0) capp = std::min<int64_t>(capp, std::max<int64_t>(1, opts.chunk_nnz - P->max_nnz));
         cut_chunks(P, P->crp, total, std::max<int64_t>(capp, 1), cap, &P->chunk_offs);
+        // §IV-C: process the chunks in decreasing order of their flops, so that a
+        // chunk's computation tends to hide under the transfer of the (larger) one before it
+        const int64_t nch = P->num_chunks();
+        if (opts.order == 1 && nch > 1) {
+            const size_t save = P->used;
+            int64_t *drows = P->alloc<int64_t>(nch + 1, "chunk rows");
+            int64_t *dfl = P->alloc<int64_t>(nch, "chunk flops");
+            std::vector<int64_t> fl(nch);
+            CK(cudaMemcpyAsync(drows, P->chunk_rows.data(), sizeof(int64_t) * (nch + 1), cudaMemcpyHostToDevice, s));
+            launch_seg_sum(P->bnd, drows, nch, dfl, s);  // bound = min(products, ncols) per row
+            CKL("chunk flops");
+            CK(cudaMemcpyAsync(fl.data(), dfl, sizeof(int64_t) * nch, cudaMemcpyDeviceToHost, s));
+            CK(cudaStreamSynchronize(s));
+            P->used = save;
+            P->unit_order.resize(nch);
+            for (int64_t j = 0; j < nch; ++j) P->unit_order[j] = j;
+            std::stable_sort(P->unit_order.begin(), P->unit_order.end(),
+                             [&](int64_t a, int64_t b) { return fl[a] > fl[b]; });
+        }
     } else {
         // fused: boundaries from the prefix of the row bounds; the symbolic pass runs per chunk
         // inside execute.  crp temporarily holds that prefix.
@@ -787,7 +812,6 @@ void finalize_profile(spgemm_plan_s *P) {
     const int64_t nch = P->pend.nch;
     const size_t per = P->pend.per;
     const bool overflow = P->pend.overflow;
-    const std::vector<int64_t> &offs = P->pend.offs;
     const int64_t total = P->pend.total;
     P->clear_stats({"num_w", "num_b", "num_g", "d2h_span", "execute_total"});
     if (P->fused) P->clear_stats({"sym_w", "sym_b", "sym_g", "scan"});
@@ -809,8 +833,7 @@ void finalize_profile(spgemm_plan_s *P) {
     for (size_t g = 0; g < gl.size() && !overflow; ++g) {
         const int64_t c = gl[g];
         cudaEvent_t end = g + 1 < gl.size() ? ev[size_t(gl[g + 1]) * per + 10] : ev[size_t(nch) * per + 1];
-        const int64_t c0 = g == 0 ? 0 : gl[g - 1] + 1;
-        P->add_stat("d2h_span", elapsed(ev[size_t(c) * per + 10], end), double(offs[c + 1] - offs[c0]) * 12);
+        P->add_stat("d2h_span", elapsed(ev[size_t(c) * per + 10], end), double(P->pend.group_nnz[g]) * 12);
     }
     P->add_stat("execute_total", elapsed(ev[size_t(nch) * per], ev[size_t(nch) * per + 1]),
                 double(total) * 12 + 8.0 * (P->R + 1));
@@ -968,11 +991,16 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
 
     Group cur{-1, 0, 0, 0, 0, 0, 0};
     int64_t target = 0;
-    static const bool one_per_unit = [] {  // ablation knob: one output chunk per unit
+    static const bool no_groups = [] {  // ablation knob: one output chunk per unit
         const char *v = getenv("SPGEMM_NO_GROUPS");
         return v && v[0] == '1';
     }();
-    for (int64_t j = 0; j < nch; ++j) {
+    // reordered chunks are not contiguous in host C: each leaves as its own copy
+    const bool reorder = !P->unit_order.empty();
+    if (reorder && sink) fail(SPGEMM_ERR_INVALID_ARGUMENT, "sink mode delivers rows in order: needs order = 0");
+    const bool one_per_unit = no_groups || reorder;
+    for (int64_t t = 0; t < nch; ++t) {
+        const int64_t j = reorder ? P->unit_order[t] : t;
         const int64_t r0 = P->chunk_rows[j], r1 = P->chunk_rows[j + 1];
         int64_t mx = P->max_nnz;
         if (P->fused) {
@@ -1050,7 +1078,11 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         P->pend.offs = offs;
         P->pend.total = total;
         P->pend.group_last.clear();
-        for (const auto &G : groups) P->pend.group_last.push_back(G.u1 - 1);
+        P->pend.group_nnz.clear();
+        for (const auto &G : groups) {
+            P->pend.group_last.push_back(G.u1 - 1);
+            P->pend.group_nnz.push_back(G.nnz);
+        }
     }
     return total;
 }

@@ -100,6 +100,8 @@ void launch_seg_max_col(const DevCSR &A, const int64_t *rows, int64_t nseg, int6
 
 // out[k] = max(x[rows[k] .. rows[k+1]-1]) for k < nseg (0 for empty segments)
 void launch_seg_max(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s);
+// out[k] = sum(x[rows[k] .. rows[k+1]-1])
+void launch_seg_sum(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s);
 // S3+S4: symbolic pass over all rows (tiering + the three tiers).  ev: NULL or 4 events recorded
 // before W, between W/B, between B/G and after G (per-kernel timing on the launching stream).
 void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);

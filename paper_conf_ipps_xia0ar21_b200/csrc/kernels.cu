@@ -1477,19 +1477,23 @@ void launch_publish(const int64_t *end, const Ctl *ctl, int64_t *host2, cudaStre
     LAUNCHED(1);
 }
 
-__global__ void __launch_bounds__(256) k_seg_max(const int64_t *__restrict__ x, const int64_t *__restrict__ rows,
-                                                 int64_t *__restrict__ out) {
+template <bool SUM>
+__global__ void __launch_bounds__(256) k_seg_reduce(const int64_t *__restrict__ x, const int64_t *__restrict__ rows,
+                                                    int64_t *__restrict__ out) {
     __shared__ int64_t s[8];
     const int64_t r0 = rows[blockIdx.x], r1 = rows[blockIdx.x + 1];
     int64_t m = 0;
-    for (int64_t i = r0 + threadIdx.x; i < r1; i += blockDim.x) m = max(m, x[i]);
+    for (int64_t i = r0 + threadIdx.x; i < r1; i += blockDim.x) m = SUM ? m + x[i] : max(m, x[i]);
 #pragma unroll
-    for (int d = 16; d > 0; d >>= 1) m = max(m, __shfl_xor_sync(FULLMASK, m, d));
+    for (int d = 16; d > 0; d >>= 1) {
+        const int64_t y = __shfl_xor_sync(FULLMASK, m, d);
+        m = SUM ? m + y : max(m, y);
+    }
     if ((threadIdx.x & 31) == 0) s[threadIdx.x >> 5] = m;
     __syncthreads();
     if (threadIdx.x == 0) {
-        for (int w = 1; w < 8; ++w) m = max(m, s[w]);
-        out[blockIdx.x] = max(m, s[0]);
+        for (int w = 1; w < 8; ++w) m = SUM ? m + s[w] : max(m, s[w]);
+        out[blockIdx.x] = m;
     }
 }
 
@@ -1519,7 +1523,13 @@ void launch_seg_max_col(const DevCSR &A, const int64_t *rows, int64_t nseg, int6
 
 void launch_seg_max(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s) {
     if (nseg <= 0) return;
-    k_seg_max<<<(unsigned)nseg, 256, 0, s>>>(x, rows, out);
+    k_seg_reduce<false><<<(unsigned)nseg, 256, 0, s>>>(x, rows, out);
+    LAUNCHED(1);
+}
+
+void launch_seg_sum(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s) {
+    if (nseg <= 0) return;
+    k_seg_reduce<true><<<(unsigned)nseg, 256, 0, s>>>(x, rows, out);
     LAUNCHED(1);
 }
 

@@ -462,3 +462,24 @@ def test_fused_sink_and_base():
     assert np.array_equal(np.array(rpg), ref[0])
     rp, c, v, info, _ = run_fused(A, A, row_ptr_base=777)
     assert rp[0] == 777 and np.array_equal(rp - 777, ref[0])
+
+
+def test_chunk_order_by_flops():
+    """§IV-C: chunks computed and transferred in decreasing order of flops give the
+    same C as row order; fused plans and sink mode reject the reordering."""
+    A = W.rmat(13, 16, seed=21)
+    ref = run(A, A, chunk_nnz=40000)
+    r = run(A, A, chunk_nnz=40000, order=1)
+    assert r[3]["num_chunks"] > 4
+    assert np.array_equal(r[0], ref[0]) and np.array_equal(r[1], ref[1])
+    assert_parity(A, A, r[0], r[1], r[2])
+    S = W.stencil_3d27(20)
+    rs = run(S, S, chunk_nnz=5000, order=1, profile=True)
+    assert_parity(S, S, rs[0], rs[1], rs[2], exact=True)
+    with pytest.raises(capi.SpgemmError) as e:
+        capi.Plan(A, A, 0, capi.opts(order=1, fused=True))
+    assert e.value.status == capi.ERR_INVALID_ARGUMENT
+    with capi.Plan(A, A, 0, capi.opts(order=1, chunk_nnz=40000)) as P:
+        with pytest.raises(capi.SpgemmError) as e:
+            P.execute_stream(lambda *a: 0)
+        assert e.value.status == capi.ERR_INVALID_ARGUMENT

@@ -8,8 +8,9 @@ through the same C ABI call as the bench step (plan + execute into pinned host C
   serial_analysis      ring 2, symbolic passes on the compute stream (no analysis/numeric overlap)
   one_copy_per_unit    ring 2, every analysis unit leaves as its own copies (no output chunks)
   two_phase            ring 2, symbolic for all rows inside spgemm_plan, then execute
+  two_phase_flops_order  two_phase with the paper's chunk schedule: decreasing flops (§IV-C)
   ring3                ring 3
-Writes gpurun_out/ablation_c2.json and prints it."""
+WL=c2 (default) or WL=rmatNN (R-MAT scale NN, C = A*A).  Writes gpurun_out/ablation_<WL>.json and prints it."""
 import json, os, subprocess, sys, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
@@ -19,6 +20,7 @@ VARIANTS = {
     "serial_analysis": ({"SPGEMM_SERIAL_ANALYSIS": "1"}, dict(ring=2, fused=True)),
     "one_copy_per_unit": ({"SPGEMM_NO_GROUPS": "1"}, dict(ring=2, fused=True)),
     "two_phase": ({}, dict(ring=2, fused=False)),
+    "two_phase_flops_order": ({}, dict(ring=2, fused=False, order=1)),
     "ring3": ({}, dict(ring=3, fused=True)),
 }
 
@@ -28,7 +30,8 @@ if len(sys.argv) > 1:  # child: one variant
     import workloads as W
     from paper_conf_ipps_xia0ar21_b200 import capi
     kw = json.loads(sys.argv[1])
-    A = W.stencil_3d27(128)
+    wl = os.environ.get("WL", "c2")
+    A = W.stencil_3d27(128) if wl == "c2" else W.rmat_torch(int(wl[4:]))
     dev = torch.device("cuda", 0)
     class D: pass
     d = D(); d.nrows, d.ncols = A.nrows, A.ncols
@@ -61,5 +64,6 @@ else:
         out[name] = json.loads(r.stdout.strip().splitlines()[-1]) if r.returncode == 0 else {"error": r.stderr[-400:]}
     out["async_vs_sync_speedup"] = out["sync"]["ms"] / out["async"]["ms"] if "ms" in out.get("sync", {}) else None
     os.makedirs("gpurun_out", exist_ok=True)
-    json.dump(out, open("gpurun_out/ablation_c2.json", "w"), indent=1)
+    out["workload"] = os.environ.get("WL", "c2")
+    json.dump(out, open(f"gpurun_out/ablation_{out['workload']}.json", "w"), indent=1)
     print(json.dumps(out, indent=1))
