@@ -522,25 +522,38 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
 // Insert with an occupancy count (CTA tables): *ins counts fresh keys; past `limit` the piece is
 // abandoned (*ovf = 1) and later inserts are skipped, so a table never fills beyond
 // limit + (threads in flight) and probing always ends.  Returns the slot, or -1 if skipped.
+// The count is aggregated per warp (one shared atomic per group of converged lanes instead of one
+// per fresh key: on R-MAT rows nearly every product is a fresh key, and 512 threads incrementing
+// one shared counter serialised the CTA tier).
 __device__ __forceinline__ int insert_counted(int32_t *keys, int32_t c, int lg, int *ins, int limit,
                                               volatile int *ovf) {
-    if (*ovf) return -1;
-    const uint32_t mask = (1u << lg) - 1;
-    uint32_t h = hslot(c, lg);
-    volatile int32_t *vk = keys;
-    while (true) {
-        const int32_t k = vk[h];
-        if (k == c) return (int)h;
-        if (k == EMPTY) {
-            const int32_t old = atomicCAS(&keys[h], EMPTY, c);
-            if (old == EMPTY) {
-                if (atomicAdd(ins, 1) >= limit) *ovf = 1;
-                return (int)h;
+    int h = -1, fresh = 0;
+    if (!*ovf) {
+        const uint32_t mask = (1u << lg) - 1;
+        uint32_t hh = hslot(c, lg);
+        volatile int32_t *vk = keys;
+        while (true) {
+            const int32_t k = vk[hh];
+            if (k == c) break;
+            if (k == EMPTY) {
+                const int32_t old = atomicCAS(&keys[hh], EMPTY, c);
+                if (old == EMPTY) {
+                    fresh = 1;
+                    break;
+                }
+                if (old == c) break;
             }
-            if (old == c) return (int)h;
+            hh = (hh + 1) & mask;
         }
-        h = (h + 1) & mask;
+        h = (int)hh;
     }
+    const unsigned m = __activemask();
+    const unsigned b = __ballot_sync(m, fresh);
+    if (b && (threadIdx.x & 31) == __ffs(m) - 1) {
+        const int cnt = __popc(b);
+        if (atomicAdd(ins, cnt) + cnt > limit) *ovf = 1;
+    }
+    return h;
 }
 
 // [cmin, cmax] of row i's columns: the first and last column of every B row it touches
@@ -1017,6 +1030,17 @@ struct CtaSortSmem {
     int64_t scan[40];
 };
 
+// fine-bucket counters of the CTA sort; they alias the product iterator's ProdSmem (not in use
+// while a table is sorted)
+constexpr int SORT_PMAX = 1024;
+struct SortCnt {
+    int cnt[SORT_PMAX], cur[SORT_PMAX], start[SORT_PMAX];
+};
+union ProdOrSort {
+    ProdSmem psm;
+    SortCnt sc;
+};
+
 template <typename T>
 __device__ __forceinline__ T warp_incl_scan(T x) {
     const int lane = threadIdx.x & 31;
@@ -1036,9 +1060,12 @@ __device__ __forceinline__ T warp_incl_scan(T x) {
 // threads call; ends with a barrier.
 template <int SB>
 __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int32_t *oc, double *ov,
-                              CtaSortSmem &ss) {
+                              CtaSortSmem &ss, SortCnt &sc) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     constexpr int NW = THREADS_B / 32;
+    // fine buckets (~4 keys each): 2^pl of them, bucket of key k = (k - lo) >> sh
+    const int pl = min(10, max(5, 32 - __clz((int)max((int64_t)1, (n + 3) / 4) - 1)));
+    for (int b = threadIdx.x; b < (1 << pl); b += THREADS_B) sc.cnt[b] = 0;
     const int P = min(64, max(1, (int)((n + 255) / 256)));
     if (threadIdx.x < 64) ss.cnt[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
@@ -1077,6 +1104,69 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         return occ_total == n;
     }
     const int64_t lo = ss.mm[0], span = (int64_t)ss.mm[1] - lo + 1;
+    {
+        // Fast path: rank inside fine buckets.  Histogram -> bucket starts -> each key staged in
+        // its bucket (in the output col area) -> each key's final position = bucket start + the
+        // number of smaller keys in its bucket.  ~4 compares per key instead of a bitonic network.
+        const int lspan = 64 - __clzll(span - 1);  // 2^lspan >= span
+        const int sh = max(0, lspan - pl);
+        for (int t = threadIdx.x; t < T; t += THREADS_B) {
+            const int32_t k = keys[t];
+            if (k != EMPTY) atomicAdd(&sc.cnt[(int)(((int64_t)k - lo) >> sh)], 1);
+        }
+        __syncthreads();
+        const int nb = (int)(((span - 1) >> sh) + 1);  // buckets in use (<= 2^pl)
+        const int b0 = 2 * threadIdx.x;
+        const int c0 = b0 < nb ? sc.cnt[b0] : 0, c1 = b0 + 1 < nb ? sc.cnt[b0 + 1] : 0;
+        int64_t tot;
+        const int64_t ex = block_excl_scan<THREADS_B>(c0 + c1, ss.scan, &tot);  // ends with a barrier
+        if (b0 < nb) sc.start[b0] = sc.cur[b0] = (int)ex;
+        if (b0 + 1 < nb) sc.start[b0 + 1] = sc.cur[b0 + 1] = (int)ex + c0;
+        int big = max(c0, c1);
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) big = max(big, __shfl_xor_sync(FULLMASK, big, d));
+        if (lane == 0) ss.occ[wid] = big;
+        __syncthreads();
+        int bmax = 0;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) bmax = max(bmax, ss.occ[w]);
+        if (bmax <= 64) {
+            for (int t = threadIdx.x; t < T; t += THREADS_B) {  // stage; keys[t] := staged position
+                const int32_t k = keys[t];
+                if (k != EMPTY) {
+                    const int pos = atomicAdd(&sc.cur[(int)(((int64_t)k - lo) >> sh)], 1);
+                    oc[pos] = k;
+                    keys[t] = pos;
+                }
+            }
+            __syncthreads();
+            for (int t = threadIdx.x; t < T; t += THREADS_B) {  // rank; value out; key parked in vals[t]
+                const int pos = keys[t];
+                if (pos != EMPTY) {
+                    const int32_t k = oc[pos];
+                    const int b = (int)(((int64_t)k - lo) >> sh);
+                    const int s0 = sc.start[b], e0 = s0 + sc.cnt[b];
+                    int r = s0, q = s0;
+                    for (; q + 4 <= e0; q += 4) {  // 4 independent loads in flight
+                        const int32_t x0 = oc[q], x1 = oc[q + 1], x2 = oc[q + 2], x3 = oc[q + 3];
+                        r += (x0 < k) + (x1 < k) + (x2 < k) + (x3 < k);
+                    }
+                    for (; q < e0; ++q) r += oc[q] < k;
+                    ov[r] = vals[t];
+                    keys[t] = r;
+                    reinterpret_cast<int32_t *>(vals + t)[0] = k;
+                }
+            }
+            __syncthreads();
+            for (int t = threadIdx.x; t < T; t += THREADS_B) {  // columns
+                const int r = keys[t];
+                if (r != EMPTY) oc[r] = reinterpret_cast<const int32_t *>(vals + t)[0];
+            }
+            __syncthreads();
+            return true;
+        }
+    }
+    // skewed columns (a fine bucket over 64 keys): coarse buckets sorted by warps in registers
     for (int t = threadIdx.x; t < T; t += THREADS_B) {
         const int32_t k = keys[t];
         if (k != EMPTY) atomicAdd(&ss.cnt[(int)(((int64_t)k - lo) * P / span)], 1);
@@ -1144,7 +1234,8 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
     extern __shared__ __align__(16) double smem_d[];
     double *vals = smem_d;
     int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);
-    __shared__ ProdSmem psm;
+    __shared__ ProdOrSort u;
+    ProdSmem &psm = u.psm;
     __shared__ CtaSortSmem ss;
     __shared__ int s_ins, s_ovf, s_span[2];
     constexpr int MAXLG = 13;  // log2(TB_NUM)
@@ -1180,7 +1271,7 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
         if (n <= CAPB_NUM) {
             const int lg = table_log2(n, MAXLG);
             pass(lg, WholeSeg{}, INT_MAX);
-            ok = cta_sort_emit<MAXLG>(keys, vals, 1 << lg, n, oc, ov, ss);
+            ok = cta_sort_emit<MAXLG>(keys, vals, 1 << lg, n, oc, ov, ss, u.sc);
         } else {
             int64_t written = 0;
             row_pieces<THREADS_B>(
@@ -1188,7 +1279,7 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
                 [&](int32_t lo, int32_t hi) { return pass(MAXLG, PieceSeg{a.B.col, cur, nxt, hi}, LIMIT); },
                 [&]() {
                     const int m = s_ins;
-                    if (written + m <= n) ok &= cta_sort_emit<MAXLG>(keys, vals, TB_NUM, m, oc + written, ov + written, ss);
+                    if (written + m <= n) ok &= cta_sort_emit<MAXLG>(keys, vals, TB_NUM, m, oc + written, ov + written, ss, u.sc);
                     else ok = false;
                     written += m;
                 });
