@@ -104,3 +104,43 @@ def test_product_package_does_not_import_oracle():
                 assert "import oracle" not in txt and "from oracle" not in txt and "liboracle" not in txt, f
     out = subprocess.run(["nm", "-D", os.path.join(pkg, "libspgemm_b200.so")], capture_output=True, text=True).stdout
     assert "oracle_" not in out
+
+
+def test_struct_layouts_match_header(capi, tmp_path):
+    """The ctypes mirrors have the C structs' sizes and field offsets (gcc on include/spgemm.h)."""
+    import ctypes as ct
+    src = tmp_path / "lay.c"
+    fields = {"spgemm_opts": ["ring", "row_begin", "workspace", "stream", "chunk_nnz", "row_ptr_base", "min_chunks",
+                              "fused", "col_panels", "order"],
+              "spgemm_info": ["num_chunks", "chunk_capacity", "rows_global", "fused", "num_copies", "col_panels"],
+              "spgemm_csr": ["row_ptr", "values", "where"], "spgemm_kernel_stat": ["launches", "ms", "bytes"]}
+    lines = ["#include <stdio.h>", "#include <stddef.h>", f'#include "{HEADER}"', "int main(void) {"]
+    for s, fs in fields.items():
+        lines.append(f'printf("{s} %zu\\n", sizeof({s}));')
+        for f in fs:
+            lines.append(f'printf("{s}.{f} %zu\\n", offsetof({s}, {f}));')
+    lines.append("return 0; }")
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "lay"
+    subprocess.run(["gcc", "-O0", "-o", str(exe), str(src)], check=True)
+    got = dict(l.split() for l in subprocess.run([str(exe)], capture_output=True, text=True).stdout.splitlines())
+    for s, fs in fields.items():
+        cls = getattr(capi, s)
+        assert int(got[s]) == ct.sizeof(cls), s
+        for f in fs:
+            assert int(got[f"{s}.{f}"]) == getattr(cls, f).offset, (s, f)
+
+
+def test_order_needs_two_phase_plan(capi):
+    """opts.order = 1 (the paper's decreasing-flops chunk schedule) is rejected on a fused plan
+    before any CUDA call."""
+    A = W.random_csr(4, 4, 0.5, seed=1)
+    ca, ka = capi.make_csr(A)
+    h = ctypes.c_void_p()
+    o = capi.opts(order=1, fused=True)
+    assert capi._lib.spgemm_plan(ctypes.byref(ca), ctypes.byref(ca), 0, ctypes.byref(o), ctypes.byref(h)) == \
+        capi.ERR_INVALID_ARGUMENT
+    assert b"two-phase" in capi._lib.spgemm_last_error()
+    o = capi.opts(order=2)
+    assert capi._lib.spgemm_plan(ctypes.byref(ca), ctypes.byref(ca), 0, ctypes.byref(o), ctypes.byref(h)) == \
+        capi.ERR_INVALID_ARGUMENT
