@@ -471,6 +471,15 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     // planning and the first chunks (the numeric pass of a chunk waits for the pieces it reads).
     std::vector<std::pair<size_t, size_t>> bval_pieces;  // (element offset, count)
     double *bval_dev = nullptr;
+    // C = A x A with host operands (A aliases B): the structure goes up in the same row pieces as
+    // the values, on the H2D stream, and the count pass of each piece's rows runs as soon as the
+    // piece has landed (it needs B.row_ptr, uploaded first, and the piece's columns), overlapping
+    // the rest of the upload
+    const bool host_alias = Bh->where == SPGEMM_HOST && Ah->where == SPGEMM_HOST && Ah->row_ptr == Bh->row_ptr &&
+                            Ah->col_idx == Bh->col_idx && Ah->values == Bh->values && Ah->nrows == Bh->nrows &&
+                            Ah->ncols == Bh->ncols;
+    const bool pieced_count = host_alias && !opts.validate && Bh->nnz > 0;
+    std::vector<cudaEvent_t> ev_col;
     if (Bh->where == SPGEMM_DEVICE) {
         P->B = DevCSR{Bh->row_ptr, Bh->col_idx, Bh->values, Bh->nrows, Bh->ncols};
     } else {
@@ -478,7 +487,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         int32_t *c = P->alloc<int32_t>(Bh->nnz, "B.col_idx");
         double *v = P->alloc<double>(Bh->nnz, "B.values");
         CK(cudaMemcpyAsync(rp, Bh->row_ptr, sizeof(int64_t) * (Bh->nrows + 1), cudaMemcpyHostToDevice, s));
-        if (Bh->nnz) CK(cudaMemcpyAsync(c, Bh->col_idx, sizeof(int32_t) * Bh->nnz, cudaMemcpyHostToDevice, s));
+        if (Bh->nnz && !pieced_count)
+            CK(cudaMemcpyAsync(c, Bh->col_idx, sizeof(int32_t) * Bh->nnz, cudaMemcpyHostToDevice, s));
         // pieces of ~32 MB of values, cut at row boundaries
         const int64_t target = std::max<int64_t>(1, (32ll << 20) / 8);
         P->bpiece_rows.push_back(0);
@@ -493,6 +503,21 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         }
         bval_dev = v;
         P->B = DevCSR{rp, c, v, Bh->nrows, Bh->ncols};
+        if (pieced_count) {
+            const size_t np = bval_pieces.size();
+            P->hstream = rs->stream(rs->hstream);
+            ev_col = rs->events(Res::PIECE, np, np);
+            cudaEvent_t rp_ready = rs->events(Res::PIECE, 2 * np, 1)[0];
+            CK(cudaEventRecord(rp_ready, s));  // allocation order + B.row_ptr queued first
+            CK(cudaStreamWaitEvent(P->hstream, rp_ready, 0));
+            for (size_t k = 0; k < np; ++k) {
+                const auto &pc = bval_pieces[k];
+                if (pc.second)
+                    CK(cudaMemcpyAsync(c + pc.first, Bh->col_idx + pc.first, sizeof(int32_t) * pc.second,
+                                       cudaMemcpyHostToDevice, P->hstream));
+                CK(cudaEventRecord(ev_col[k], P->hstream));
+            }
+        }
     }
     // S0 residency + S1 row panel: A
     if (Ah->where == SPGEMM_DEVICE) {
@@ -558,7 +583,19 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
 
     // S2 count
     pe.rec(1, s);
-    launch_count(P->A, P->B, P->bnd, P->ctl, s);
+    if (pieced_count) {
+        for (size_t k = 0; k + 1 < P->bpiece_rows.size(); ++k) {
+            const int64_t g0 = std::max<int64_t>(P->bpiece_rows[k], rb), g1 = std::min<int64_t>(P->bpiece_rows[k + 1], re);
+            CK(cudaStreamWaitEvent(s, ev_col[k], 0));
+            if (g1 <= g0) continue;
+            DevCSR Ak = P->A;
+            Ak.rp = P->A.rp + (g0 - rb);
+            Ak.nrows = g1 - g0;
+            launch_count(Ak, P->B, P->bnd + (g0 - rb), P->ctl, s);
+        }
+    } else {
+        launch_count(P->A, P->B, P->bnd, P->ctl, s);
+    }
     CKL("count");
     pe.rec(2, s);
     // fused plans: the prefix of the row bounds (chunk boundaries) is scanned before the first
@@ -749,7 +786,9 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     if (P->profile) {
         P->stats.clear();
         P->add_stat("plan_device_span", elapsed(pe.ev[0], pe.ev[9]), 0);
+        P->add_stat("plan_upload", elapsed(pe.ev[0], pe.ev[1]), 0);  // operand H2D (host operands) + setup
         P->add_stat("count", elapsed(pe.ev[1], pe.ev[2]), 0);
+        P->add_stat("plan_cut", elapsed(pe.ev[2], pe.ev[9]), 0);     // scans, cuts, round trips, ring
         if (!P->fused) {
             P->add_stat("sym_w", elapsed(pe.ev[4], pe.ev[5]), 0);
             P->add_stat("sym_b", elapsed(pe.ev[5], pe.ev[6]), 0);

@@ -1589,13 +1589,16 @@ __global__ void __launch_bounds__(256) k_seg_reduce(const int64_t *__restrict__ 
 }
 
 // out[k] = largest column index in A's rows [rows[k], rows[k+1]) (-1 if they hold no entry): the
-// last row of B a chunk reads
+// last row of B a chunk reads.  Rows are sorted, so a row's largest column is its last entry:
+// O(rows), not O(entries).
 __global__ void __launch_bounds__(256) k_seg_max_col(DevCSR A, const int64_t *__restrict__ rows,
                                                      int64_t *__restrict__ out) {
     __shared__ int s[8];
-    const int64_t p0 = A.rp[rows[blockIdx.x]], p1 = A.rp[rows[blockIdx.x + 1]];
     int m = -1;
-    for (int64_t p = p0 + threadIdx.x; p < p1; p += blockDim.x) m = max(m, A.col[p]);
+    for (int64_t i = rows[blockIdx.x] + threadIdx.x; i < rows[blockIdx.x + 1]; i += blockDim.x) {
+        const int64_t e = A.rp[i + 1];
+        if (e > A.rp[i]) m = max(m, A.col[e - 1]);
+    }
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) m = max(m, __shfl_xor_sync(FULLMASK, m, d));
     if ((threadIdx.x & 31) == 0) s[threadIdx.x >> 5] = m;
