@@ -26,6 +26,7 @@ for rep in range(4):
     P.execute_capacity(rp, col, val, z)
     t2 = time.perf_counter()
     tl = capi.timeline(P)
+    rows_, offs_ = P.chunks()
     st = P.stats()
     P.free()
     torch.cuda.synchronize()
@@ -34,3 +35,11 @@ for rep in range(4):
 t = tl
 for c in range(len(t)):
     print(f"  c{c:02d} sym {t[c,0]:7.3f}-{t[c,1]:7.3f}  num {t[c,2]:7.3f}-{t[c,3]:7.3f}  d2h {t[c,4]:7.3f}-{t[c,5]:7.3f}  gap {t[c,4]-(t[c-1,5] if c else 0):6.3f}")
+
+# copy-engine view: busy time, idle gaps and rate while busy (copies recorded on each group's last unit)
+g = [c for c in range(len(t)) if t[c, 4] >= 0]
+busy = sum(t[c, 5] - t[c, 4] for c in g)
+span = t[g[-1], 5] - t[g[0], 4]
+nbytes = 12 * int(offs_[-1] - offs_[0])
+print(f"copies {len(g)}: first start {t[g[0], 4]:.3f} ms, span {span:.3f}, busy {busy:.3f}, idle {span - busy:.3f} ms, "
+      f"rate while busy {nbytes / busy / 1e6:.2f} GB/s")
