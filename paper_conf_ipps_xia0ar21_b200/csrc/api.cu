@@ -1179,10 +1179,19 @@ struct Panels {
     cudaStream_t h = nullptr, z = nullptr;
     int64_t max_piece_nnz = 0;                    // largest (row, panel) piece
     bool validate = false;
+    // built panels parked in pinned host memory by the plan (execute then uploads each panel
+    // instead of rebuilding it from all of B); NULL if that memory could not be had
+    char *hpan = nullptr;
+    std::vector<size_t> hoff;                     // per panel: byte offset of rp | col | val
+    cudaEvent_t ev_saved = nullptr;
+    bool saved_pending = false;
 };
 
 void delete_panels(Panels *p) {
-    if (p) pin_release(p->hnp);
+    if (p) {
+        pin_release(p->hnp);
+        pin_release(p->hpan);
+    }
     delete p;
 }
 
@@ -1319,12 +1328,13 @@ void do_panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, co
     P->ev_d2h = rs->events(Res::PLAIN, P->ring, P->ring);
     P->ev_ready = rs->events(Res::PLAIN, 2 * P->ring, 1)[0];
     {
-        auto e = rs->events(Res::PLAIN, 2 * size_t(P->ring) + 1, 5);
+        auto e = rs->events(Res::PLAIN, 2 * size_t(P->ring) + 1, 6);
         Q.ev_staged[0] = e[0];
         Q.ev_staged[1] = e[1];
         Q.ev_used[0] = e[2];
         Q.ev_used[1] = e[3];
         Q.ev_scat_all = e[4];
+        Q.ev_saved = e[5];
     }
     cudaStream_t s = P->stream;
     const int64_t R = P->R, K = Bh->nrows;
@@ -1493,6 +1503,24 @@ void do_panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, co
     Q.bj_col = P->alloc<int32_t>(Q.bj_cap, "B[j].col_idx");
     Q.bj_val = P->alloc<double>(Q.bj_cap, "B[j].values");
     Q.group.assign(np, 32);
+    {
+        size_t off = 0;
+        Q.hoff.assign(size_t(np) * 3, 0);
+        for (int j = 0; j < np; ++j) {
+            Q.hoff[3 * j] = off;
+            off += al256(size_t(K + 1) * 8);
+            Q.hoff[3 * j + 1] = off;
+            off += al256(size_t(Q.pnnz[j]) * 4);
+            Q.hoff[3 * j + 2] = off;
+            off += al256(size_t(Q.pnnz[j]) * 8);
+        }
+        try {
+            Q.hpan = (char *)pin_acquire(off);
+        } catch (const Err &) {
+            Q.hpan = nullptr;  // execute rebuilds every panel from B instead
+            cudaGetLastError();
+        }
+    }
 
     // symbolic phase: per panel, build B[j] then count + symbolic of every row unit
     Q.sym_units = cut_rows(R, [&](int64_t a, int64_t b) {
@@ -1500,7 +1528,17 @@ void do_panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, co
     });
     CK(cudaMemsetAsync(Q.tot, 0, sizeof(int32_t) * R, s));
     for (int j = 0; j < np; ++j) {
+        if (Q.saved_pending) CK(cudaStreamWaitEvent(s, Q.ev_saved, 0));  // B[j-1] parked on the host
         DevCSR Bj = build_panel(P, Q, j);
+        if (Q.hpan) {  // park B[j] in pinned host memory on the copy stream, under the symbolic units
+            CK(cudaEventRecord(P->ev_ready, s));
+            CK(cudaStreamWaitEvent(Q.z, P->ev_ready, 0));
+            CK(cudaMemcpyAsync(Q.hpan + Q.hoff[3 * j], Q.bj_rp, size_t(K + 1) * 8, cudaMemcpyDeviceToHost, Q.z));
+            CK(cudaMemcpyAsync(Q.hpan + Q.hoff[3 * j + 1], Q.bj_col, size_t(Q.pnnz[j]) * 4, cudaMemcpyDeviceToHost, Q.z));
+            CK(cudaMemcpyAsync(Q.hpan + Q.hoff[3 * j + 2], Q.bj_val, size_t(Q.pnnz[j]) * 8, cudaMemcpyDeviceToHost, Q.z));
+            CK(cudaEventRecord(Q.ev_saved, Q.z));
+            Q.saved_pending = true;
+        }
         DevCSR Bc = Bj;  // the count's bound uses the panel width
         Bc.ncols = std::max<int64_t>(1, int64_t(Q.lo[j + 1]) - Q.lo[j]);
         Q.group[j] = choose_group(Bj, Q.pnnz[j]);
@@ -1596,6 +1634,7 @@ void do_panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, co
     P->chunk_offs.clear();
     P->chunk_rows.clear();
     P->panel_units = nunits;
+    if (Q.saved_pending) CK(cudaStreamWaitEvent(s, Q.ev_saved, 0));
     CK(cudaStreamSynchronize(s));
 }
 
@@ -1639,7 +1678,15 @@ int64_t run_panels(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double *
     int64_t unit = 0;
     CK(cudaMemsetAsync(Q.pre, 0, sizeof(int32_t) * R, s));
     for (int j = 0; j < Q.P; ++j) {
-        DevCSR Bj = build_panel(P, Q, j);
+        DevCSR Bj{Q.bj_rp, Q.bj_col, Q.bj_val, Q.B.nrows, Q.B.ncols};
+        if (Q.hpan) {  // upload the panel parked by the plan (after panel j-1's numeric passes, in order on s)
+            const int64_t K = Q.B.nrows;
+            CK(cudaMemcpyAsync(Q.bj_rp, Q.hpan + Q.hoff[3 * j], size_t(K + 1) * 8, cudaMemcpyHostToDevice, s));
+            CK(cudaMemcpyAsync(Q.bj_col, Q.hpan + Q.hoff[3 * j + 1], size_t(Q.pnnz[j]) * 4, cudaMemcpyHostToDevice, s));
+            CK(cudaMemcpyAsync(Q.bj_val, Q.hpan + Q.hoff[3 * j + 2], size_t(Q.pnnz[j]) * 8, cudaMemcpyHostToDevice, s));
+        } else {
+            Bj = build_panel(P, Q, j);
+        }
         if (j > 0) {  // panel j-1's scatters still read crpj, npj and pre
             CK(cudaStreamWaitEvent(s, Q.ev_scat_all, 0));
             launch_acc_i32(Q.npj, Q.pre, R, nullptr, s);
