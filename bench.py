@@ -9,9 +9,10 @@ scan, chunk cut) + execute (numeric + sort per chunk, D2H overlapped) through th
   e2e    the same through the public API with HOST operands: the H2D of A (= B) from pinned
          memory and the D2H of C are inside the timed region.
 
-Multi-GPU (torchrun, one rank per GPU): rows of A are dealt as contiguous panels; B reaches
-every rank by NCCL broadcast in the e2e step; each rank's nnz is all-gathered for the global
-row_ptr base; every rank drains its own rows of C.  Total work is fixed -> scaling "strong".
+Multi-GPU (torchrun, one rank per GPU): rows of A are dealt as contiguous panels; in the e2e
+step every rank uploads 1/world of B over its own host link and an NCCL all-gather over NVLink
+assembles B on every GPU; each rank's nnz is all-gathered for the global row_ptr base; every rank
+drains its own rows of C.  Total work is fixed -> scaling "strong".
 
 --impl reference runs the CPU oracle (the reference arm of this tier) on bounded samples.
 """
@@ -283,11 +284,17 @@ def main():
         pass
 
     def to_dev(M):
+        # storage padded to a multiple of the world size: the e2e step refills these arrays with a
+        # scatter (each rank uploads 1/world) + all-gather over NVLink (dist.scatter_allgather_csr)
         d = Dev()
         d.nrows, d.ncols = M.nrows, M.ncols
-        d.row_ptr = torch.from_numpy(M.row_ptr).to(dev)
-        d.col = torch.from_numpy(M.col).to(dev)
-        d.val = torch.from_numpy(M.val).to(dev)
+        d.store = []
+        for name, x in (("row_ptr", M.row_ptr), ("col", M.col), ("val", M.val)):
+            t = torch.from_numpy(x)
+            buf = torch.zeros(pdist.padded_len(t.numel(), world), dtype=t.dtype, device=dev)
+            buf[:t.numel()].copy_(t)
+            d.store.append(buf)
+            setattr(d, name, buf[:t.numel()])
         return d
 
     dB = to_dev(B)
@@ -490,22 +497,21 @@ def main():
                     P.free()
                     return
             else:
-                # rank 0 stages B from pinned host memory; NCCL broadcast over NVLink to every rank
-                if rank == 0:
-                    dB.row_ptr.copy_(hB.row_ptr, non_blocking=True)
-                    dB.col.copy_(hB.col, non_blocking=True)
-                    dB.val.copy_(hB.val, non_blocking=True)
+                # B from pinned host memory: every rank uploads 1/world of each array over its own
+                # host link, an all-gather over NVLink (NCCL) assembles B on every GPU
+                hb = [hB.row_ptr, hB.col, hB.val]
                 if cdev is not None:
-                    pdist.broadcast_csr([dB.row_ptr, dB.col, dB.val], src=0)
-                else:  # gloo control-flow test: stage through host tensors
-                    hb = [x.cpu() for x in (dB.row_ptr, dB.col, dB.val)]
-                    pdist.broadcast_csr(hb, src=0)
-                    for x, y in zip((dB.row_ptr, dB.col, dB.val), hb):
+                    pdist.scatter_allgather_csr(hb, dB.store)
+                else:  # gloo control-flow test (several ranks on one GPU): stage through host tensors
+                    st = [x.cpu() for x in dB.store]
+                    pdist.scatter_allgather_csr(hb, st)
+                    for x, y in zip(dB.store, st):
                         x.copy_(y)
-                if not same:
-                    dA.row_ptr.copy_(hA.row_ptr, non_blocking=True)
-                    dA.col.copy_(hA.col, non_blocking=True)
-                    dA.val.copy_(hA.val, non_blocking=True)
+                if not same:  # A: only this rank's row panel goes up
+                    p0, p1 = int(A.row_ptr[r0]), int(A.row_ptr[r1])
+                    dA.row_ptr[r0:r1 + 1].copy_(hA.row_ptr[r0:r1 + 1], non_blocking=True)
+                    dA.col[p0:p1].copy_(hA.col[p0:p1], non_blocking=True)
+                    dA.val[p0:p1].copy_(hA.val[p0:p1], non_blocking=True)
                 P = capi.Plan(dA, dB, wbytes, mk_opts())
                 if fused:
                     z = P.execute_capacity(h_rp, h_col, h_val, nnz_local)
@@ -534,7 +540,7 @@ def main():
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
         e2e = {"value": 2.0 * products_total * args.steps / (ems / 1e3) / 1e9, "unit": "GFLOP/s",
-               "h2d_bytes_per_step": int(h2d if rank == 0 else 0) if world > 1 else int(h2d),
+               "h2d_bytes_per_step": int(h2d),  # over all ranks (each rank uploads 1/world of B)
                "d2h_bytes_per_step": int(12 * nnz_total + 8 * (A.nrows + 1)), "ms_per_step": ems / args.steps}
 
     cpu = None

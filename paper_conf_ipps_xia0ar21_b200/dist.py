@@ -3,8 +3,10 @@
 Rows of C are independent (§III-A: "final values within a chunk of the output
 matrix C are independent"), so A is dealt across ranks as contiguous row panels (§III-A,
 §III-D) and every rank needs all of B.  The only exchanges on the path are
-  * B (and A when A is B) reaching every GPU: a broadcast from the rank that staged it
-    (`broadcast_csr`, NCCL over NVLink/NVSwitch on a B200 box, gloo in the CPU tests);
+  * B (and A when A is B) reaching every GPU from host memory: every rank uploads 1/world of each
+    CSR array over its OWN host link and an all-gather over NVLink/NVSwitch assembles the whole
+    on every GPU (`scatter_allgather_csr`; H2D time / world instead of one rank uploading all of
+    it and broadcasting, `broadcast_csr`; NCCL on a B200 box, gloo in the CPU tests);
   * the 8-byte nnz of every rank's slice (`slice_bases`, an all_gather) so that each rank writes
     its C rows with GLOBAL row_ptr values into its part of one logical host CSR.
 After that every rank drains its own C chunks over its own host link; nothing else crosses GPUs.
@@ -54,6 +56,31 @@ def broadcast_csr(arrays: Sequence, src: int = 0, group=None) -> None:
     import torch.distributed as dist
     for a in arrays:
         dist.broadcast(a, src=src, group=group)
+
+
+def padded_len(n: int, world: int) -> int:
+    """Length of a device array that `scatter_allgather_csr` can fill: n rounded up to a multiple
+    of the world size (the all-gather moves equal chunks)."""
+    return ((int(n) + world - 1) // world) * world
+
+
+def scatter_allgather_csr(host_arrays: Sequence, dev_arrays: Sequence, group=None) -> None:
+    """Every rank copies its 1/world chunk of each host array (pinned, true length n) into the same
+    place of the matching device array (length padded_len(n, world)) over its own host link, then
+    an in-place all-gather (NCCL over NVLink on GPUs) gives every rank the whole array in
+    dev_array[:n]."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    for h, d in zip(host_arrays, dev_arrays):
+        n = int(h.numel())
+        chunk = int(d.numel()) // world
+        assert chunk * world == int(d.numel()) and chunk * world >= n
+        lo, hi = min(rank * chunk, n), min((rank + 1) * chunk, n)
+        mine = d[rank * chunk:(rank + 1) * chunk]
+        if hi > lo:
+            mine[:hi - lo].copy_(h[lo:hi], non_blocking=True)
+        dist.all_gather_into_tensor(d, mine, group=group)
 
 
 def gather_rows_global(parts: Sequence[Tuple[np.ndarray, np.ndarray, np.ndarray]]):

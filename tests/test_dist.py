@@ -85,3 +85,37 @@ def test_gloo_world2_slices_stitch_to_whole():
     assert res[0][6] == res[1][6] == whole["row_ptr"][-1]
     assert np.array_equal(rp, whole["row_ptr"]) and np.array_equal(col, whole["col"])
     assert np.array_equal(val, whole["val"])
+
+
+def _worker_allgather(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        A = W.rmat(9, 8, seed=6)
+        host = [torch.from_numpy(A.row_ptr), torch.from_numpy(A.col), torch.from_numpy(A.val)]
+        dev = [torch.full((pdist.padded_len(h.numel(), world),), -7, dtype=h.dtype) for h in host]
+        pdist.scatter_allgather_csr(host, dev)
+        ok = all(torch.equal(d[:h.numel()], h) for h, d in zip(host, dev))
+        q.put((rank, ok))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_gloo_scatter_allgather_b(world):
+    """B reaches every rank with each rank uploading 1/world of every array, then an all-gather
+    (the multi-GPU e2e upload; uneven lengths are padded to a multiple of the world size)."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_allgather, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(ok for _, ok in res), res
