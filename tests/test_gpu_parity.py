@@ -483,3 +483,21 @@ def test_chunk_order_by_flops():
         with pytest.raises(capi.SpgemmError) as e:
             P.execute_stream(lambda *a: 0)
         assert e.value.status == capi.ERR_INVALID_ARGUMENT
+
+
+def test_matmul_scipy_inputs():
+    """The Python convenience wrapper with scipy.sparse operands (unsorted indices are sorted)."""
+    sp = pytest.importorskip("scipy.sparse")
+    rng = np.random.default_rng(4)
+    A = sp.random(300, 200, density=0.05, random_state=1, format="csr") + sp.identity(300, format="csr")[:, :200]
+    B = sp.random(200, 500, density=0.04, random_state=2, format="csr")
+    A = A.tocsr()
+    A.indices = A.indices.copy()
+    C = spg.matmul(A, B)
+    Aw = spg.as_csr(A)
+    Bw = spg.as_csr(B)
+    Ao = W.CSR(Aw.nrows, Aw.ncols, Aw.row_ptr, Aw.col, Aw.val)
+    Bo = W.CSR(Bw.nrows, Bw.ncols, Bw.row_ptr, Bw.col, Bw.val)
+    assert_parity(Ao, Bo, C.row_ptr.numpy(), C.col.numpy(), C.val.numpy())
+    C2 = spg.matmul(Ao, Bo, col_panels=2)
+    assert np.array_equal(C2.col.numpy(), C.col.numpy())
