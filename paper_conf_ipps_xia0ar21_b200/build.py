@@ -12,7 +12,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-SOURCES = [os.path.join(CSRC, f) for f in ("api.cu", "kernels.cu")]
+SOURCES = [os.path.join(CSRC, f) for f in ("api.cu", "panels.cu", "kernels.cu")]
 HEADERS = [os.path.join(CSRC, "internal.h"), os.path.join(ROOT, "include", "spgemm.h")]
 LIB = os.path.join(HERE, "libspgemm_b200.so")
 
