@@ -280,3 +280,30 @@ def test_sampled_rows_full_c2():
     assert np.array_equal(np.diff(S["row_ptr"]), CF.c2_row_nnz(128, rows))
     i = np.repeat(rows, np.diff(S["row_ptr"]))
     assert np.array_equal(S["val"], CF.c2_entry(128, i, S["col"].astype(np.int64)))
+
+
+hyp = pytest.importorskip("hypothesis")
+from hypothesis import HealthCheck, given, settings  # noqa: E402
+from hypothesis import strategies as st  # noqa: E402
+
+
+@settings(max_examples=150, deadline=None, derandomize=True, suppress_health_check=[HealthCheck.too_slow])
+@given(seed=st.integers(0, 2**31 - 1), m=st.integers(0, 24), k=st.integers(0, 24), n=st.integers(0, 24),
+       da=st.floats(0.0, 1.0), db=st.floats(0.0, 1.0))
+def test_dense_brute_force_property(seed, m, k, n, da, db):
+    """Hypothesis-driven brute force over tiny shapes and densities (incl. empty and full rows, and
+    explicit zeros): structure = boolean product, values = exact dense product of small integers,
+    products per row = A's pattern times B's row counts."""
+    rng = np.random.default_rng(seed)
+    A = W.random_csr(m, k, da, seed=seed % 1000, values="ones")
+    B = W.random_csr(k, n, db, seed=seed % 1000 + 1, values="ones")
+    A.val = rng.integers(-3, 4, size=A.nnz).astype(np.float64)
+    B.val = rng.integers(-3, 4, size=B.nnz).astype(np.float64)
+    C = oracle.spgemm(A, B)
+    pa, pb = _dense_pattern(A), _dense_pattern(B)
+    pat = (pa @ pb) > 0
+    assert C["row_ptr"][-1] == pat.sum()
+    for i in range(m):
+        assert list(C["col"][C["row_ptr"][i]:C["row_ptr"][i + 1]]) == list(np.nonzero(pat[i])[0])
+    assert np.array_equal(_as_dense(C, (m, n)), A.dense() @ B.dense())
+    assert np.array_equal(oracle.products(A, B), pa @ pb.sum(axis=1) if m else np.zeros(0, np.int64))
