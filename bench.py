@@ -480,6 +480,11 @@ def main():
                 if tr:
                     roof["traffic"] = tr["bytes_per_launch"]
                     roof["traffic_source"] = tr.get("source")
+                    if "lsu_pipe_frac_of_peak" in tr:  # the unit that actually binds the hash kernels
+                        roof["binding_unit"] = {"unit": "LSU data pipe (shared memory + L1)",
+                                                "frac_of_peak": tr["lsu_pipe_frac_of_peak"],
+                                                "sm_throughput_frac": tr.get("sm_throughput_frac"),
+                                                "source": tr.get("source")}
             except Exception:  # noqa: BLE001
                 pass
 
