@@ -303,15 +303,33 @@ __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR
         }
         if (threadIdx.x == 0) sm.off[nb] = tot;
         __syncthreads();
-        for (int64_t q = threadIdx.x; q < tot; q += NT) {
+        // Each warp takes 32 consecutive products per step (coalesced B loads).  Two lanes find
+        // the segments of the warp's first and last product; every lane then searches only that
+        // window (usually 1-3 segments) instead of all nb A entries of the batch.
+        const int lane = threadIdx.x & 31;
+        for (int64_t qb = threadIdx.x - lane; qb < tot; qb += NT) {  // warp-uniform trip count
+            const int64_t q = qb + lane;
             int lo = 0, hi = nb;  // invariant: off[lo] <= q < off[hi]
-            while (hi - lo > 1) {
-                const int mid = (lo + hi) >> 1;
-                if (sm.off[mid] <= q) lo = mid;
-                else hi = mid;
+            if (lane < 2) {
+                const int64_t qq = lane ? min(qb + 31, tot - 1) : qb;
+                while (hi - lo > 1) {
+                    const int mid = (lo + hi) >> 1;
+                    if (sm.off[mid] <= qq) lo = mid;
+                    else hi = mid;
+                }
             }
-            const int64_t pos = sm.bs[lo] + (q - sm.off[lo]);
-            f(__ldg(&B.col[pos]), VALS ? sm.a[lo] * __ldg(&B.val[pos]) : 0.0);
+            const int wlo = __shfl_sync(FULLMASK, lo, 0), whi = __shfl_sync(FULLMASK, lo, 1) + 1;
+            if (q < tot) {
+                lo = wlo;
+                hi = whi;
+                while (hi - lo > 1) {
+                    const int mid = (lo + hi) >> 1;
+                    if (sm.off[mid] <= q) lo = mid;
+                    else hi = mid;
+                }
+                const int64_t pos = sm.bs[lo] + (q - sm.off[lo]);
+                f(__ldg(&B.col[pos]), VALS ? sm.a[lo] * __ldg(&B.val[pos]) : 0.0);
+            }
         }
         __syncthreads();
     }
