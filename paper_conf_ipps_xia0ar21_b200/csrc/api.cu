@@ -125,11 +125,16 @@ namespace {
 // ramp up (1/4, 3/8, 1/2, 3/4 of capp, then capp) so that the first D2H starts
 // early and each later chunk is computed while the previous one is being copied.
 void cut_chunks(spgemm_plan_s *P, const int64_t *pre, int64_t total, int64_t capp, int64_t limit,
-                std::vector<int64_t> *offs_out) {
+                std::vector<int64_t> *offs_out, std::vector<int64_t> *maxb_out = nullptr,
+                std::vector<int64_t> *maxcol_out = nullptr) {
+    // maxb_out / maxcol_out: per chunk, the largest row bound and the largest column its rows
+    // read -- reduced on the device over the fine ids and returned in the same round trip
     const int64_t R = P->R;
     cudaStream_t s = P->stream;
     P->chunk_rows.clear();
     if (offs_out) offs_out->clear();
+    if (maxb_out) maxb_out->clear();
+    if (maxcol_out) maxcol_out->clear();
     if (total <= 0) return;
     constexpr int F = 8;
     const bool ramp = capp >= F && total / capp >= 4;
@@ -138,12 +143,18 @@ void cut_chunks(spgemm_plan_s *P, const int64_t *pre, int64_t total, int64_t cap
     const size_t save = P->used;  // temporary arrays at the start of the (not yet used) ring region
     int64_t *bounds = P->alloc<int64_t>(nids + 1, "chunk bounds");
     int64_t *offs = P->alloc<int64_t>(nids + 1, "chunk offsets");
+    int64_t *fmax = maxb_out ? P->alloc<int64_t>(nids, "fine max bound") : nullptr;
+    int64_t *fcol = maxcol_out ? P->alloc<int64_t>(nids, "fine max column") : nullptr;
     launch_cut(pre, R, capp, bounds, nids, s);
     launch_gather(pre, bounds, nids + 1, offs, s);
+    if (fmax) launch_seg_max(P->bnd, bounds, nids, fmax, s);
+    if (fcol) launch_seg_max_col(P->A, bounds, nids, fcol, s);
     CKL("cut");
-    std::vector<int64_t> hb(nids + 1), ho(nids + 1);
+    std::vector<int64_t> hb(nids + 1), ho(nids + 1), hm(fmax ? nids : 0), hc(fcol ? nids : 0);
     CK(cudaMemcpyAsync(hb.data(), bounds, sizeof(int64_t) * (nids + 1), cudaMemcpyDeviceToHost, s));
     CK(cudaMemcpyAsync(ho.data(), offs, sizeof(int64_t) * (nids + 1), cudaMemcpyDeviceToHost, s));
+    if (fmax) CK(cudaMemcpyAsync(hm.data(), fmax, sizeof(int64_t) * nids, cudaMemcpyDeviceToHost, s));
+    if (fcol) CK(cudaMemcpyAsync(hc.data(), fcol, sizeof(int64_t) * nids, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     P->used = save;
     P->chunk_rows.push_back(hb[0]);
@@ -159,11 +170,20 @@ void cut_chunks(spgemm_plan_s *P, const int64_t *pre, int64_t total, int64_t cap
             ends.push_back(std::min(id, nids));
         }
     }
+    int64_t id0 = 0, mb = 0, mc = -1;  // fine ids not yet in an emitted chunk, and their maxima
     for (int64_t c : ends) {
+        for (; id0 < c; ++id0) {
+            if (fmax) mb = std::max(mb, hm[id0]);
+            if (fcol) mc = std::max(mc, hc[id0]);
+        }
         if (hb[c] == P->chunk_rows.back()) continue;
         if (ho[c] - last_off > limit) fail(SPGEMM_ERR_STATE, "internal: chunk exceeds the ring capacity");
         P->chunk_rows.push_back(hb[c]);
         if (offs_out) offs_out->push_back(ho[c]);
+        if (maxb_out) maxb_out->push_back(mb);
+        if (maxcol_out) maxcol_out->push_back(mc);
+        mb = 0;
+        mc = -1;
         last_off = ho[c];
     }
     if (P->chunk_rows.front() != 0 || P->chunk_rows.back() != R)
@@ -459,6 +479,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         return cap;
     };
 
+    std::vector<int64_t> chunk_maxcol;  // host operands: largest column each chunk reads
     if (!P->fused) {
         // S3+S4 symbolic and S5 scan over all rows, then cut by exact nnz
         SymArgs sa = sym_args(P, 0, R, sym_tiers(P->max_bound));
@@ -517,22 +538,13 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         if (minc <= 0) minc = std::min<int64_t>(64, std::max<int64_t>(1, total_b * 12 / (512ll << 20)));
         if (minc > 1) capp = std::min<int64_t>(capp, std::max<int64_t>(1, (total_b + minc - 1) / minc));
         if (opts.chunk_nnz > 0) capp = std::min<int64_t>(capp, std::max<int64_t>(1, opts.chunk_nnz - P->max_bound));
-        cut_chunks(P, P->crp, total_b, std::max<int64_t>(capp, 1), cap, nullptr);
+        // with the cut: per chunk the max row bound (which symbolic tiers a chunk needs) and, for
+        // host operands, the largest column it reads (which value pieces its numeric pass waits for)
+        // -- one round trip, no H2D (a small H2D would queue behind the value pieces on the copy engine)
+        cut_chunks(P, P->crp, total_b, std::max<int64_t>(capp, 1), cap, nullptr, &P->chunk_maxb,
+                   P->ev_piece.empty() ? nullptr : &chunk_maxcol);
         CK(cudaMemsetAsync(P->crp, 0, sizeof(int64_t), s));
         const int64_t nch = P->num_chunks();
-        // per-chunk max row bound: decides which symbolic tiers a chunk needs
-        P->chunk_maxb.assign(nch, 0);
-        if (nch > 0) {
-            const size_t save = P->used;
-            int64_t *drows = P->alloc<int64_t>(nch + 1, "chunk rows");
-            int64_t *dmax = P->alloc<int64_t>(nch, "chunk max bound");
-            CK(cudaMemcpyAsync(drows, P->chunk_rows.data(), sizeof(int64_t) * (nch + 1), cudaMemcpyHostToDevice, s));
-            launch_seg_max(P->bnd, drows, nch, dmax, s);
-            CKL("chunk max");
-            CK(cudaMemcpyAsync(P->chunk_maxb.data(), dmax, sizeof(int64_t) * nch, cudaMemcpyDeviceToHost, s));
-            CK(cudaStreamSynchronize(s));
-            P->used = save;
-        }
         P->ev_tot = rs->events(Res::PLAIN, ev_base, nch);
         // the symbolic passes get their own stream so that chunk j+1's symbolic pass overlaps
         // chunk j's numeric pass (the two passes have separate lists and arena scratch)
@@ -545,16 +557,19 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         const int64_t nch = P->num_chunks();
         P->chunk_wait.assign(nch, -1);
         if (!P->ev_piece.empty() && nch > 0) {
-            const size_t save = P->used;
-            int64_t *drows = P->alloc<int64_t>(nch + 1, "chunk rows");
-            int64_t *dmax = P->alloc<int64_t>(nch, "chunk max column");
-            std::vector<int64_t> hmax(nch);
-            CK(cudaMemcpyAsync(drows, P->chunk_rows.data(), sizeof(int64_t) * (nch + 1), cudaMemcpyHostToDevice, s));
-            launch_seg_max_col(P->A, drows, nch, dmax, s);
-            CKL("chunk max column");
-            CK(cudaMemcpyAsync(hmax.data(), dmax, sizeof(int64_t) * nch, cudaMemcpyDeviceToHost, s));
-            CK(cudaStreamSynchronize(s));
-            P->used = save;
+            std::vector<int64_t> &hmax = chunk_maxcol;
+            if ((int64_t)hmax.size() != nch) {  // two-phase plans: one more round trip
+                hmax.resize(nch);
+                const size_t save = P->used;
+                int64_t *drows = P->alloc<int64_t>(nch + 1, "chunk rows");
+                int64_t *dmax = P->alloc<int64_t>(nch, "chunk max column");
+                CK(cudaMemcpyAsync(drows, P->chunk_rows.data(), sizeof(int64_t) * (nch + 1), cudaMemcpyHostToDevice, s));
+                launch_seg_max_col(P->A, drows, nch, dmax, s);
+                CKL("chunk max column");
+                CK(cudaMemcpyAsync(hmax.data(), dmax, sizeof(int64_t) * nch, cudaMemcpyDeviceToHost, s));
+                CK(cudaStreamSynchronize(s));
+                P->used = save;
+            }
             for (int64_t j = 0; j < nch; ++j) {
                 int64_t need = hmax[j];
                 if (P->a_alias) need = std::max<int64_t>(need, rb + P->chunk_rows[j + 1] - 1);
