@@ -17,6 +17,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <thread>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -295,6 +296,43 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
                             Ah->col_idx == Bh->col_idx && Ah->values == Bh->values && Ah->nrows == Bh->nrows &&
                             Ah->ncols == Bh->ncols;
     const bool pieced_count = host_alias && !opts.validate && Bh->nnz > 0;
+    // Host cut: with short rows the plan needs no count pass at all.  Every row bound
+    // min(products, ncols) is at most ub = min(ncols, maxlen^2) (maxlen = longest row of B = A),
+    // so when ub <= CAPB_NUM (no long-row scratch) chunks are cut on the host from A.row_ptr by
+    // nnz(A) x maxlen, and each chunk's count pass runs in execute, right before its symbolic pass,
+    // once the pieces it reads have landed -- the first chunk starts ~1 ms into the upload instead
+    // of after the whole structure.  SPGEMM_NO_HOST_CUT=1 disables it (ablation).
+    int64_t hc_maxlen = -1;
+    if (pieced_count && P->fused) {
+        const char *no = getenv("SPGEMM_NO_HOST_CUT");
+        if (!(no && no[0] == '1')) {
+            const int64_t lim = Bh->ncols <= CAPB_NUM ? INT64_MAX : 64;  // maxlen^2 <= CAPB_NUM
+            // longest row: one pass over row_ptr, split over host threads (C2: 2 M rows, ~1.7 ms
+            // on one core, on the critical path of the step), each stopping once past `lim`
+            const int64_t *brp = Bh->row_ptr;
+            const int64_t n = Bh->nrows;
+            const int nt = n < (1 << 18) ? 1 : int(std::min<unsigned>(8, std::max(1u, std::thread::hardware_concurrency())));
+            std::vector<int64_t> part(nt, 0);
+            auto scan = [&](int t) {
+                const int64_t a = n * t / nt, b = n * (t + 1) / nt;
+                int64_t ml = 0;
+                for (int64_t r = a; r < b && ml <= lim; r += 4096) {
+                    const int64_t e = std::min<int64_t>(r + 4096, b);
+                    int64_t m = 0;
+                    for (int64_t q = r; q < e; ++q) m = std::max<int64_t>(m, brp[q + 1] - brp[q]);
+                    ml = std::max(ml, m);
+                }
+                part[t] = ml;
+            };
+            std::vector<std::thread> th;
+            for (int t = 1; t < nt; ++t) th.emplace_back(scan, t);
+            scan(0);
+            for (auto &x : th) x.join();
+            const int64_t ml = *std::max_element(part.begin(), part.end());
+            if (ml <= lim && std::min<int64_t>(Bh->ncols, ml * ml) <= CAPB_NUM) hc_maxlen = ml;
+        }
+    }
+    P->host_cut = hc_maxlen >= 0;
     std::vector<cudaEvent_t> ev_col;
     if (Bh->where == SPGEMM_DEVICE) {
         P->B = DevCSR{Bh->row_ptr, Bh->col_idx, Bh->values, Bh->nrows, Bh->ncols};
@@ -302,15 +340,19 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         int64_t *rp = P->alloc<int64_t>(Bh->nrows + 1, "B.row_ptr");
         int32_t *c = P->alloc<int32_t>(Bh->nnz, "B.col_idx");
         double *v = P->alloc<double>(Bh->nnz, "B.values");
-        CK(cudaMemcpyAsync(rp, Bh->row_ptr, sizeof(int64_t) * (Bh->nrows + 1), cudaMemcpyHostToDevice, s));
+        if (!P->host_cut)
+            CK(cudaMemcpyAsync(rp, Bh->row_ptr, sizeof(int64_t) * (Bh->nrows + 1), cudaMemcpyHostToDevice, s));
         if (Bh->nnz && !pieced_count)
             CK(cudaMemcpyAsync(c, Bh->col_idx, sizeof(int32_t) * Bh->nnz, cudaMemcpyHostToDevice, s));
-        // pieces of ~32 MB of values, cut at row boundaries
-        const int64_t target = std::max<int64_t>(1, (32ll << 20) / 8);
+        // pieces of ~32 MB of values, cut at row boundaries; the first ones smaller (1/8, 1/4,
+        // 1/2) so that the first chunk's rows land early
+        int64_t target = std::max<int64_t>(1, (32ll << 20) / 8);
+        if (const char *pn = getenv("SPGEMM_PIECE_NNZ")) target = std::max<int64_t>(1, atoll(pn));  // test hook
         P->bpiece_rows.push_back(0);
         int64_t r = 0;
         while (r < Bh->nrows) {
-            const int64_t want = Bh->row_ptr[r] + target;
+            const size_t k = bval_pieces.size();
+            const int64_t want = Bh->row_ptr[r] + (k < 3 ? std::max<int64_t>(1, target >> (3 - k)) : target);
             int64_t e = std::upper_bound(Bh->row_ptr + r + 1, Bh->row_ptr + Bh->nrows + 1, want) - Bh->row_ptr - 1;
             e = std::max<int64_t>(e, r + 1);
             bval_pieces.push_back({size_t(Bh->row_ptr[r]), size_t(Bh->row_ptr[e] - Bh->row_ptr[r])});
@@ -319,7 +361,35 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         }
         bval_dev = v;
         P->B = DevCSR{rp, c, v, Bh->nrows, Bh->ncols};
-        if (pieced_count) {
+        if (P->host_cut) {
+            // piece k = row_ptr (b_k, b_k+1] (+ entry 0 with the first) , col_idx, values of its
+            // rows, in that order on the H2D stream; ev_col[k] / ev_piece[k] after its structure /
+            // values.  A chunk waits for the piece holding the largest row it reads (its own last
+            // row, or the largest column of its rows), which covers every earlier piece.
+            const size_t np = bval_pieces.size();
+            P->hstream = rs->stream(rs->hstream);
+            P->ev_col = rs->events(Res::PIECE, np, np);
+            P->ev_piece = rs->events(Res::PIECE, 0, np);
+            cudaEvent_t alloc_ready = rs->events(Res::PIECE, 2 * np, 1)[0];
+            CK(cudaEventRecord(alloc_ready, s));  // allocation order: after everything queued so far
+            CK(cudaStreamWaitEvent(P->hstream, alloc_ready, 0));
+            for (size_t k = 0; k < np; ++k) {
+                const int64_t b0 = P->bpiece_rows[k], b1 = P->bpiece_rows[k + 1];
+                const int64_t q0 = k == 0 ? 0 : b0 + 1;
+                CK(cudaMemcpyAsync(rp + q0, Bh->row_ptr + q0, sizeof(int64_t) * (b1 + 1 - q0), cudaMemcpyHostToDevice,
+                                   P->hstream));
+                const auto &pc = bval_pieces[k];
+                if (pc.second)
+                    CK(cudaMemcpyAsync(c + pc.first, Bh->col_idx + pc.first, sizeof(int32_t) * pc.second,
+                                       cudaMemcpyHostToDevice, P->hstream));
+                CK(cudaEventRecord(P->ev_col[k], P->hstream));
+                if (pc.second)
+                    CK(cudaMemcpyAsync(v + pc.first, Bh->values + pc.first, sizeof(double) * pc.second,
+                                       cudaMemcpyHostToDevice, P->hstream));
+                CK(cudaEventRecord(P->ev_piece[k], P->hstream));
+            }
+            bval_pieces.clear();  // queued
+        } else if (pieced_count) {
             const size_t np = bval_pieces.size();
             P->hstream = rs->stream(rs->hstream);
             ev_col = rs->events(Res::PIECE, np, np);
@@ -347,6 +417,10 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         if (alias) {
             P->A = DevCSR{P->B.rp + rb, P->B.col, P->B.val, P->R, Ah->ncols};
             P->a_alias = true;
+            if (P->host_cut) {
+                P->hA_rp = Ah->row_ptr + rb;
+                P->hA_col = Ah->col_idx;
+            }
         } else {
             int64_t *rp = P->alloc<int64_t>(P->R + 1, "A.row_ptr");
             int32_t *c = P->alloc<int32_t>(p1 - p0, "A.col_idx");
@@ -397,9 +471,14 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         CKL("validate");
     }
 
-    // S2 count
+    // S2 count (host cut: per chunk, inside execute)
     pe.rec(1, s);
-    if (pieced_count) {
+    if (P->host_cut) {
+        P->products = -1;  // known after the first execution
+        P->max_u = -1;
+        P->max_bound = std::min<int64_t>(P->ncols, hc_maxlen * hc_maxlen);  // an upper bound
+        P->max_deg = hc_maxlen;
+    } else if (pieced_count) {
         for (size_t k = 0; k + 1 < P->bpiece_rows.size(); ++k) {
             const int64_t g0 = std::max<int64_t>(P->bpiece_rows[k], rb), g1 = std::min<int64_t>(P->bpiece_rows[k + 1], re);
             CK(cudaStreamWaitEvent(s, ev_col[k], 0));
@@ -417,20 +496,22 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     // fused plans: the prefix of the row bounds (chunk boundaries) is scanned before the first
     // host round trip, which then reads both the count totals and the prefix total
     int64_t total_b = 0;
-    if (P->fused) {
+    if (P->fused && !P->host_cut) {
         launch_scan64(P->bnd, P->R, P->crp, P->tmp, s);
         CKL("bound scan");
         CK(cudaMemcpyAsync(&total_b, P->crp + P->R, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     }
     Ctl hc;
-    CK(cudaMemcpyAsync(&hc, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    if (hc.err & 2u)
-        fail(SPGEMM_ERR_INVALID_ARGUMENT, "input validation failed (unsorted/duplicate/out-of-range col_idx or bad row_ptr)");
-    P->products = (int64_t)hc.sum_u;
-    P->max_u = (int64_t)hc.max_u;
-    P->max_bound = (int64_t)hc.max_bound;
-    P->max_deg = (int64_t)hc.max_deg;
+    if (!P->host_cut) {
+        CK(cudaMemcpyAsync(&hc, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (hc.err & 2u)
+            fail(SPGEMM_ERR_INVALID_ARGUMENT, "input validation failed (unsorted/duplicate/out-of-range col_idx or bad row_ptr)");
+        P->products = (int64_t)hc.sum_u;
+        P->max_u = (int64_t)hc.max_u;
+        P->max_bound = (int64_t)hc.max_bound;
+        P->max_deg = (int64_t)hc.max_deg;
+    }
 
     // arena-resident accumulator scratch, sized only if a row can exceed one CTA-tier piece:
     //   cursors of the pieced CTA tier (per CTA: 2 x curstride int32 for each pass -- separate,
@@ -526,6 +607,41 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
             std::stable_sort(P->unit_order.begin(), P->unit_order.end(),
                              [&](int64_t a, int64_t b) { return fl[a] > fl[b]; });
         }
+    } else if (P->host_cut) {
+        // host cut: a chunk of rows [r0, r1) has sum of row bounds <= (A.row_ptr[r1] - A.row_ptr[r0]) x
+        // maxlen, so chunks are cut by nnz(A) with that product <= capp (one row alone if longer); the
+        // products are estimated as nnz(A) x mean row length of B for the chunk count only
+        const int64_t ml = std::max<int64_t>(hc_maxlen, 1);
+        const int64_t *hrp = P->hA_rp;
+        const int64_t nnzA = hrp[R] - hrp[0];
+        const int64_t est = Bh->nrows ? int64_t(double(nnzA) * (double(Bh->nnz) / double(Bh->nrows))) : 0;
+        P->sum_bound = -1;
+        int64_t cap = ring_cap(P->max_bound);
+        cap = std::max<int64_t>(std::min<int64_t>(cap, std::max<int64_t>(nnzA * ml, 1)), std::max<int64_t>(P->max_bound, 1));
+        P->cap = cap;
+        int64_t capp = std::max<int64_t>(1, cap - P->max_bound);
+        int64_t minc = opts.min_chunks;
+        if (minc <= 0) minc = std::min<int64_t>(64, std::max<int64_t>(1, est * 12 / (512ll << 20)));
+        if (minc > 1) capp = std::min<int64_t>(capp, std::max<int64_t>(1, (est + minc - 1) / minc));
+        if (opts.chunk_nnz > 0) capp = std::min<int64_t>(capp, std::max<int64_t>(1, opts.chunk_nnz - P->max_bound));
+        // ramp as in cut_chunks: 2/8, 3/8, 4/8, 6/8 of capp, then capp
+        const bool ramp = capp >= 8 && est / capp >= 4;
+        P->chunk_rows.assign(1, 0);
+        int64_t r = 0;
+        for (int k = 0; r < R; ++k) {
+            static const int units[] = {2, 3, 4, 6};
+            const int64_t sz = ramp && k < 4 ? std::max<int64_t>(1, capp / 8 * units[k]) : capp;
+            const int64_t want = hrp[r] + std::max<int64_t>(sz / ml, 1);
+            int64_t e = std::upper_bound(hrp + r + 1, hrp + R + 1, want) - hrp - 1;
+            e = std::max<int64_t>(e, r + 1);
+            P->chunk_rows.push_back(e);
+            r = e;
+        }
+        if (nnzA == 0) P->chunk_rows.clear();  // every row is empty: no chunk (as cut_chunks)
+        P->chunk_maxb.assign(P->num_chunks(), P->max_bound);
+        const int64_t nch = P->num_chunks();
+        P->ev_tot = rs->events(Res::PLAIN, ev_base, nch);
+        P->astream = rs->stream(rs->astream);
     } else {
         // fused: boundaries from the prefix of the row bounds; the symbolic pass runs per chunk
         // inside execute.  crp temporarily holds that prefix.
@@ -555,8 +671,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     // with A aliasing B also the chunk's own rows)
     {
         const int64_t nch = P->num_chunks();
-        P->chunk_wait.assign(nch, -1);
-        if (!P->ev_piece.empty() && nch > 0) {
+        P->chunk_wait.assign(nch, -1);  // host cut: set per chunk in execute (enqueue_analysis)
+        if (!P->ev_piece.empty() && nch > 0 && !P->host_cut) {
             std::vector<int64_t> &hmax = chunk_maxcol;
             if ((int64_t)hmax.size() != nch) {  // two-phase plans: one more round trip
                 hmax.resize(nch);
@@ -640,6 +756,24 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t slot_off, int64
 void enqueue_analysis(spgemm_plan_s *P, int64_t j, cudaEvent_t *ev) {
     const int64_t r0 = P->chunk_rows[j], r1 = P->chunk_rows[j + 1];
     cudaStream_t as = P->astream;
+    if (P->host_cut) {
+        // the piece holding the largest row chunk j reads: its own last row or the largest column
+        // of its rows (each row's last entry, rows sorted); the count and symbolic passes wait for
+        // its structure, the numeric pass (chunk_wait) for its values
+        int64_t need = P->row_begin + r1 - 1;
+        const int64_t *hrp = P->hA_rp;
+        for (int64_t r = r0; r < r1; ++r)
+            if (hrp[r + 1] > hrp[r]) need = std::max<int64_t>(need, P->hA_col[hrp[r + 1] - 1]);
+        const auto it = std::upper_bound(P->bpiece_rows.begin(), P->bpiece_rows.end(), need);
+        const int w = int(it - P->bpiece_rows.begin()) - 1;
+        P->chunk_wait[j] = w;
+        CK(cudaStreamWaitEvent(as, P->ev_col[w], 0));
+        DevCSR Ak = P->A;
+        Ak.rp = P->A.rp + r0;
+        Ak.nrows = r1 - r0;
+        launch_count(Ak, P->B, P->bnd + r0, P->ctl, as);
+        CKL("count");
+    }
     SymArgs sa = sym_args(P, r0, r1, sym_tiers(P->chunk_maxb[j]));
     launch_symbolic(sa, P->num_sms, as, ev);
     CKL("symbolic");
@@ -735,7 +869,12 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         // the analysis stream starts after everything already queued on the compute stream
         CK(cudaEventRecord(P->ev_ready, s));
         CK(cudaStreamWaitEvent(P->astream, P->ev_ready, 0));
-        CK(cudaMemcpyAsync(P->crp, P->h_small, sizeof(int64_t), cudaMemcpyHostToDevice, P->astream));
+        // crp[0] = base without an H2D (a small copy would queue behind the operand pieces)
+        CK(cudaMemsetAsync(P->crp, 0, sizeof(int64_t), P->astream));
+        launch_add(P->crp, 0, base, P->astream);
+        CKL("row_ptr base");
+        if (P->host_cut)  // the count passes of this execution accumulate sum_u / max_u / max_bound
+            CK(cudaMemsetAsync(&P->ctl[0].sum_u, 0, 3 * sizeof(unsigned long long), P->astream));
         P->base_applied = base;
     } else {
         if (P->base_wanted != P->base_applied) {
@@ -885,6 +1024,15 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         cur.nnz += n;
         cur.u1 = j + 1;
         cur.r1 = r1;
+        if (one_per_unit || (cur.nnz >= target && cur.nnz > 0)) {
+            // the group reached its target: its copy goes now, not one analysis pass later when
+            // the next unit's total is known (the first group is one unit: the first copy starts
+            // right after the first numeric pass)
+            close_group(cur);
+            groups.push_back(cur);
+            target = std::min<int64_t>(P->cap, 2 * cur.nnz);
+            cur.b = -1;
+        }
         if (P->fused && j + 1 < nch) enqueue_analysis(P, j + 1, pe.at(size_t(j + 1) * per));
     }
     if (cur.b >= 0) {
@@ -911,6 +1059,10 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         P->rows_w = (int64_t)hc.rows_w;
         P->rows_b = (int64_t)hc.rows_b;
         P->rows_g = (int64_t)hc.rows_g;
+        if (P->host_cut) {
+            P->products = (int64_t)hc.sum_u;
+            P->max_u = (int64_t)hc.max_u;
+        }
     }
     if (P->profile) {  // per-kernel times are read from the events lazily (finalize_profile)
         P->pend.active = true;

@@ -139,6 +139,12 @@ struct spgemm_plan_s {
     std::vector<int64_t> bpiece_rows;       // B row boundaries of the pieces
     std::vector<int> chunk_wait;            // per chunk: last piece its numeric pass reads (-1: none)
     bool a_alias = false;
+    // host cut (fused C = A x A with host operands and short rows): chunks cut on the host from
+    // A.row_ptr; each chunk's count pass runs inside execute after the pieces it reads landed
+    bool host_cut = false;
+    std::vector<cudaEvent_t> ev_col;        // one per structure piece (row_ptr + col_idx), upload order
+    const int64_t *hA_rp = nullptr;         // borrowed host A (the plan's rows start at hA_rp[0])
+    const int32_t *hA_col = nullptr;
     Ctl *ctl = nullptr;  // [0] count / symbolic passes, [1] numeric passes
 
     uint32_t *gbits = nullptr, *gbits_sym = nullptr;

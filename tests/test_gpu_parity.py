@@ -501,3 +501,59 @@ def test_matmul_scipy_inputs():
     assert_parity(Ao, Bo, C.row_ptr.numpy(), C.col.numpy(), C.val.numpy())
     C2 = spg.matmul(Ao, Bo, col_panels=2)
     assert np.array_equal(C2.col.numpy(), C.col.numpy())
+
+
+@pytest.mark.parametrize("case", ["c2", "c1", "random", "slice", "empty_rows"])
+def test_host_cut_matches_oracle(case, monkeypatch):
+    """Fused C = A*A with host operands and short rows: chunks cut on the host from A.row_ptr,
+    per-chunk count inside execute, operands uploaded in interleaved row_ptr/col/value pieces
+    (SPGEMM_PIECE_NNZ forces many pieces so chunks wait on different ones).  Same C as the
+    oracle, and as the same plan with the host cut disabled; products known after execute."""
+    kw = {"fused": True}
+    rows = None
+    if case == "c2":
+        A = W.stencil_3d27(20)
+        kw["min_chunks"] = 9
+    elif case == "c1":
+        A = W.stencil_2d5(64)
+        kw["chunk_nnz"] = 3000
+    elif case == "random":
+        A = W.random_csr_sparse(3000, 3000, 6.0, seed=31)
+        kw["chunk_nnz"] = 20000
+    elif case == "slice":
+        A = W.stencil_3d27(16)
+        kw.update(row_begin=700, row_end=3500, chunk_nnz=40000)
+        rows = list(range(700, 3500))
+    else:
+        A = W.random_csr(2000, 2000, 0.002, seed=5)  # many empty rows
+        kw["chunk_nnz"] = 5000
+    monkeypatch.setenv("SPGEMM_PIECE_NNZ", "7000")
+    outs = []
+    for off in ("0", "1"):
+        monkeypatch.setenv("SPGEMM_NO_HOST_CUT", off)
+        with capi.Plan(A, A, 0, capi.opts(**kw)) as P:
+            pre = P.info()
+            n = info_nrows = pre["nrows"]
+            cap = int(oracle.row_nnz(A, A, rows=rows).sum()) if rows else int(oracle.row_nnz(A, A).sum())
+            rp = torch.empty(info_nrows + 1, dtype=torch.int64, pin_memory=True)
+            col = torch.empty(max(cap, 1), dtype=torch.int32, pin_memory=True)
+            val = torch.empty(max(cap, 1), dtype=torch.float64, pin_memory=True)
+            z = P.execute_capacity(rp, col, val, cap)
+            info = P.info()
+            assert z == cap == info["nnz"] and n == info["nrows"]
+            u = oracle.products(A, A)
+            p = int(u[rows].sum()) if rows else int(u.sum())
+            assert info["products"] == p
+            if off == "0" and case != "empty_rows":
+                assert pre["products"] == -1  # host cut: counted inside execute
+            # a second execution of the same plan (count totals reset, not accumulated)
+            z2 = P.execute_capacity(rp, col, val, cap)
+            assert z2 == z and P.info()["products"] == p
+        outs.append((rp.numpy().copy(), col.numpy()[:z].copy(), val.numpy()[:z].copy()))
+    rp, col, val = outs[0]
+    if rows is None:
+        assert_parity(A, A, rp, col, val, exact=case in ("c2", "c1"))
+    else:  # the slice's C (row_ptr from 0) against the oracle's selected rows
+        E = oracle.spgemm(A, A, rows=rows)
+        assert oracle.compare(rp, col, val, E)["ok"] and np.array_equal(val, E["val"])
+    assert all(np.array_equal(x, y) for x, y in zip(outs[0][:2], outs[1][:2]))
