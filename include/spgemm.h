@@ -94,7 +94,13 @@ typedef struct {
                            /*   nnz(C) is known before execute (reuse, caller-sized outputs);       */
                            /* 1 = fused: spgemm_plan only counts products and cuts chunks from the  */
                            /*   row bounds min(products, ncols); each chunk's symbolic pass + scan  */
-                           /*   run inside execute, overlapped with the previous chunk's D2H        */
+                           /*   run inside execute, overlapped with the previous chunk's D2H.       */
+                           /*   C = A x A with HOST operands (A and B the same arrays) whose rows   */
+                           /*   are short (longest row^2 <= 4096): the plan does not even count --  */
+                           /*   chunks are cut on the host from A.row_ptr (nnz(A) x longest row),   */
+                           /*   each chunk's count pass runs in execute once its operand pieces     */
+                           /*   landed, and products / max_row_products are -1 until executed       */
+                           /*   (env SPGEMM_NO_HOST_CUT=1 keeps the count in the plan)               */
     int32_t col_panels;    /* column panels of B (Alg. 3 line 4, §III-D):                   */
                            /*   0 = automatic: B is used whole when it fits the budget; if it does  */
                            /*       not (SPGEMM_ERR_BUDGET), the plan is retried with B cut into the */
@@ -139,7 +145,8 @@ typedef struct {
     int64_t chunk_capacity;     /* nonzeros per ring buffer                                       */
     int64_t arena_bytes, arena_used, ring_bytes;
     int64_t rows_warp, rows_block, rows_global; /* rows per accumulator tier in the symbolic pass   */
-    int32_t fused;              /* 1 if the plan is fused (nnz, max_row_nnz = -1 until executed)    */
+    int32_t fused;              /* 1 if the plan is fused (nnz, max_row_nnz = -1 until executed;    */
+                                /* products, max_row_products too on host-cut plans, see fused)   */
     int32_t num_copies;         /* output chunks of the last execution: runs of consecutive chunks  */
                                 /* (num_chunks = symbolic/numeric units) that share one ring slot   */
                                 /* and leave in one copy per array (0 before the first execution)  */
