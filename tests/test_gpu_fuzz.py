@@ -93,3 +93,42 @@ def test_fuzz_parity(seed, m, k, n, deg, hubs, kind, fused, ring, chunk, panels,
     assert res["ok"], (res, kw, total)
     if kind == "int":
         assert np.array_equal(val.numpy()[:nloc], Es["val"])
+
+
+@settings(max_examples=int(os.environ.get("FUZZ_EXAMPLES", "30")), deadline=None, derandomize=True,
+          suppress_health_check=[HealthCheck.too_slow, HealthCheck.data_too_large,
+                                 HealthCheck.function_scoped_fixture])
+@given(seed=st.integers(0, 2**31 - 1), m=st.integers(1, 3000), deg=st.floats(0.0, 9.0), hubs=st.integers(0, 2),
+       kind=st.sampled_from(["real", "int", "zeros"]), ring=st.integers(1, 3),
+       chunk=st.sampled_from([0, 1, 97, 5000]), piece=st.sampled_from([1, 50, 999, 0]), split=st.booleans(),
+       host_cut=st.booleans())
+def test_fuzz_square_host_operands(seed, m, deg, hubs, kind, ring, chunk, piece, split, host_cut, monkeypatch):
+    """C = A*A with the same host arrays for A and B (fused): the host-cut plan (chunks cut from
+    A.row_ptr, count per chunk in execute, interleaved operand pieces of SPGEMM_PIECE_NNZ entries)
+    whenever ncols <= 4096 or the rows are short, else the counted plan; both against the oracle."""
+    rng = np.random.default_rng(seed)
+    A = make(rng, m, m, deg, hubs, kind)
+    monkeypatch.setenv("SPGEMM_NO_HOST_CUT", "0" if host_cut else "1")
+    if piece:
+        monkeypatch.setenv("SPGEMM_PIECE_NNZ", str(piece))
+    else:
+        monkeypatch.delenv("SPGEMM_PIECE_NNZ", raising=False)
+    E = oracle.spgemm(A, A)
+    r0, r1 = (m // 3, m - m // 4) if split and m > 2 else (0, m)
+    base = int(E["row_ptr"][r0])
+    nloc = int(E["row_ptr"][r1]) - base
+    kw = dict(ring=ring, chunk_nnz=chunk, row_begin=r0, row_end=r1, row_ptr_base=base, fused=True)
+    with capi.Plan(A, A, 0, capi.opts(**kw)) as P:
+        rp = torch.empty(r1 - r0 + 1, dtype=torch.int64, pin_memory=True)
+        col = torch.empty(max(nloc, 1), dtype=torch.int32, pin_memory=True)
+        val = torch.empty(max(nloc, 1), dtype=torch.float64, pin_memory=True)
+        z = P.execute_capacity(rp, col, val, nloc)
+        info = P.info()
+    assert z == nloc
+    u = oracle.products(A, A)
+    assert info["products"] == int(u[r0:r1].sum())
+    Es = oracle.spgemm(A, A, rows=np.arange(r0, r1)) if (r0, r1) != (0, m) else E
+    res = oracle.compare(rp.numpy() - base, col.numpy()[:nloc], val.numpy()[:nloc], Es)
+    assert res["ok"], (res, kw)
+    if kind == "int":
+        assert np.array_equal(val.numpy()[:nloc], Es["val"])

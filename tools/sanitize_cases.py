@@ -1,5 +1,5 @@
 """Small multiplies through every path for compute-sanitizer (memcheck / racecheck / synccheck):
-in-core two-phase and fused plans, forced chunking, long-row tiers, column panels, sink mode."""
+in-core two-phase and fused plans (host cut included), forced chunking, long-row tiers, column panels, sink mode."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
@@ -34,4 +34,10 @@ for kw in ({}, {"fused": True}, {"chunk_nnz": 3000, "ring": 3}, {"fused": True, 
     run(S, S, **kw)
     run(R, R, **kw)
     run(LA, LB, **kw)
+# host cut (fused C = A*A from host arrays) with many small interleaved operand pieces
+os.environ["SPGEMM_PIECE_NNZ"] = "500"
+for kw in ({"fused": True}, {"fused": True, "chunk_nnz": 3000, "ring": 1}):
+    run(S, S, **kw)
+    run(R, R, **kw)
+del os.environ["SPGEMM_PIECE_NNZ"]
 print("sanitize cases ok")
