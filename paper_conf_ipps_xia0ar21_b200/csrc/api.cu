@@ -552,7 +552,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     auto ring_cap = [&](int64_t need_row) {
         const size_t freeb = P->arena_bytes > P->used + 4096 ? P->arena_bytes - P->used - 4096 : 0;
         const size_t slot = (freeb / P->ring) & ~size_t(255);
-        int64_t cap = int64_t(slot / 12) & ~int64_t(63);
+        // RING_PAD elements per slot stay free for the alignment pad of run_pipeline's groups
+        int64_t cap = (int64_t(slot / 12) & ~int64_t(63)) - 2 * RING_PAD;
         if (opts.chunk_nnz > 0) cap = std::min<int64_t>(cap, std::max<int64_t>(opts.chunk_nnz, need_row));
         if (cap < std::max<int64_t>(need_row, 1))
             fail(SPGEMM_ERR_BUDGET, "ring buffer of " + std::to_string(cap) +
@@ -703,8 +704,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->ring_val.assign(P->ring, nullptr);
     if (P->num_chunks() > 0) {
         for (int r = 0; r < P->ring; ++r) {
-            P->ring_val[r] = P->alloc<double>(P->cap, "ring values");
-            P->ring_col[r] = P->alloc<int32_t>(P->cap, "ring col_idx");
+            P->ring_val[r] = P->alloc<double>(P->cap + RING_PAD, "ring values");
+            P->ring_col[r] = P->alloc<int32_t>(P->cap + RING_PAD, "ring col_idx");
         }
         P->ring_bytes = size_t(P->ring) * size_t(P->cap) * 12;
     }
@@ -930,9 +931,19 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
     // next unit would not fit the slot, when it reaches its target (the first group: one unit;
     // each later target: twice the previous group), or when the previous group's copy has
     // finished (so the copy engine never waits for a large group to fill).
+    static const bool no_pad = [] {  // ablation knob: ring data at the start of the slot
+        const char *v = getenv("SPGEMM_NO_ALIGN_PAD");
+        return v && v[0] == '1';
+    }();
+    // A group's data starts `pad` elements into its ring slot, chosen so that the slot addresses
+    // and the host destinations agree modulo 256 bytes; its copy is split into a head up to the
+    // first 256-byte boundary of the host values and an aligned bulk.  Copy-engine D2H copies to
+    // unaligned host addresses ran ~3.5 % slower on the host link (tools/d2h_interference.py:
+    // 52.4 vs 54.0 GB/s for the C2 chunk copies; aligning source and destination to each other
+    // alone gained nothing).
     struct Group {
         int b;
-        int64_t u0, u1, r0, r1, off, nnz;
+        int64_t u0, u1, r0, r1, off, nnz, pad;
     };
     std::vector<Group> groups;
     int64_t done_cb = 0;
@@ -958,8 +969,20 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         int32_t *dcol = sink ? st_col(G.b) : col_out + G.off;
         double *dval = sink ? st_val(G.b) : val_out + G.off;
         if (G.nnz > 0) {
-            CK(cudaMemcpyAsync(dcol, P->ring_col[G.b], sizeof(int32_t) * G.nnz, cudaMemcpyDeviceToHost, cp));
-            CK(cudaMemcpyAsync(dval, P->ring_val[G.b], sizeof(double) * G.nnz, cudaMemcpyDeviceToHost, cp));
+            // a head of < 32 elements up to the first 256-byte boundary of the host values, then
+            // the bulk with source and destination both aligned
+            int64_t h = 0;
+            if (!no_pad) h = std::min<int64_t>(G.nnz, int64_t(((256u - (reinterpret_cast<uintptr_t>(dval) & 255u)) & 255u) / 8u));
+            const int32_t *scol = P->ring_col[G.b] + G.pad;
+            const double *sval = P->ring_val[G.b] + G.pad;
+            if (h > 0) {
+                CK(cudaMemcpyAsync(dcol, scol, sizeof(int32_t) * h, cudaMemcpyDeviceToHost, cp));
+                CK(cudaMemcpyAsync(dval, sval, sizeof(double) * h, cudaMemcpyDeviceToHost, cp));
+            }
+            if (G.nnz > h) {
+                CK(cudaMemcpyAsync(dcol + h, scol + h, sizeof(int32_t) * (G.nnz - h), cudaMemcpyDeviceToHost, cp));
+                CK(cudaMemcpyAsync(dval + h, sval + h, sizeof(double) * (G.nnz - h), cudaMemcpyDeviceToHost, cp));
+            }
         }
         if (sink) {
             CK(cudaMemcpyAsync(st_rp(G.b), P->crp + G.r0, sizeof(int64_t) * (G.r1 - G.r0 + 1), cudaMemcpyDeviceToHost, cp));
@@ -971,7 +994,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         CK(cudaEventRecord(P->ev_d2h[G.b], cp));
     };
 
-    Group cur{-1, 0, 0, 0, 0, 0, 0};
+    Group cur{-1, 0, 0, 0, 0, 0, 0, 0};
     int64_t target = 0;
     static const bool no_groups = [] {  // ablation knob: one output chunk per unit
         const char *v = getenv("SPGEMM_NO_GROUPS");
@@ -1010,7 +1033,12 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         }
         if (cur.b < 0) {  // open a group in the next ring slot
             const int64_t g = int64_t(groups.size());
-            cur = Group{int(g % ring), j, j, r0, r0, o, 0};
+            cur = Group{int(g % ring), j, j, r0, r0, o, 0, 0};
+            if (!sink && val_out && !no_pad) {
+                const uintptr_t hv = reinterpret_cast<uintptr_t>(val_out + o);
+                const uintptr_t rv = reinterpret_cast<uintptr_t>(P->ring_val[cur.b]);
+                cur.pad = int64_t(((hv - rv) & 255u) / 8u);  // < RING_PAD
+            }
             if (g >= ring) {
                 CK(cudaStreamWaitEvent(s, P->ev_d2h[cur.b], 0));
                 if (sink) consume(g - ring);  // frees staging slot cur.b
@@ -1020,7 +1048,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         if (!P->chunk_wait.empty() && P->chunk_wait[j] >= 0)       // host operands: value pieces
             CK(cudaStreamWaitEvent(s, P->ev_piece[P->chunk_wait[j]], 0));
         pe.rec(size_t(j) * per + 5, s);
-        enqueue_numeric(P, j, cur.b, cur.nnz, mx, pe.at(size_t(j) * per + 6));
+        enqueue_numeric(P, j, cur.b, cur.pad + cur.nnz, mx, pe.at(size_t(j) * per + 6));
         cur.nnz += n;
         cur.u1 = j + 1;
         cur.r1 = r1;

@@ -14,6 +14,8 @@
 namespace spgh {
 using namespace spg;
 
+// spare elements per ring slot for the alignment pad of an output chunk (run_pipeline)
+constexpr int64_t RING_PAD = 32;
 
 extern thread_local std::string g_err;
 
