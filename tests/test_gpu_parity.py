@@ -557,3 +557,24 @@ def test_host_cut_matches_oracle(case, monkeypatch):
         E = oracle.spgemm(A, A, rows=rows)
         assert oracle.compare(rp, col, val, E)["ok"] and np.array_equal(val, E["val"])
     assert all(np.array_equal(x, y) for x, y in zip(outs[0][:2], outs[1][:2]))
+
+
+@pytest.mark.parametrize("shift", [0, 1, 3, 17])
+def test_unaligned_host_outputs(shift):
+    """Output chunks are padded in their ring slots to the host destination's alignment and copied
+    as a head + an aligned bulk: host buffers at any element offset get the same C (fused and
+    two-phase plans, small chunks so that many chunks start at odd offsets)."""
+    A = W.stencil_3d27(14)
+    z = int(oracle.row_nnz(A, A).sum())
+    E = oracle.spgemm(A, A)
+    for fused in (True, False):
+        with capi.Plan(A, A, 0, capi.opts(fused=fused, chunk_nnz=9000, ring=3)) as P:
+            rp = torch.empty(A.nrows + 1, dtype=torch.int64, pin_memory=True)
+            colb = torch.full((z + shift,), -7, dtype=torch.int32, pin_memory=True)
+            valb = torch.full((z + shift,), -7.0, dtype=torch.float64, pin_memory=True)
+            col, val = colb[shift:], valb[shift:]
+            assert P.execute_capacity(rp, col, val, z) == z
+        assert (colb[:shift] == -7).all() and (valb[:shift] == -7.0).all()
+        res = oracle.compare(rp.numpy(), col.numpy(), val.numpy(), E)
+        assert res["ok"], res
+        assert np.array_equal(val.numpy(), E["val"])
