@@ -29,4 +29,23 @@ for rep in range(3):
         if mode in ("h2d", "both"):
             r["h2d_ms"] = b0.elapsed_time(b1); r["h2d_GBps"] = n_h2d / r["h2d_ms"] / 1e6
         out[mode] = r
+# paced: the D2H in 16 pieces; H2D piece k starts when D2H piece k starts (the H2D spread over
+# the whole D2H instead of bunched at its start)
+K = 16
+for rep in range(3):
+    torch.cuda.synchronize()
+    a0, a1, b1 = ev(), ev(), ev()
+    a0.record(s1)
+    for k in range(K):
+        e = torch.cuda.Event()
+        e.record(s1)
+        s2.wait_event(e)
+        with torch.cuda.stream(s1):
+            hdst[k * n_d2h // K:(k + 1) * n_d2h // K].copy_(dsrc[k * n_d2h // K:(k + 1) * n_d2h // K], non_blocking=True)
+        with torch.cuda.stream(s2):
+            ddst[k * n_h2d // K:(k + 1) * n_h2d // K].copy_(hsrc[k * n_h2d // K:(k + 1) * n_h2d // K], non_blocking=True)
+    a1.record(s1); b1.record(s2)
+    torch.cuda.synchronize()
+    out["paced"] = {"d2h_ms": a0.elapsed_time(a1), "h2d_end_ms": a0.elapsed_time(b1)}
+    out["paced"]["d2h_GBps"] = n_d2h / out["paced"]["d2h_ms"] / 1e6
 print(json.dumps(out))
