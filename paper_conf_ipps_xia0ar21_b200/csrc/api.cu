@@ -329,7 +329,9 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
             scan(0);
             for (auto &x : th) x.join();
             const int64_t ml = *std::max_element(part.begin(), part.end());
-            if (ml <= lim && std::min<int64_t>(Bh->ncols, ml * ml) <= CAPB_NUM) hc_maxlen = ml;
+            // (ml * ml only when ml <= 2^31: a longer row means invalid input or ncols <= CAPB_NUM)
+            const int64_t ub = ml > (int64_t(1) << 31) ? Bh->ncols : std::min<int64_t>(Bh->ncols, ml * ml);
+            if (ml <= lim && ub <= CAPB_NUM) hc_maxlen = ml;
         }
     }
     P->host_cut = hc_maxlen >= 0;
@@ -476,7 +478,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     if (P->host_cut) {
         P->products = -1;  // known after the first execution
         P->max_u = -1;
-        P->max_bound = std::min<int64_t>(P->ncols, hc_maxlen * hc_maxlen);  // an upper bound
+        P->max_bound = hc_maxlen > (int64_t(1) << 31) ? P->ncols
+                                                      : std::min<int64_t>(P->ncols, hc_maxlen * hc_maxlen);  // upper bound
         P->max_deg = hc_maxlen;
     } else if (pieced_count) {
         for (size_t k = 0; k + 1 < P->bpiece_rows.size(); ++k) {
