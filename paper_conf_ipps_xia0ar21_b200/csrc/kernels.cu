@@ -400,10 +400,20 @@ __device__ __forceinline__ void warp_fill_zero(double *v, int n) {
 
 // ------------------------------------------------------------------------------------------ S2
 
-// 8 lanes per row, 4 rows per warp step, entries of a row strided over its 8 lanes: a warp has
-// the A-column loads and B.row_ptr gathers of 4 rows in flight at once (one row per warp left
-// this pass latency-bound: 0.41 ms for C2's 2 M rows of 27 entries).
-constexpr int COUNT_G = 8;
+// COUNT_G lanes per row, 32 / COUNT_G rows per warp step, entries of a row strided over its
+// lanes: a warp has the A-column loads and B.row_ptr gathers of 8 rows in flight at once (one row
+// per warp left this pass latency-bound: 0.41 ms for C2's 2 M rows of 27 entries; 8 lanes per
+// row 0.23 ms, 4 lanes 0.13 ms).  Rows longer than COUNT_LONG entries (power-law hubs) are done
+// afterwards by the whole warp, one at a time, so that no 4-lane group walks a 10^4-entry row.
+constexpr int COUNT_G = 4, COUNT_LONG = 256;
+__device__ __forceinline__ void count_row_done(int64_t acc, int64_t deg, int64_t ncols, unsigned long long &lsum,
+                                               unsigned long long &lmax, unsigned long long &lmaxb,
+                                               unsigned long long &ldeg) {
+    lsum += acc;
+    lmax = max(lmax, (unsigned long long)acc);
+    lmaxb = max(lmaxb, (unsigned long long)min(acc, ncols));
+    ldeg = max(ldeg, (unsigned long long)deg);
+}
 __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__restrict__ u, Ctl *ctl) {
     const int lane = threadIdx.x & 31, sl = lane % COUNT_G;
     const int64_t ngroups = (int64_t)gridDim.x * (blockDim.x / COUNT_G);
@@ -417,20 +427,37 @@ __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__re
         if (i < A.nrows) {
             s = A.rp[i];
             e = A.rp[i + 1];
+            if (e - s <= COUNT_LONG) {
 #pragma unroll 4
-            for (int64_t p = s + sl; p < e; p += COUNT_G) {
-                const int32_t k = __ldg(&A.col[p]);
-                acc += __ldg(&B.rp[k + 1]) - __ldg(&B.rp[k]);
+                for (int64_t p = s + sl; p < e; p += COUNT_G) {
+                    const int32_t k = __ldg(&A.col[p]);
+                    acc += __ldg(&B.rp[k + 1]) - __ldg(&B.rp[k]);
+                }
             }
         }
 #pragma unroll
         for (int o = COUNT_G / 2; o > 0; o >>= 1) acc += __shfl_xor_sync(FULLMASK, acc, o);
-        if (sl == 0 && i < A.nrows) {
+        const bool lng = i < A.nrows && e - s > COUNT_LONG;
+        if (sl == 0 && i < A.nrows && !lng) {
             u[i] = min(acc, B.ncols);  // the row's nnz bound: distinct columns <= min(products, ncols)
-            lsum += acc;
-            lmax = max(lmax, (unsigned long long)acc);
-            lmaxb = max(lmaxb, (unsigned long long)min(acc, B.ncols));
-            ldeg = max(ldeg, (unsigned long long)(e - s));
+            count_row_done(acc, e - s, B.ncols, lsum, lmax, lmaxb, ldeg);
+        }
+        unsigned lm = __ballot_sync(FULLMASK, lng && sl == 0);
+        while (lm) {  // long rows of this step: the whole warp, one row at a time
+            const int src = __ffs(lm) - 1;
+            lm &= lm - 1;
+            const int64_t ri = __shfl_sync(FULLMASK, i, src);
+            const int64_t rs = __shfl_sync(FULLMASK, s, src), re = __shfl_sync(FULLMASK, e, src);
+            int64_t a2 = 0;
+            for (int64_t p = rs + lane; p < re; p += 32) {
+                const int32_t k = __ldg(&A.col[p]);
+                a2 += __ldg(&B.rp[k + 1]) - __ldg(&B.rp[k]);
+            }
+            a2 = warp_sum(a2);
+            if (lane == 0) {
+                u[ri] = min(a2, B.ncols);
+                count_row_done(a2, re - rs, B.ncols, lsum, lmax, lmaxb, ldeg);
+            }
         }
     }
     // warp reduction of the block maxima / sums, one atomic each per warp
