@@ -940,10 +940,10 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
     }();
     // A group's data starts `pad` elements into its ring slot, chosen so that the slot addresses
     // and the host destinations agree modulo 256 bytes; its copy is split into a head up to the
-    // first 256-byte boundary of the host values and an aligned bulk.  Copy-engine D2H copies to
-    // unaligned host addresses ran ~3.5 % slower on the host link (tools/d2h_interference.py:
-    // 52.4 vs 54.0 GB/s for the C2 chunk copies; aligning source and destination to each other
-    // alone gained nothing).
+    // next 8 KB boundary of the host values and a bulk that starts page-aligned on the host and
+    // 256-byte aligned on the device.  On some boxes copy-engine D2H copies whose host destination
+    // does not start on a page ran 6 % slower (tools/d2h_offsets.py: C2's output in 9 copies at
+    // 53.7 GB/s with 128-byte-aligned starts, 56.7 with 4 KB-aligned ones, 57.1 as one copy).
     struct Group {
         int b;
         int64_t u0, u1, r0, r1, off, nnz, pad;
@@ -974,8 +974,10 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         if (G.nnz > 0) {
             // a head of < 32 elements up to the first 256-byte boundary of the host values, then
             // the bulk with source and destination both aligned
+            // head: up to the next 8 KB boundary of the host values (then, with page-aligned host
+            // arrays, the columns start on a 4 KB boundary too)
             int64_t h = 0;
-            if (!no_pad) h = std::min<int64_t>(G.nnz, int64_t(((256u - (reinterpret_cast<uintptr_t>(dval) & 255u)) & 255u) / 8u));
+            if (!no_pad) h = std::min<int64_t>(G.nnz, int64_t(((8192u - (reinterpret_cast<uintptr_t>(dval) & 8191u)) & 8191u) / 8u));
             const int32_t *scol = P->ring_col[G.b] + G.pad;
             const double *sval = P->ring_val[G.b] + G.pad;
             if (h > 0) {
@@ -990,8 +992,13 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         if (sink) {
             CK(cudaMemcpyAsync(st_rp(G.b), P->crp + G.r0, sizeof(int64_t) * (G.r1 - G.r0 + 1), cudaMemcpyDeviceToHost, cp));
         } else if (rp_out && P->fused && G.r1 > G.r0) {
-            CK(cudaMemcpyAsync(rp_out + G.r0 + 1, P->crp + G.r0 + 1, sizeof(int64_t) * (G.r1 - G.r0),
-                               cudaMemcpyDeviceToHost, cp));
+            int64_t *drp = rp_out + G.r0 + 1;
+            const int64_t n = G.r1 - G.r0;
+            int64_t h = 0;  // head up to the next 4 KB boundary of the host destination
+            if (!no_pad) h = std::min<int64_t>(n, int64_t(((4096u - (reinterpret_cast<uintptr_t>(drp) & 4095u)) & 4095u) / 8u));
+            if (h > 0) CK(cudaMemcpyAsync(drp, P->crp + G.r0 + 1, sizeof(int64_t) * h, cudaMemcpyDeviceToHost, cp));
+            if (n > h)
+                CK(cudaMemcpyAsync(drp + h, P->crp + G.r0 + 1 + h, sizeof(int64_t) * (n - h), cudaMemcpyDeviceToHost, cp));
         }
         pe.rec(size_t(G.u1 - 1) * per + 11, cp);
         CK(cudaEventRecord(P->ev_d2h[G.b], cp));
