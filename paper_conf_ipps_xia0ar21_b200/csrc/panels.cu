@@ -387,13 +387,16 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
     {
         size_t off = 0;
         Q.hoff.assign(size_t(np) * 3, 0);
+        // every parked array starts on a host page (copies to or from an offset within a page
+        // ran up to 6 % slower on some boxes, tools/d2h_offsets.py)
+        auto al4k = [](size_t x) { return (x + 4095) & ~size_t(4095); };
         for (int j = 0; j < np; ++j) {
             Q.hoff[3 * j] = off;
-            off += al256(size_t(K + 1) * 8);
+            off += al4k(size_t(K + 1) * 8);
             Q.hoff[3 * j + 1] = off;
-            off += al256(size_t(Q.pnnz[j]) * 4);
+            off += al4k(size_t(Q.pnnz[j]) * 4);
             Q.hoff[3 * j + 2] = off;
-            off += al256(size_t(Q.pnnz[j]) * 8);
+            off += al4k(size_t(Q.pnnz[j]) * 8);
         }
         try {
             Q.hpan = (char *)pin_acquire(off);
