@@ -22,6 +22,16 @@
  * stored (Alg. 1 L42-44; reading R1).  Values are the fp64 sums of the products in some order;
  * each satisfies |c - c_exact| <= 1e-12 * sum_k |a_ik * b_kj| (BASELINE.json north_star).
  *
+ * Input preconditions (§II-A "column ids are sorted for each row"; reading R2):
+ * every row's col_idx strictly increasing (sorted, no duplicates), 0 <= col < ncols, row_ptr
+ * non-decreasing.  opts.validate = 1 checks all of it on the device and fails the plan with
+ * SPGEMM_ERR_INVALID_ARGUMENT BEFORE any kernel indexes the operands with those offsets or
+ * columns.  With validate = 0 the preconditions are the caller's: a column repeated inside a row
+ * of B keeps the structure of C exact (the hash passes count distinct columns) but its value is
+ * undefined (the warp tier adds one B row's products without atomics, relying on distinct columns
+ * within a row); an unsorted row may be cut wrongly into column pieces; an out-of-range index or
+ * offset is undefined behaviour (typically SPGEMM_ERR_CUDA, an illegal address).
+ *
  * Errors: every call returns a status; on error a thread-local message is available from
  * spgemm_last_error(), out-parameters are left untouched (plan_out is set to NULL), and the
  * library has released whatever the failed call allocated.  No call aborts the process.
@@ -38,7 +48,7 @@
 extern "C" {
 #endif
 
-#define SPGEMM_ABI_VERSION 2
+#define SPGEMM_ABI_VERSION 3
 
 typedef enum {
     SPGEMM_OK = 0,
@@ -78,7 +88,8 @@ typedef struct {
 
 typedef struct {
     int32_t device;        /* CUDA ordinal; -1 = the calling thread's current device                */
-    int32_t validate;      /* 1 = check both inputs on the device (sortedness, bounds, row_ptr)     */
+    int32_t validate;      /* 1 = check both inputs (row_ptr monotone and within the arrays, columns */
+                           /*   strictly increasing and in range) before any kernel reads them     */
     int32_t ring;          /* device C chunk buffers, >= 1 (1 = synchronous ablation); default 2    */
     int32_t profile;       /* 1 = time every kernel class with CUDA events (spgemm_stats)           */
     int64_t row_begin;     /* rows [row_begin, row_end) of A are this plan's row panel (multi-GPU  */
@@ -190,6 +201,23 @@ spgemm_status spgemm_execute(spgemm_plan_t plan, spgemm_csr_out *C_out);
 typedef int (*spgemm_chunk_cb)(void *user, int64_t row0, int64_t row1, const int64_t *row_ptr,
                                const int32_t *col_idx, const double *values, int64_t nnz);
 spgemm_status spgemm_execute_stream(spgemm_plan_t plan, spgemm_chunk_cb cb, void *user);
+
+/* S2 on its own ("row analysis", §III-B): u_out[i - row_begin] = the number of
+ * intermediate products of row i of A x B, sum over k in A_i* of nnz(B_k*) (the trip count of
+ * Alg. 1 line 4, L40), for i in [opts.row_begin, opts.row_end) -- the same k_count kernel the
+ * plan runs, without the plan's clamp to min(u_i, ncols).  Reads A.row_ptr, A.col_idx and
+ * B.row_ptr only; host operands are copied into a temporary device buffer (cudaMalloc, freed
+ * before return; this is an analysis call, not the pipeline).  u_out: HOST memory, one int64 per
+ * row; *total_out (may be NULL): the sum.  Synchronises opts.stream (NULL = legacy default).
+ * Errors: as spgemm_plan for the operands; opts.validate is ignored (no check of col_idx). */
+spgemm_status spgemm_row_products(const spgemm_csr *A, const spgemm_csr *B, const spgemm_opts *opts,
+                                  int64_t *u_out, int64_t *total_out);
+
+/* The plan's per-row bounds b_i = min(u_i, ncols) (S2: the count pass's output that sizes
+ * the row tiers and the fused chunk cut) copied to HOST bnd_out [nrows of the plan's slice].
+ * SPGEMM_ERR_STATE for column-panel plans, and for host-cut plans before their first execution
+ * (their count passes run inside execute). */
+spgemm_status spgemm_plan_row_bounds(spgemm_plan_t plan, int64_t *bnd_out);
 
 /* Add `delta` to n host row_ptr entries (multi-GPU with fused plans: a rank's global base is known
  * only after every rank has counted its nnz, i.e. after execution).  Host memory, in place. */

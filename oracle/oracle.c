@@ -32,6 +32,19 @@
  * -ffast-math (fp64 products must round exactly once, Alg. 1 line 5).
  *
  * Index widths (reading R3): row_ptr int64, col int32, val fp64.
+ *
+ * Comparison rule (SURVEY.md §8(c) "Comparison rule"), used by oracle_verify
+ * below and, identically, by oracle.compare() in Python:
+ *   row_ptr and col_idx bit-identical to the oracle's (sorted, unique columns, §II-B);
+ *   each value v against ref = (double) long-double sum and tol = (double)(1e-12 * sum |a*b|):
+ *     NaN on either side   -> good iff both are NaN;
+ *     Inf on either side   -> good iff v == ref (same infinity);
+ *     otherwise            -> good iff |v - ref| <= tol  (tol = 0 -> v must equal ref, +-0.0).
+ * oracle_verify checks a candidate's rows while it computes them, without storing the oracle's
+ * output (full-size parity of C3 / C4 / C5, whose C is larger than host memory).  Structure:
+ * the candidate row must be strictly increasing, every column must be in the oracle's set S_i
+ * (the marker array of Alg. 1 line 6) and the counts must agree -- which is the same as
+ * col == sorted(S_i) element by element, without sorting S_i.
  */
 #include <math.h>
 #include <pthread.h>
@@ -48,6 +61,16 @@ typedef struct {
 
 /* ---------------------------------------------------------------------------------------- */
 /* thread pool over a row selection                                                          */
+
+/* verification statistics (oracle_verify) */
+typedef struct {
+    int64_t rows, entries, products;   /* rows / candidate entries checked, products walked        */
+    int64_t bad_rows, bad_row_ptr, bad_col, bad_val, bad_products;
+    int64_t first_bad_row;             /* -1 if none (smallest failing row index)                  */
+    int32_t first_bad_kind;            /* 0 none, 1 row_ptr (nnz), 2 col, 3 value, 4 products      */
+    int32_t pad;
+    double worst_ratio;                /* max |v - ref| / tol over good-by-tolerance entries        */
+} vstat;
 
 typedef struct job job;
 typedef void (*row_fn)(job *, void *scratch, int64_t sel_index, int64_t row);
@@ -66,6 +89,16 @@ struct job {
     int32_t *col;
     double *val, *ref, *tol;
     int status;
+    /* oracle_verify: candidate rows (offsets relative to crp[0]) and merged statistics */
+    int64_t row0;
+    const int64_t *crp;
+    const int32_t *ccol;
+    const double *cval;
+    const int64_t *cprod;  /* optional candidate products per row (NULL: not checked) */
+    vstat *vout;
+    pthread_mutex_t mu;
+    struct spa **pool;  /* optional persistent scratch, one per thread (oracle_verify_ctx) */
+    int pool_n, pool_next;
 };
 
 static void *worker(void *arg) {
@@ -129,7 +162,8 @@ int oracle_products(const ocsr *A, const ocsr *B, const int64_t *rows, int64_t n
 /* ---------------------------------------------------------------------------------------- */
 /* Alg. 1 with a dense marker array                                                          */
 
-typedef struct {
+
+typedef struct spa {
     int64_t *mark;      /* mark[j] == gen  <=>  C_ij in C_i* for the row being built (Alg. 1 line 6) */
     int64_t gen;        /* one fresh stamp per row (rows may repeat in a selection) */
     double *acc;        /* fp64 accumulator, Alg. 1 order */
@@ -137,12 +171,14 @@ typedef struct {
     long double *absL;  /* sum of |products| for the tolerance */
     int32_t *touched;   /* columns inserted in this row (insert(), Alg. 1 line 7) */
     int64_t ntouched;
+    vstat vs;           /* oracle_verify: this thread's statistics */
 } spa;
 
-static void *spa_new(job *J) {
-    int64_t n = J->B->ncols > 0 ? J->B->ncols : 1;
+static void *spa_alloc(int64_t ncols) {
+    int64_t n = ncols > 0 ? ncols : 1;
     spa *s = (spa *)calloc(1, sizeof(spa));
     if (!s) return NULL;
+    s->vs.first_bad_row = -1;
     s->mark = (int64_t *)malloc(sizeof(int64_t) * n);
     s->acc = (double *)malloc(sizeof(double) * n);
     s->accL = (long double *)malloc(sizeof(long double) * n);
@@ -152,6 +188,8 @@ static void *spa_new(job *J) {
     for (int64_t j = 0; j < n; ++j) s->mark[j] = -1;
     return s;
 }
+
+static void *spa_new(job *J) { return spa_alloc(J->B->ncols); }
 
 static void spa_free_members(spa *s) {
     free(s->mark); free(s->acc); free(s->accL); free(s->absL); free(s->touched);
@@ -222,10 +260,22 @@ static void numeric_row(job *J, void *sv, int64_t t, int64_t i) {
     }
 }
 
+static void vmerge(job *J, const vstat *x);
+
 /* worker wrapper that frees the spa members (scratch is a struct of pointers) */
 static void *worker_spa(void *arg) {
     job *J = (job *)arg;
-    spa *s = (spa *)spa_new(J);
+    spa *s = NULL;
+    if (J->pool) {  /* persistent scratch: marks stay valid (stamps only grow), stats restart */
+        int k = __atomic_fetch_add(&J->pool_next, 1, __ATOMIC_RELAXED);
+        if (k < J->pool_n) {
+            s = J->pool[k];
+            memset(&s->vs, 0, sizeof s->vs);
+            s->vs.first_bad_row = -1;
+        }
+    } else {
+        s = (spa *)spa_new(J);
+    }
     if (!s) {
         __atomic_store_n(&J->status, -1, __ATOMIC_SEQ_CST);
         return NULL;
@@ -236,8 +286,11 @@ static void *worker_spa(void *arg) {
         int64_t e = b + 64 < J->nsel ? b + 64 : J->nsel;
         for (int64_t t = b; t < e; ++t) J->fn(J, s, t, J->rows ? J->rows[t] : t);
     }
-    spa_free_members(s);
-    free(s);
+    if (J->vout) vmerge(J, &s->vs);
+    if (!J->pool) {
+        spa_free_members(s);
+        free(s);
+    }
     return NULL;
 }
 
@@ -342,4 +395,173 @@ int oracle_numeric_esc(const ocsr *A, const ocsr *B, const int64_t *rows, int64_
     J.A = A; J.B = B; J.rows = rows; J.nsel = nsel; J.fn = esc_row;
     J.out_rp = out_rp; J.col = col; J.val = val;
     return run(&J, nthreads);
+}
+
+/* ---------------------------------------------------------------------------------------- */
+/* verification of a candidate's rows against Alg. 1 (full-size parity without storing C)     */
+
+static void vbad(vstat *v, int64_t row, int kind) {
+    if (v->first_bad_row < 0 || row < v->first_bad_row) {
+        v->first_bad_row = row;
+        v->first_bad_kind = kind;
+    }
+}
+
+static void vmerge(job *J, const vstat *x) {
+    pthread_mutex_lock(&J->mu);
+    vstat *o = J->vout;
+    o->rows += x->rows;
+    o->entries += x->entries;
+    o->products += x->products;
+    o->bad_rows += x->bad_rows;
+    o->bad_row_ptr += x->bad_row_ptr;
+    o->bad_col += x->bad_col;
+    o->bad_val += x->bad_val;
+    o->bad_products += x->bad_products;
+    if (x->first_bad_row >= 0 && (o->first_bad_row < 0 || x->first_bad_row < o->first_bad_row)) {
+        o->first_bad_row = x->first_bad_row;
+        o->first_bad_kind = x->first_bad_kind;
+    }
+    if (x->worst_ratio > o->worst_ratio) o->worst_ratio = x->worst_ratio;
+    pthread_mutex_unlock(&J->mu);
+}
+
+/* the comparison rule of the header: 1 = good; *ratio = |v - ref| / tol for finite values */
+static int value_good(double v, double ref, double tol, double *ratio) {
+    *ratio = 0.0;
+    if (isnan(v) || isnan(ref)) return isnan(v) && isnan(ref);
+    if (isinf(v) || isinf(ref)) return v == ref;
+    double err = fabs(v - ref);
+    if (err == 0.0) return 1;
+    *ratio = tol > 0.0 ? err / tol : INFINITY;
+    return err <= tol;
+}
+
+static void verify_row(job *J, void *sv, int64_t t, int64_t i_local) {
+    spa *s = (spa *)sv;
+    const ocsr *A = J->A, *B = J->B;
+    const int64_t i = J->row0 + i_local;
+    vstat *v = &s->vs;
+    /* Alg. 1 lines 3-10 for row i: structure in mark[], reference sums in accL/absL */
+    const int64_t g = ++s->gen;
+    int64_t nset = 0, u = 0;
+    for (int64_t p = A->rp[i]; p < A->rp[i + 1]; ++p) {
+        int32_t k = A->col[p];
+        long double a = (long double)A->val[p];
+        for (int64_t q = B->rp[k]; q < B->rp[k + 1]; ++q) {
+            int32_t j = B->col[q];
+            long double valueL = a * (long double)B->val[q];
+            if (s->mark[j] != g) {
+                s->mark[j] = g;
+                s->accL[j] = valueL;
+                s->absL[j] = fabsl(valueL);
+                nset++;
+            } else {
+                s->accL[j] += valueL;
+                s->absL[j] += fabsl(valueL);
+            }
+            u++;
+        }
+    }
+    v->rows++;
+    v->products += u;
+    int bad = 0;
+    if (J->cprod && J->cprod[t] != u) {
+        v->bad_products++;
+        vbad(v, i, 4);
+        bad = 1;
+    }
+    const int64_t o = J->crp[t] - J->crp[0], n = J->crp[t + 1] - J->crp[t];
+    if (n != nset) {
+        v->bad_row_ptr++;
+        vbad(v, i, 1);
+        v->bad_rows++;
+        return;
+    }
+    const int64_t nc = B->ncols;
+    int64_t prev = -1;
+    for (int64_t e = 0; e < n; ++e) {  /* structure first: sorted, in range, in S_i */
+        const int64_t j = J->ccol[o + e];
+        if (j <= prev || j < 0 || j >= nc || s->mark[j] != g) {
+            v->bad_col++;
+            vbad(v, i, 2);
+            v->bad_rows++;
+            return;
+        }
+        prev = j;
+    }
+    for (int64_t e = 0; e < n; ++e) {  /* then every value against its reference sum */
+        const int32_t j = J->ccol[o + e];
+        double r;
+        v->entries++;
+        if (!value_good(J->cval[o + e], (double)s->accL[j], (double)(1e-12L * s->absL[j]), &r)) {
+            v->bad_val++;
+            vbad(v, i, 3);
+            bad = 1;
+        } else if (r > v->worst_ratio) {
+            v->worst_ratio = r;
+        }
+    }
+    if (bad) v->bad_rows++;
+}
+
+/* Check candidate rows row0 .. row0+nrows-1 of C = A x B: crp [nrows+1] offsets (any base),
+ * ccol / cval the rows' entries from ccol[0] (= offset crp[0]), cprod [nrows] optional products
+ * per row.  *out is overwritten.  Returns 0, or < 0 on allocation failure / bad arguments. */
+/* persistent per-thread scratch for repeated oracle_verify calls over the same B (a sink checks
+ * one chunk after another: allocating and stamping a dense marker array of ncols entries per
+ * thread per call would cost more than the check of a small chunk) */
+typedef struct {
+    int64_t ncols;
+    int n;
+    spa **s;
+} vctx;
+
+void oracle_verify_ctx_free(void *c) {
+    vctx *x = (vctx *)c;
+    if (!x) return;
+    for (int t = 0; t < x->n; ++t)
+        if (x->s[t]) {
+            spa_free_members(x->s[t]);
+            free(x->s[t]);
+        }
+    free(x->s);
+    free(x);
+}
+
+void *oracle_verify_ctx_new(int64_t ncols, int nthreads) {
+    if (nthreads < 1) nthreads = 1;
+    if (nthreads > 256) nthreads = 256;
+    vctx *x = (vctx *)calloc(1, sizeof(vctx));
+    if (!x) return NULL;
+    x->ncols = ncols;
+    x->n = nthreads;
+    x->s = (spa **)calloc((size_t)nthreads, sizeof(spa *));
+    if (!x->s) { free(x); return NULL; }
+    for (int t = 0; t < nthreads; ++t)
+        if (!(x->s[t] = (spa *)spa_alloc(ncols))) { oracle_verify_ctx_free(x); return NULL; }
+    return x;
+}
+
+int oracle_verify(const ocsr *A, const ocsr *B, int64_t row0, int64_t nrows, const int64_t *crp,
+                  const int32_t *ccol, const double *cval, const int64_t *cprod, int nthreads, vstat *out,
+                  void *ctx) {
+    memset(out, 0, sizeof *out);
+    out->first_bad_row = -1;
+    if (row0 < 0 || nrows < 0 || row0 + nrows > A->nrows) return -3;
+    job J;
+    memset(&J, 0, sizeof J);
+    J.A = A; J.B = B; J.rows = NULL; J.nsel = nrows; J.fn = verify_row;
+    J.row0 = row0; J.crp = crp; J.ccol = ccol; J.cval = cval; J.cprod = cprod; J.vout = out;
+    if (ctx) {
+        vctx *x = (vctx *)ctx;
+        if (x->ncols != B->ncols) return -4;
+        J.pool = x->s;
+        J.pool_n = x->n;
+        if (nthreads > x->n) nthreads = x->n;
+    }
+    pthread_mutex_init(&J.mu, NULL);
+    int rc = run_spa(&J, nthreads);
+    pthread_mutex_destroy(&J.mu);
+    return rc;
 }

@@ -244,6 +244,12 @@ class Plan:
             raise err[0]
         _check(st)
 
+    def row_bounds(self) -> np.ndarray:
+        """The plan's per-row bounds min(products, ncols) (spgemm_plan_row_bounds)."""
+        out = np.zeros(max(self.info()["nrows"], 1), dtype=np.int64)
+        _check(_lib.spgemm_plan_row_bounds(self.h, out.ctypes.data))
+        return out[:self.info()["nrows"]]
+
     def set_row_ptr_base(self, base: int):
         _check(_lib.spgemm_set_row_ptr_base(self.h, int(base)))
 
@@ -320,3 +326,25 @@ def rebase_host(row_ptr, delta: int) -> None:
     """row_ptr[:] += delta in place (host int64 array / tensor), in the library."""
     n = row_ptr.shape[0]
     _check(_lib.spgemm_rebase_host(_ptr(row_ptr), int(n), int(delta)))
+
+
+_lib.spgemm_row_products.restype = ctypes.c_int
+_lib.spgemm_row_products.argtypes = [ctypes.POINTER(spgemm_csr), ctypes.POINTER(spgemm_csr),
+                                     ctypes.POINTER(spgemm_opts), _P, ctypes.POINTER(ctypes.c_int64)]
+_lib.spgemm_plan_row_bounds.restype = ctypes.c_int
+_lib.spgemm_plan_row_bounds.argtypes = [_P, _P]
+EXPORTED = EXPORTED + ("spgemm_row_products", "spgemm_plan_row_bounds")
+
+
+def row_products(A, B, o: Optional[spgemm_opts] = None):
+    """(u, total): intermediate products of every row of A x B in the plan's row range, by the
+    library's count kernel (spgemm_row_products)."""
+    ca, ka = make_csr(A)
+    cb, kb = make_csr(B)
+    o = o if o is not None else opts()
+    r1 = int(A.nrows) if o.row_end < 0 else int(o.row_end)
+    u = np.zeros(max(r1 - int(o.row_begin), 1), dtype=np.int64)
+    tot = ctypes.c_int64(0)
+    _check(_lib.spgemm_row_products(ctypes.byref(ca), ctypes.byref(cb), ctypes.byref(o), u.ctypes.data,
+                                    ctypes.byref(tot)))
+    return u[:r1 - int(o.row_begin)], tot.value

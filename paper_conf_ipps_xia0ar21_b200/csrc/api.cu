@@ -20,6 +20,7 @@
 #include <thread>
 #include <cstdio>
 #include <cstdlib>
+#include <cstddef>
 #include <cstring>
 #include <functional>
 #include <mutex>
@@ -117,6 +118,15 @@ void spgh::check_csr(const spgemm_csr *M, const char *name) {
         if (M->row_ptr[M->nrows] != M->nnz)
             fail(SPGEMM_ERR_INVALID_ARGUMENT, std::string(name) + ".row_ptr[nrows] != nnz");
     }
+}
+
+// validate = 1, host operand: row_ptr non-decreasing (O(nrows) on the host, before any copy is
+// sized from it); the columns are checked on the device by k_validate
+void spgh::check_rows_host(const spgemm_csr *M, const char *name) {
+    if (M->where != SPGEMM_HOST) return;
+    for (int64_t r = 0; r < M->nrows; ++r)
+        if (M->row_ptr[r + 1] < M->row_ptr[r])
+            fail(SPGEMM_ERR_INVALID_ARGUMENT, std::string(name) + ".row_ptr decreases at row " + std::to_string(r));
 }
 
 namespace {
@@ -222,6 +232,10 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     spgemm_opts opts;
     spgemm_opts_default(&opts);
     if (o) opts = *o;
+    if (opts.validate) {
+        check_rows_host(Ah, "A");
+        check_rows_host(Bh, "B");
+    }
     const int64_t rb = opts.row_begin, re = opts.row_end < 0 ? Ah->nrows : opts.row_end;
     if (rb < 0 || re < rb || re > Ah->nrows) fail(SPGEMM_ERR_SHAPE, "row range outside A");
     if (re - rb > INT32_MAX) fail(SPGEMM_ERR_INDEX_OVERFLOW, "more than INT32_MAX rows in one plan");
@@ -468,9 +482,19 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     CK(cudaMemsetAsync(P->crp, 0, sizeof(int64_t), s));
 
     if (opts.validate) {
-        launch_validate(P->A, P->ctl, s);
-        launch_validate(P->B, P->ctl, s);
+        // every offset checked against the caller's whole array (device: its own first entry;
+        // host: the arena copy), and the result read back BEFORE any kernel indexes the operands
+        // with these offsets or columns
+        const int64_t *a0 = Ah->where == SPGEMM_DEVICE ? Ah->row_ptr : P->a_alias ? P->B.rp : P->A.rp;
+        const int64_t an = Ah->where == SPGEMM_DEVICE ? Ah->nnz : P->a_alias ? Bh->nnz : P->nnzA;
+        launch_validate(P->A, a0, an, P->ctl, s);
+        launch_validate(P->B, Bh->where == SPGEMM_DEVICE ? Bh->row_ptr : P->B.rp, Bh->nnz, P->ctl, s);
         CKL("validate");
+        unsigned verr = 0;
+        CK(cudaMemcpyAsync(&verr, &P->ctl[0].err, sizeof(unsigned), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (verr & 2u)
+            fail(SPGEMM_ERR_INVALID_ARGUMENT, "input validation failed (unsorted/duplicate/out-of-range col_idx or bad row_ptr)");
     }
 
     // S2 count (host cut: per chunk, inside execute)
@@ -879,6 +903,9 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         CKL("row_ptr base");
         if (P->host_cut)  // the count passes of this execution accumulate sum_u / max_u / max_bound
             CK(cudaMemsetAsync(&P->ctl[0].sum_u, 0, 3 * sizeof(unsigned long long), P->astream));
+        // the symbolic passes of this execution accumulate max_nnz and the per-tier row counts
+        static_assert(offsetof(Ctl, rows_g) == offsetof(Ctl, max_nnz) + 3 * sizeof(unsigned long long), "Ctl layout");
+        CK(cudaMemsetAsync(&P->ctl[0].max_nnz, 0, 4 * sizeof(unsigned long long), P->astream));
         P->base_applied = base;
     } else {
         if (P->base_wanted != P->base_applied) {
@@ -1331,6 +1358,85 @@ spgemm_status spgemm_execute_stream(spgemm_plan_t P, spgemm_chunk_cb cb, void *u
     });
     mark_failed(P, st);
     return st;
+}
+
+spgemm_status spgemm_row_products(const spgemm_csr *A, const spgemm_csr *B, const spgemm_opts *o, int64_t *u_out,
+                                  int64_t *total_out) {
+    return guarded([&] {
+        check_csr(A, "A");
+        check_csr(B, "B");
+        if (!u_out) fail(SPGEMM_ERR_INVALID_ARGUMENT, "u_out is NULL");
+        if (A->ncols != B->nrows) fail(SPGEMM_ERR_SHAPE, "A.ncols != B.nrows");
+        spgemm_opts opts;
+        spgemm_opts_default(&opts);
+        if (o) opts = *o;
+        const int64_t rb = opts.row_begin, re = opts.row_end < 0 ? A->nrows : opts.row_end;
+        if (rb < 0 || re < rb || re > A->nrows) fail(SPGEMM_ERR_SHAPE, "row range outside A");
+        int dev = opts.device;
+        if (dev < 0) CK(cudaGetDevice(&dev));
+        DeviceGuard g(dev);
+        cudaStream_t s = (cudaStream_t)opts.stream;
+        const int64_t R = re - rb;
+        // the count reads A.rp, A.col and B.rp: host operands go up into one temporary buffer
+        // (this call is analysis, not the pipeline: no arena)
+        const int64_t p0 = A->where == SPGEMM_HOST ? A->row_ptr[rb] : 0;
+        const int64_t p1 = A->where == SPGEMM_HOST ? A->row_ptr[re] : 0;
+        size_t bytes = 256 + size_t(R) * 8 + sizeof(Ctl) + 256;
+        if (A->where == SPGEMM_HOST) bytes += size_t(R + 1) * 8 + size_t(p1 - p0) * 4 + 512;
+        if (B->where == SPGEMM_HOST) bytes += size_t(B->nrows + 1) * 8 + 256;
+        char *buf = nullptr;
+        CK(cudaMalloc(&buf, bytes));
+        struct Free {
+            char *p;
+            ~Free() { cudaFree(p); }
+        } fr{buf};
+        size_t off = 0;
+        auto take = [&](size_t n) {
+            char *q = buf + off;
+            off = (off + n + 255) & ~size_t(255);
+            return q;
+        };
+        int64_t *du = reinterpret_cast<int64_t *>(take(size_t(std::max<int64_t>(R, 1)) * 8));
+        Ctl *ctl = reinterpret_cast<Ctl *>(take(sizeof(Ctl)));
+        CK(cudaMemsetAsync(ctl, 0, sizeof(Ctl), s));
+        DevCSR dA{}, dB{};
+        if (A->where == SPGEMM_DEVICE) {
+            dA = DevCSR{A->row_ptr + rb, A->col_idx, A->values, R, A->ncols};
+        } else {
+            int64_t *rp = reinterpret_cast<int64_t *>(take(size_t(R + 1) * 8));
+            int32_t *c = reinterpret_cast<int32_t *>(take(size_t(std::max<int64_t>(p1 - p0, 1)) * 4));
+            CK(cudaMemcpyAsync(rp, A->row_ptr + rb, size_t(R + 1) * 8, cudaMemcpyHostToDevice, s));
+            if (p1 > p0) CK(cudaMemcpyAsync(c, A->col_idx + p0, size_t(p1 - p0) * 4, cudaMemcpyHostToDevice, s));
+            launch_rebase(rp, R + 1, p0, s);
+            CKL("rebase");
+            dA = DevCSR{rp, c, nullptr, R, A->ncols};
+        }
+        if (B->where == SPGEMM_DEVICE) {
+            dB = DevCSR{B->row_ptr, B->col_idx, B->values, B->nrows, B->ncols};
+        } else {
+            int64_t *rp = reinterpret_cast<int64_t *>(take(size_t(B->nrows + 1) * 8));
+            CK(cudaMemcpyAsync(rp, B->row_ptr, size_t(B->nrows + 1) * 8, cudaMemcpyHostToDevice, s));
+            dB = DevCSR{rp, nullptr, nullptr, B->nrows, B->ncols};
+        }
+        launch_count(dA, dB, du, ctl, s, true);
+        CKL("count");
+        Ctl hc;
+        if (R > 0) CK(cudaMemcpyAsync(u_out, du, size_t(R) * 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaMemcpyAsync(&hc, ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (total_out) *total_out = (int64_t)hc.sum_u;
+    });
+}
+
+spgemm_status spgemm_plan_row_bounds(spgemm_plan_t P, int64_t *bnd_out) {
+    return guarded([&] {
+        if (!P || !bnd_out) fail(SPGEMM_ERR_INVALID_ARGUMENT, "NULL argument");
+        if (P->pan) fail(SPGEMM_ERR_STATE, "column-panel plans keep no row bounds (one per panel and unit)");
+        if (P->host_cut && P->products < 0) fail(SPGEMM_ERR_STATE, "host-cut plan: bounds are counted in execute");
+        DeviceGuard g(P->device);
+        if (P->R > 0) CK(cudaMemcpyAsync(bnd_out, P->bnd, size_t(P->R) * 8, cudaMemcpyDeviceToHost, P->stream));
+        CK(cudaStreamSynchronize(P->stream));
+    });
 }
 
 spgemm_status spgemm_rebase_host(int64_t *row_ptr, int64_t n, int64_t delta) {

@@ -250,6 +250,7 @@ struct spgemm_plan_s {
 
 namespace spgh {
 void check_csr(const spgemm_csr *M, const char *name);
+void check_rows_host(const spgemm_csr *M, const char *name);
 // column-panel mode (panels.cu)
 void do_panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const spgemm_opts *o, spgemm_plan_s *P);
 int64_t run_panels(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double *val_out, int64_t capacity,

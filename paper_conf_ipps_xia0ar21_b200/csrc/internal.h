@@ -59,11 +59,14 @@ struct Ctl {
 
 // --- launchers (all asynchronous on `s`) ---------------------------------------------------
 
-// S2: bnd[i] = min(sum_{k in A_i} nnz(B_k), ncols) for i in [0, A.nrows); ctl gets the sum and max of products
-void launch_count(const DevCSR &A, const DevCSR &B, int64_t *u, Ctl *ctl, cudaStream_t s);
+// S2: bnd[i] = min(sum_{k in A_i} nnz(B_k), ncols) for i in [0, A.nrows) (raw: the sum itself); ctl
+// gets the sum and max of products.  Reads A.rp, A.col and B.rp only.
+void launch_count(const DevCSR &A, const DevCSR &B, int64_t *u, Ctl *ctl, cudaStream_t s, bool raw = false);
 
-// Validation of a CSR operand (rows strictly increasing, 0 <= col < ncols, rp non-decreasing).
-void launch_validate(const DevCSR &M, Ctl *ctl, cudaStream_t s);
+// Validation of a CSR operand (rows strictly increasing, 0 <= col < ncols, rp non-decreasing and
+// within [*rp0, *rp0 + nnz], rp0 = device pointer to the first row_ptr entry of the whole array);
+// sets ctl->err bit 1.  The caller must check it before any kernel reads the operand.
+void launch_validate(const DevCSR &M, const int64_t *rp0, int64_t nnz, Ctl *ctl, cudaStream_t s);
 
 // rp[i] -= sub for i in [0, n)
 void launch_rebase(int64_t *rp, int64_t n, int64_t sub, cudaStream_t s);

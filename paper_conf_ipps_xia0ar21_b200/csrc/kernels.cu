@@ -414,7 +414,8 @@ __device__ __forceinline__ void count_row_done(int64_t acc, int64_t deg, int64_t
     lmaxb = max(lmaxb, (unsigned long long)min(acc, ncols));
     ldeg = max(ldeg, (unsigned long long)deg);
 }
-__global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__restrict__ u, Ctl *ctl) {
+// raw = 1: u[i] = the product count itself (spgemm_row_products); 0: the row bound min(u_i, ncols)
+__global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__restrict__ u, Ctl *ctl, int raw) {
     const int lane = threadIdx.x & 31, sl = lane % COUNT_G;
     const int64_t ngroups = (int64_t)gridDim.x * (blockDim.x / COUNT_G);
     unsigned long long lsum = 0, lmax = 0, lmaxb = 0, ldeg = 0;
@@ -439,7 +440,7 @@ __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__re
         for (int o = COUNT_G / 2; o > 0; o >>= 1) acc += __shfl_xor_sync(FULLMASK, acc, o);
         const bool lng = i < A.nrows && e - s > COUNT_LONG;
         if (sl == 0 && i < A.nrows && !lng) {
-            u[i] = min(acc, B.ncols);  // the row's nnz bound: distinct columns <= min(products, ncols)
+            u[i] = raw ? acc : min(acc, B.ncols);  // the row's nnz bound: distinct columns <= min(products, ncols)
             count_row_done(acc, e - s, B.ncols, lsum, lmax, lmaxb, ldeg);
         }
         unsigned lm = __ballot_sync(FULLMASK, lng && sl == 0);
@@ -455,7 +456,7 @@ __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__re
             }
             a2 = warp_sum(a2);
             if (lane == 0) {
-                u[ri] = min(a2, B.ncols);
+                u[ri] = raw ? a2 : min(a2, B.ncols);
                 count_row_done(a2, re - rs, B.ncols, lsum, lmax, lmaxb, ldeg);
             }
         }
@@ -478,12 +479,17 @@ __global__ void __launch_bounds__(256) k_count(DevCSR A, DevCSR B, int64_t *__re
 
 // --------------------------------------------------------------------------------- validation
 
-__global__ void k_validate(DevCSR M, Ctl *ctl) {
+// Rows of M must have lo <= rp[i] <= rp[i+1] <= lo + nnz (lo = *rp0, the first row_ptr entry of
+// the caller's whole array, so a row panel or a device base is checked against the caller's
+// allocation) and strictly increasing columns in [0, ncols).  A row whose offsets are out of that
+// range is flagged without reading its columns (no access outside the caller's arrays).
+__global__ void k_validate(DevCSR M, const int64_t *rp0, int64_t nnz, Ctl *ctl) {
     const int lane = threadIdx.x & 31;
+    const int64_t lo = *rp0, hi = lo + nnz;
     const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
     for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < M.nrows; i += nw) {
         const int64_t s = M.rp[i], e = M.rp[i + 1];
-        bool bad = e < s;
+        bool bad = e < s || s < lo || e > hi;
         if (!bad)
             for (int64_t p = s + lane; p < e; p += 32) {
                 const int32_t c = M.col[p];
@@ -1467,20 +1473,20 @@ static int grid_for(int64_t n, int threads, int cap) {
     return (int)(b < cap ? b : cap);
 }
 
-void launch_count(const DevCSR &A, const DevCSR &B, int64_t *u, Ctl *ctl, cudaStream_t s) {
+void launch_count(const DevCSR &A, const DevCSR &B, int64_t *u, Ctl *ctl, cudaStream_t s, bool raw) {
     if (A.nrows == 0) return;
     int dev = 0;
     cudaGetDevice(&dev);
     int sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int blocks = grid_for(A.nrows, 256 / COUNT_G, grids(dev, sms).count_blocks);
-    k_count<<<blocks, 256, 0, s>>>(A, B, u, ctl);
+    k_count<<<blocks, 256, 0, s>>>(A, B, u, ctl, raw ? 1 : 0);
     LAUNCHED(1);
 }
 
-void launch_validate(const DevCSR &M, Ctl *ctl, cudaStream_t s) {
+void launch_validate(const DevCSR &M, const int64_t *rp0, int64_t nnz, Ctl *ctl, cudaStream_t s) {
     if (M.nrows == 0) return;
-    k_validate<<<grid_for(M.nrows, 8, 148 * 16), 256, 0, s>>>(M, ctl);
+    k_validate<<<grid_for(M.nrows, 8, 148 * 16), 256, 0, s>>>(M, rp0, nnz, ctl);
     LAUNCHED(1);
 }
 
@@ -1722,8 +1728,10 @@ __global__ void __launch_bounds__(256) k_col_hist(const int32_t *__restrict__ co
     __shared__ unsigned int h[4096];
     for (int b = threadIdx.x; b < nbins; b += blockDim.x) h[b] = 0;
     __syncthreads();
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-        atomicAdd(&h[__ldg(&col[i]) >> shift], 1u);
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t c = __ldg(&col[i]);
+        if (c >= 0 && (c >> shift) < nbins) atomicAdd(&h[c >> shift], 1u);  // (invalid ids: flagged by k_validate)
+    }
     __syncthreads();
     for (int b = threadIdx.x; b < nbins; b += blockDim.x)
         if (h[b]) atomicAdd(&hist[b], (unsigned long long)h[b]);

@@ -198,6 +198,10 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
     Q.B = *Bh;
     Q.rb = rb;
     Q.validate = opts.validate != 0;
+    if (Q.validate) {  // host row_ptr monotone before any staging copy is sized from it
+        check_rows_host(Ah, "A");
+        check_rows_host(Bh, "B");
+    }
     P->res = res_acquire(P->device);
     Res *rs = P->res;
     P->stream = opts.stream ? (cudaStream_t)opts.stream : rs->stream(rs->own);
@@ -233,6 +237,14 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
         Q.brp = Q.brp_copy.data();
     } else {
         Q.brp = Bh->row_ptr;
+    }
+    if (Q.validate && (Ah->where == SPGEMM_DEVICE || Bh->where == SPGEMM_DEVICE)) {  // the host views too
+        spgemm_csr av = *Ah, bv = *Bh;
+        av.where = bv.where = SPGEMM_HOST;
+        av.row_ptr = Q.arp;
+        bv.row_ptr = Q.brp;
+        check_rows_host(&av, "A");
+        check_rows_host(&bv, "B");
     }
     const int64_t *arp = Q.arp + rb;  // plan rows
     int64_t max_deg = 0, max_brow = 0;
@@ -320,7 +332,9 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
         const int64_t k0 = Q.bpieces[q], k1 = Q.bpieces[q + 1];
         const int32_t *c0 = nullptr;
         DevCSR v = stage_rows(P, Q, Q.B, Q.brp, k0, k1, false, &c0);
-        if (Q.validate) launch_validate(v, P->ctl, s);
+        if (Q.validate)  // (k_col_hist skips out-of-range ids; the plan fails below if any)
+            launch_validate(v, Bh->where == SPGEMM_DEVICE ? Bh->row_ptr : v.rp,
+                            Bh->where == SPGEMM_DEVICE ? Bh->nnz : Q.brp[k1] - Q.brp[k0], P->ctl, s);
         launch_col_hist(c0, Q.brp[k1] - Q.brp[k0], shift, nbins, dhist, s);
         CKL("column histogram");
         stage_done(P, Q);
@@ -336,11 +350,17 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
         auto ab = cut_rows(R, [&](int64_t a, int64_t b) { return stage_need(arp, a, b, false) <= Q.stage_bytes; });
         for (size_t q = 0; q + 1 < ab.size(); ++q) {
             DevCSR v = stage_rows(P, Q, Q.A, Q.arp, rb + ab[q], rb + ab[q + 1], false, nullptr);
-            launch_validate(v, P->ctl, s);
+            launch_validate(v, v.rp, Q.arp[rb + ab[q + 1]] - Q.arp[rb + ab[q]], P->ctl, s);
             stage_done(P, Q);
         }
     } else if (Q.validate) {
-        launch_validate(DevCSR{Ah->row_ptr + rb, Ah->col_idx, Ah->values, R, Ah->ncols}, P->ctl, s);
+        launch_validate(DevCSR{Ah->row_ptr + rb, Ah->col_idx, Ah->values, R, Ah->ncols}, Ah->row_ptr, Ah->nnz, P->ctl, s);
+    }
+    if (Q.validate) {  // A checked before any kernel reads it
+        Ctl hv;
+        CK(cudaMemcpyAsync(&hv, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (hv.err & 2u) fail(SPGEMM_ERR_INVALID_ARGUMENT, "input validation failed (A)");
     }
 
     // panel count and boundaries: the fewest panels whose largest one fits, with at least ~20% of

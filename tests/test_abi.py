@@ -49,7 +49,7 @@ def test_defaults_and_strings(capi):
     o = capi.spgemm_opts()
     capi._lib.spgemm_opts_default(ctypes.byref(o))
     assert (o.device, o.ring, o.row_begin, o.row_end, o.validate) == (-1, 2, 0, -1, 0)
-    assert capi.abi_version() == 2
+    assert capi.abi_version() == 3
     for st in range(10):
         assert capi.status_string(st).startswith("SPGEMM_")
     assert capi.status_string(4) == "SPGEMM_ERR_BUDGET"

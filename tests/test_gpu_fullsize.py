@@ -4,8 +4,9 @@ C2 (configs[1]): 3-D 27-point 128^3, device budget 2 GiB, fused plan, ring 2 -- 
 workload.  Every row_ptr entry is checked against the closed form (nnz per row = product of
 per-axis widths), every column and value of a contiguous block of rows and of sampled rows against
 the closed form A^2 = 729 I - 54 S + K^2 (x) K^2 (x) K^2 and against the oracle, and sum(C) against
-its closed form.  C3 (configs[2], R-MAT s22) streams its ~0.3 TB of C through the sink and checks
-sampled rows of every chunk against the oracle.
+its closed form.  C3 (configs[2], R-MAT s22) streams its ~0.3 TB of C through the sink and every
+row is checked against the oracle as it arrives (oracle.verify); likewise every row of the C4 / C5
+row panels one rank of an 8-GPU deal owns.
 """
 import os
 
@@ -83,83 +84,66 @@ def test_c2_full_size_budget_2gib():
     assert oracle.compare(gp, col[idx], val[idx], E)["ok"]
 
 
-def _streamed_panel_check(A, B, r1, picks_per_chunk=2, chunk_nnz=300_000_000, seed=7):
-    """Stream rows [0, r1) of C = A*B through the sink (fused plan, ring 3), keep a few sampled rows
-    per chunk, and check them against the oracle in one call at the end."""
+def _streamed_verify(A, B, r0, r1, chunk_nnz=400_000_000):
+    """Stream rows [r0, r1) of C = A*B through the sink (fused plan, ring 3, device operands) and
+    check EVERY row of every output chunk against the oracle while it is delivered (oracle.verify:
+    Alg. 1 per row on all host cores, structure bit-exact, values within the bound; nothing of C
+    is stored).  Also checks the plan's per-row bounds against the oracle's product counts."""
     dev = torch.device("cuda", 0)
     dA = _device_csr(A, dev)
     dB = dA if B is A else _device_csr(B, dev)
-    rng = np.random.default_rng(seed)
-    kept = []
-    seen = {"rows": 0, "nnz": 0, "chunks": 0}
+    ops = oracle.Operands(A, B)
+    tot = {"rows": 0, "entries": 0, "products": 0, "chunks": 0, "worst_ratio": 0.0, "bad": []}
 
-    def sink(r0, r1_, rp, col, val):
-        seen["chunks"] += 1
-        seen["rows"] += r1_ - r0
-        seen["nnz"] += int(rp[-1])
-        for r in sorted({r0, r1_ - 1} | set(rng.integers(r0, r1_, picks_per_chunk).tolist())):
-            lr = r - r0
-            kept.append((r, col[rp[lr]:rp[lr + 1]].copy(), val[rp[lr]:rp[lr + 1]].copy()))
+    def sink(ra, rb, rp, col, val):
+        res = oracle.verify(A, B, ra, rp, col, val, ops=ops)
+        tot["chunks"] += 1
+        for k in ("rows", "entries", "products"):
+            tot[k] += res[k]
+        tot["worst_ratio"] = max(tot["worst_ratio"], res["worst_ratio"])
+        if not res["ok"]:
+            tot["bad"].append((ra, rb, res["first_bad_row"], res["first_bad_kind"]))
 
-    o = capi.opts(fused=True, ring=3, chunk_nnz=chunk_nnz, row_end=r1)
+    o = capi.opts(fused=True, ring=3, chunk_nnz=chunk_nnz, row_begin=r0, row_end=r1)
     with capi.Plan(dA, dB, 0, o) as P:
+        bnd = P.row_bounds()
         P.execute_stream(sink)
         info = P.info()
-    assert seen["rows"] == r1 and seen["nnz"] == info["nnz"] and seen["chunks"] == info["num_copies"]
-    rows = np.array([k[0] for k in kept])
-    E = oracle.spgemm(A, B, rows=rows)
-    gp = np.concatenate([[0], np.cumsum([len(k[1]) for k in kept])])
-    res = oracle.compare(gp, np.concatenate([k[1] for k in kept]), np.concatenate([k[2] for k in kept]), E)
-    assert res["ok"], res
-    return info
+    assert not tot["bad"], tot["bad"][:5]
+    assert tot["rows"] == r1 - r0 and tot["entries"] == info["nnz"] and tot["products"] == info["products"]
+    assert tot["chunks"] == info["num_copies"]
+    u = oracle.products(A, B, rows=np.arange(r0, r1))
+    assert np.array_equal(bnd, np.minimum(u, B.ncols)) and int(u.sum()) == info["products"]
+    print(f"rows {r0}..{r1}: {tot['rows']} rows, {tot['entries']} entries, {tot['products']} products checked "
+          f"in {tot['chunks']} chunks, worst |c - ref| / tol = {tot['worst_ratio']:.3g}")
+    return info, tot
 
 
 @pytest.mark.skipif(os.environ.get("SPGEMM_SKIP_C45") == "1", reason="C4/C5 panel runs disabled")
 def test_c4_rmat_s24_rank_panel():
-    """configs[3] (R-MAT s24 ef16, C several TB) -- the row panel one rank of an 8-GPU deal owns."""
+    """configs[3] (R-MAT s24 ef16, C several TB): EVERY row of the row panel one rank of an 8-GPU
+    deal owns (1/8 of the rows, ~2e11 bytes of C), checked against the oracle."""
     A = W.rmat_torch(24, 16, seed=20210518)
-    info = _streamed_panel_check(A, A, A.nrows // 8)
-    assert info["rows_global"] > 0
+    info, tot = _streamed_verify(A, A, 0, A.nrows // 8)
+    assert info["rows_block"] + info["rows_global"] > 0
 
 
 @pytest.mark.skipif(os.environ.get("SPGEMM_SKIP_C45") == "1", reason="C4/C5 panel runs disabled")
 def test_c5_rectangular_rank_panel():
-    """configs[4]: A = 2^24 x 2^22 power-law, B = 2^22 x 2^24 (2^28 generated edges each), rank 0's
-    panel of an 8-GPU deal."""
+    """configs[4]: A = 2^24 x 2^22 power-law, B = 2^22 x 2^24 (2^28 generated edges each): every row
+    of rank 0's panel and of the LAST rank's panel of an 8-GPU deal (the two ends of the skew)."""
     A = W.rmat_torch(24, col_scale=22, nedges=1 << 28, seed=11, symmetric=False)
     B = W.rmat_torch(22, col_scale=24, nedges=1 << 28, seed=12, symmetric=False)
     assert A.nnz + B.nnz > 4e8
-    _streamed_panel_check(A, B, A.nrows // 8)
+    _streamed_verify(A, B, 0, A.nrows // 8)
+    _streamed_verify(A, B, A.nrows - A.nrows // 8, A.nrows)
 
 
 @pytest.mark.skipif(os.environ.get("SPGEMM_SKIP_C3") == "1", reason="C3 full-size run disabled")
 def test_c3_rmat_s22_streamed():
-    """configs[2] at full size: ~2.9e10 products, C of ~0.3 TB streamed through the sink; in every
-    chunk the first, last and a random row are compared with the oracle."""
+    """configs[2] at full size: ~2.9e10 products, C of ~0.3 TB streamed through the sink; EVERY row
+    of C is compared with the oracle as its chunk arrives."""
     A = W.rmat(22, 16)
-    dev = torch.device("cuda", 0)
-    dA = _device_csr(A, dev)
-    u = oracle.products(A, A)
-    rng = np.random.default_rng(5)
-    seen = {"rows": 0, "nnz": 0, "chunks": 0, "checked": 0}
-
-    def sink(r0, r1, rp, col, val):
-        seen["chunks"] += 1
-        seen["rows"] += r1 - r0
-        seen["nnz"] += int(rp[-1])
-        picks = sorted({r0, r1 - 1, int(rng.integers(r0, r1))})
-        E = oracle.spgemm(A, A, rows=np.array(picks), threads=8)
-        lr = np.array(picks) - r0
-        gp = np.concatenate([[0], np.cumsum(rp[lr + 1] - rp[lr])])
-        idx = np.concatenate([np.arange(rp[k], rp[k + 1]) for k in lr])
-        res = oracle.compare(gp, col[idx], val[idx], E)
-        assert res["ok"], (r0, r1, res)
-        seen["checked"] += len(picks)
-
-    o = capi.opts(fused=True, ring=3, chunk_nnz=400_000_000)
-    with capi.Plan(dA, dA, 0, o) as P:
-        P.execute_stream(sink)
-        info = P.info()
-    assert seen["rows"] == A.nrows and seen["nnz"] == info["nnz"] and info["products"] == int(u.sum())
-    assert seen["chunks"] == info["num_copies"] and seen["checked"] >= 2 * seen["chunks"]
+    info, tot = _streamed_verify(A, A, 0, A.nrows)
+    assert tot["rows"] == A.nrows == 1 << 22
     assert info["rows_global"] + info["rows_block"] > 0  # the skewed tiers were exercised

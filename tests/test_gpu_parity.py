@@ -224,14 +224,15 @@ def test_rmat_skewed():
 # ------------------------------------------------------------------------------------- out-of-core
 
 def test_forced_chunking_invariance():
-    """Chunked == unchunked, ring 1 (synchronous) == ring 2/3 (S8-S10 must not change the result)."""
+    """Any chunking, ring 1 (synchronous) or 2/3: every run equals the oracle, bit for bit on this
+    integer-valued stencil (S8-S10 must not change the result; P:L122 chunk independence)."""
     A = W.stencil_3d27(20)
-    ref = run(A, A)
-    for kw in ({"chunk_nnz": 5000}, {"chunk_nnz": 5000, "ring": 1}, {"chunk_nnz": 777, "ring": 3},
+    E = oracle.spgemm(A, A)
+    for kw in ({}, {"chunk_nnz": 5000}, {"chunk_nnz": 5000, "ring": 1}, {"chunk_nnz": 777, "ring": 3},
                {"min_chunks": 17}):
         rp, col, val, info, chunks = run(A, A, **kw)
-        assert info["num_chunks"] > 2
-        assert np.array_equal(rp, ref[0]) and np.array_equal(col, ref[1]) and np.array_equal(val, ref[2])
+        assert kw == {} or info["num_chunks"] > 2
+        assert oracle.compare(rp, col, val, E)["ok"] and np.array_equal(val, E["val"])
         rows, offs = chunks
         assert rows[0] == 0 and rows[-1] == A.nrows and np.all(np.diff(offs) <= info["chunk_capacity"])
 
@@ -255,7 +256,6 @@ def test_one_row_per_chunk():
 
 def test_execute_stream_sink_matches():
     A = W.rmat(12, 16, seed=2)
-    ref = run(A, A)
     got_rp, got_col, got_val = [0], [], []
     with capi.Plan(A, A, 0, capi.opts(chunk_nnz=20000, ring=2)) as P:
         seen = []
@@ -268,20 +268,34 @@ def test_execute_stream_sink_matches():
 
         P.execute_stream(sink)
         assert len(seen) == P.info()["num_copies"] and seen[0][0] == 0 and seen[-1][1] == A.nrows
-    assert np.array_equal(np.array(got_rp), ref[0])
-    assert np.array_equal(np.concatenate(got_col), ref[1])
+    assert all(a[1] == b[0] for a, b in zip(seen, seen[1:]))  # consecutive row ranges, in order
     # values: fp64 atomics make the summation order (not the bound) run-dependent (R10)
     assert_parity(A, A, np.array(got_rp), np.concatenate(got_col), np.concatenate(got_val))
 
 
-def test_repeat_execute_same_plan():
+@pytest.mark.parametrize("fused", [False, True])
+def test_repeat_execute_same_plan(fused):
+    """Every execution of one plan equals the oracle, and the plan's info does not drift between
+    executions (per-tier row counts are per execution)."""
     A = W.stencil_3d27(16)
-    with capi.Plan(A, A, 0, capi.opts(chunk_nnz=3000)) as P:
-        a = P.execute()
-        a = [x.copy() for x in a]
-        b = P.execute()
-        for x, y in zip(a, b):
-            assert np.array_equal(x, y)
+    E = oracle.spgemm(A, A)
+    z = len(E["col"])
+    infos = []
+    with capi.Plan(A, A, 0, capi.opts(chunk_nnz=3000, fused=fused)) as P:
+        for _ in range(3):
+            if fused:
+                rp = torch.empty(A.nrows + 1, dtype=torch.int64, pin_memory=True)
+                col = torch.empty(z, dtype=torch.int32, pin_memory=True)
+                val = torch.empty(z, dtype=torch.float64, pin_memory=True)
+                assert P.execute_capacity(rp, col, val, z) == z
+                got = (rp.numpy(), col.numpy(), val.numpy())
+            else:
+                got = [x.copy() for x in P.execute()]
+            assert oracle.compare(*got, E)["ok"] and np.array_equal(got[2], E["val"])
+            infos.append(P.info())
+    for k in ("nnz", "products", "rows_warp", "rows_block", "rows_global", "max_row_nnz"):
+        assert infos[0][k] == infos[1][k] == infos[2][k], k
+    assert infos[0]["rows_warp"] + infos[0]["rows_block"] + infos[0]["rows_global"] <= A.nrows
 
 
 # ------------------------------------------------------------------------------------- device inputs
@@ -303,19 +317,17 @@ def test_device_inputs_with_base_and_row_panels():
     row panel [row_begin, row_end) with a global row_ptr base: the union of panels == whole."""
     A = W.rmat(12, 8, seed=7)
     B = W.random_csr_sparse(A.ncols, 3000, 5.0, seed=8)
-    full = run(A, B)
+    E = oracle.spgemm(A, B)
     dA, dB = _to_dev(A, base=13), _to_dev(B, base=5)
     rp, col, val, _, _ = run(dA, dB, stream=torch.cuda.current_stream().cuda_stream)
-    assert np.array_equal(rp, full[0]) and np.array_equal(col, full[1])
-    assert np.array_equal(val, full[2]) or oracle.compare(rp, col, val, oracle.spgemm(A, B))["ok"]
+    assert oracle.compare(rp, col, val, E)["ok"]
     cuts = [0, 700, 701, 2500, A.nrows]
-    parts = []
     for r0, r1 in zip(cuts[:-1], cuts[1:]):
-        base = int(full[0][r0])
+        base = int(E["row_ptr"][r0])  # the global offset of the panel (what the ranks exchange)
         prp, pcol, pval, info, _ = run(dA, dB, row_begin=r0, row_end=r1, row_ptr_base=base)
-        assert prp[0] == base and np.array_equal(prp, full[0][r0:r1 + 1])
-        parts.append((pcol, pval))
-    assert np.array_equal(np.concatenate([p[0] for p in parts]), full[1])
+        assert prp[0] == base
+        Ep = oracle.spgemm(A, B, rows=np.arange(r0, r1))
+        assert oracle.compare(prp, pcol, pval, Ep, rows_offset=base)["ok"]
 
 
 def test_no_leak_across_plans():
@@ -367,6 +379,114 @@ def test_errors():
     with pytest.raises(capi.SpgemmError) as e:
         capi.spgemm_multiply(AA, AA, 0, None, *out, capacity=10)
     assert e.value.status == capi.ERR_CAPACITY
+
+
+def _mutated(M, kind):
+    """A copy of M broken in one way (validate must catch each before any kernel reads)."""
+    X = W.CSR(M.nrows, M.ncols, M.row_ptr.copy(), M.col.copy(), M.val.copy())
+    if kind == "col_high":
+        X.col[len(X.col) // 2] = M.ncols + 1000
+    elif kind == "col_high_last":
+        X.col[-1] = 2 ** 31 - 1
+    elif kind == "col_neg":
+        X.col[len(X.col) // 3] = -7
+    elif kind == "rp_decreasing":
+        r = M.nrows // 2
+        X.row_ptr[r] = X.row_ptr[r + 1] + 5  # rows r-1, r: one past the next offset
+    elif kind == "unsorted":
+        r = int(np.argmax(np.diff(M.row_ptr) >= 2))
+        p = int(M.row_ptr[r])
+        X.col[p], X.col[p + 1] = X.col[p + 1], X.col[p]
+    elif kind == "duplicate":
+        r = int(np.argmax(np.diff(M.row_ptr) >= 2))
+        p = int(M.row_ptr[r])
+        X.col[p + 1] = X.col[p]
+    return X
+
+
+@pytest.mark.parametrize("where", ["host", "device"])
+@pytest.mark.parametrize("operand", ["A", "B"])
+@pytest.mark.parametrize("kind", ["col_high", "col_high_last", "col_neg", "rp_decreasing", "unsorted", "duplicate"])
+def test_validate_rejects_bad_operands_before_reading(kind, operand, where):
+    """validate = 1: every malformed operand is SPGEMM_ERR_INVALID_ARGUMENT (not an illegal address
+    / sticky CUDA error), for host and device operands, in-core and column-panel plans; the
+    context stays healthy (a valid multiply afterwards matches the oracle)."""
+    A = W.random_csr_sparse(300, 200, 6.0, seed=5)
+    B = W.random_csr_sparse(200, 260, 6.0, seed=6)
+    bad = _mutated(A if operand == "A" else B, kind)
+    X, Y = (bad, B) if operand == "A" else (A, bad)
+    if where == "device":
+        X, Y = _to_dev(X, base=3), _to_dev(Y, base=0)
+    for cp in (1, 3):
+        with pytest.raises(capi.SpgemmError) as e:
+            capi.Plan(X, Y, 0, capi.opts(validate=True, col_panels=cp))
+        assert e.value.status == capi.ERR_INVALID_ARGUMENT, (kind, operand, where, cp, str(e.value))
+    torch.cuda.synchronize()
+    rp, col, val, _, _ = run(A, B, validate=True)
+    assert_parity(A, B, rp, col, val)
+
+
+@pytest.mark.parametrize("fused", [False, True])
+def test_duplicates_unvalidated_keep_structure(fused):
+    """validate = 0 with a column repeated inside rows of B (include/spgemm.h, DESIGN R2): the
+    structure of C is that of the deduplicated B, exactly; values are undefined there, and exact
+    elsewhere (rows that touch no damaged B row)."""
+    A = W.random_csr_sparse(400, 300, 5.0, seed=8)
+    B = W.random_csr_sparse(300, 250, 40.0, seed=9)   # long B rows: the G = 32 warp tier
+    Bd = W.CSR(B.nrows, B.ncols, B.row_ptr.copy(), B.col.copy(), B.val.copy())
+    damaged = []
+    for k in range(0, B.nrows, 7):
+        s, e = int(B.row_ptr[k]), int(B.row_ptr[k + 1])
+        if e - s >= 2:
+            Bd.col[s + 1] = Bd.col[s]
+            damaged.append(k)
+    # the same matrix with the duplicate dropped (structure reference)
+    keep = np.ones(len(Bd.col), bool)
+    for k in damaged:
+        keep[int(B.row_ptr[k]) + 1] = False
+    cnt = np.diff(B.row_ptr) - np.isin(np.arange(B.nrows), damaged)
+    Bu = W.CSR(B.nrows, B.ncols, np.concatenate([[0], np.cumsum(cnt)]).astype(np.int64), Bd.col[keep].copy(),
+               Bd.val[keep].copy())
+    with pytest.raises(capi.SpgemmError):
+        capi.Plan(A, Bd, 0, capi.opts(validate=True))
+    if fused:
+        rp, col, val, info, _ = run_fused(A, Bd)
+    else:
+        rp, col, val, info, _ = run(A, Bd)
+    E = oracle.spgemm(A, Bu)
+    assert np.array_equal(rp, E["row_ptr"]) and np.array_equal(col, E["col"])
+    clean = np.array([not np.isin(A.col[A.row_ptr[i]:A.row_ptr[i + 1]], damaged).any() for i in range(A.nrows)])
+    rows = np.nonzero(clean)[0]
+    assert len(rows) > 10
+    assert_parity(A, Bu, rp, col, val, rows=rows)
+
+
+@pytest.mark.parametrize("case", ["stencil", "rmat", "rect"])
+def test_row_products_and_plan_bounds_per_row(case):
+    """S2 per row: the library's count kernel gives u_i == the oracle's Alg. 1 line-4 trip count for
+    EVERY row (spgemm_row_products), and the plan's own bound array is min(u_i, ncols) for every
+    row (spgemm_plan_row_bounds) -- in two-phase and fused plans, host and device operands, and a
+    row panel."""
+    if case == "stencil":
+        A = B = W.stencil_3d27(20)
+    elif case == "rmat":
+        A = B = W.rmat(13, 16, seed=4)
+    else:
+        A = W.rmat_rect(12, 10, 40_000, seed=5)
+        B = W.rmat_rect(10, 13, 30_000, seed=6)
+    u = oracle.products(A, B)
+    got, tot = capi.row_products(A, B)
+    assert np.array_equal(got, u) and tot == int(u.sum())
+    dA, dB = _to_dev(A, base=11), _to_dev(B, base=2)
+    r0, r1 = A.nrows // 3, A.nrows - 5
+    got, tot = capi.row_products(dA, dB, capi.opts(row_begin=r0, row_end=r1))
+    assert np.array_equal(got, u[r0:r1]) and tot == int(u[r0:r1].sum())
+    for fused in (False, True):
+        with capi.Plan(A, B, 0, capi.opts(fused=fused)) as P:
+            assert np.array_equal(P.row_bounds(), np.minimum(u, B.ncols))
+            assert P.info()["products"] == int(u.sum())
+        with capi.Plan(dA, dB, 0, capi.opts(fused=fused, row_begin=r0, row_end=r1)) as P:
+            assert np.array_equal(P.row_bounds(), np.minimum(u[r0:r1], B.ncols))
 
 
 def test_multiply_one_shot():
@@ -423,11 +543,11 @@ def test_fused_matches_oracle(case):
         assert rows[0] == 0 and rows[-1] == A.nrows and offs[-1] == info["nnz"]
 
 
-def test_fused_two_phase_and_ring1_identical_structure():
+def test_fused_two_phase_and_ring1_match_oracle():
     A = W.rmat(12, 16, seed=9)
-    a = run(A, A, chunk_nnz=30000)
-    b = run_fused(A, A, chunk_nnz=30000, ring=1)
-    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    E = oracle.spgemm(A, A)
+    for r in (run(A, A, chunk_nnz=30000), run_fused(A, A, chunk_nnz=30000, ring=1)):
+        assert oracle.compare(r[0], r[1], r[2], E)["ok"]
 
 
 def test_fused_capacity_error_reports_nnz_and_plan_stays_usable():
@@ -449,29 +569,26 @@ def test_fused_capacity_error_reports_nnz_and_plan_stays_usable():
 
 def test_fused_sink_and_base():
     A = W.rmat(12, 16, seed=11)
-    ref = run(A, A)
+    E = oracle.spgemm(A, A)
     parts = []
     with capi.Plan(A, A, 0, capi.opts(fused=True, chunk_nnz=40000, ring=2, row_ptr_base=1000)) as P:
         P.execute_stream(lambda r0, r1, rp, col, val: parts.append((r0, r1, rp.copy(), col.copy(), val.copy())))
     assert parts[0][0] == 0 and parts[-1][1] == A.nrows
-    col = np.concatenate([p[3] for p in parts])
-    assert np.array_equal(col, ref[1])
     rpg = [0]
     for p in parts:
         rpg.extend((p[2][1:] + rpg[-1]).tolist())
-    assert np.array_equal(np.array(rpg), ref[0])
+    assert oracle.compare(np.array(rpg), np.concatenate([p[3] for p in parts]), np.concatenate([p[4] for p in parts]),
+                          E)["ok"]
     rp, c, v, info, _ = run_fused(A, A, row_ptr_base=777)
-    assert rp[0] == 777 and np.array_equal(rp - 777, ref[0])
+    assert rp[0] == 777 and oracle.compare(rp, c, v, E, rows_offset=777)["ok"]
 
 
 def test_chunk_order_by_flops():
     """§IV-C: chunks computed and transferred in decreasing order of flops give the
     same C as row order; fused plans and sink mode reject the reordering."""
     A = W.rmat(13, 16, seed=21)
-    ref = run(A, A, chunk_nnz=40000)
     r = run(A, A, chunk_nnz=40000, order=1)
     assert r[3]["num_chunks"] > 4
-    assert np.array_equal(r[0], ref[0]) and np.array_equal(r[1], ref[1])
     assert_parity(A, A, r[0], r[1], r[2])
     S = W.stencil_3d27(20)
     rs = run(S, S, chunk_nnz=5000, order=1, profile=True)
