@@ -1,26 +1,36 @@
 """bench.py -- C = A*A GFLOP/s (2 x intermediate products) including the D2H of all of C.
 
-Default workload (N = 1): BASELINE.json configs[1] = 3-D 27-point stencil 128^3, device budget
-forced to 2 GiB, so C (3.07 GB) is produced out-of-core in chunks and streamed to pinned host
-memory.  One step = the whole hot path (DESIGN.md §8 rows S0-S10): plan (count, symbolic,
-scan, chunk cut) + execute (numeric + sort per chunk, D2H overlapped) through the C ABI.
+Default workload (N = 1): BASELINE.json configs[2] = R-MAT scale 22, edge factor 16, symmetric
+(com-LiveJournal-like skew, 134 M nnz), C = A*A: 2.9e10 intermediate products and 2.7e10 nonzeros
+of C = 0.33 TB, larger than host memory, so every output chunk streams into a pinned staging ring
+and is handed to a sink that drops it (the paper's timing scope: "include the time for
+transferring all chunks of the output matrix", §V-C).  This is the largest
+configuration that fits one GPU ("1 GPU" in BASELINE.json); configs[0] is the oracle-sized case
+and configs[1] / [3] / [4] are selectable with --config (C2 writes C into host memory).
 
-  value  inputs resident in HBM when the timed region starts (device operands, where=DEVICE);
-  e2e    the same through the public API with HOST operands: the H2D of A (= B) from pinned
-         memory and the D2H of C are inside the timed region.
+One step = the whole hot path (DESIGN.md §2 rows S0-S10) through the C ABI: spgemm_plan (count,
+chunk cut) + spgemm_execute_stream (per chunk: symbolic + scan, numeric + sort, D2H overlapped)
++ spgemm_free, on a fused plan.
 
-Multi-GPU (torchrun, one rank per GPU): rows of A are dealt as contiguous panels; in the e2e
-step every rank uploads 1/world of B over its own host link and an NCCL all-gather over NVLink
-assembles B on every GPU; each rank's nnz is all-gathered for the global row_ptr base; every rank
-drains its own rows of C.  Total work is fixed -> scaling "strong".
+  value  operands resident in HBM when the timed region starts (device operands);
+  e2e    the same through the public API with HOST operands: the H2D of A (= B) from pinned host
+         memory and the D2H of every chunk of C are inside the timed region.
+
+Multi-GPU (torchrun, one rank per GPU, NCCL): rows of A are dealt as contiguous panels balanced by
+intermediate products (each rank counts 1/N of the rows with the library's count kernel, one
+all_gather gives everyone the same cuts); every rank drains its own chunks over its own host link;
+in the e2e step every rank uploads 1/N of B and an NCCL all-gather over NVLink assembles B.  Total
+work is fixed -> scaling "strong".
 
 --impl reference runs the CPU oracle (the reference arm of this tier) on bounded samples.
 """
 from __future__ import annotations
 
 import argparse
+import hashlib
 import json
 import os
+import re
 import subprocess
 import sys
 import threading
@@ -45,12 +55,16 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", type=int, default=1, help="BASELINE.json configs index (1 = 27-pt 128^3, 2 GiB)")
+    ap.add_argument("--config", type=int, default=2, help="BASELINE.json configs index (2 = R-MAT s22, C = A*A)")
     ap.add_argument("--n", type=int, default=128, help="stencil edge for config 1")
-    ap.add_argument("--ring", type=int, default=2)
+    ap.add_argument("--scale", type=int, default=0, help="R-MAT scale override for configs 2/3 (tests)")
+    ap.add_argument("--ring", type=int, default=3)
+    ap.add_argument("--chunk-nnz", type=int, default=200_000_000,
+                    help="sink mode: nonzeros per output chunk (pinned staging = ring x 12 B x this)")
+    ap.add_argument("--e2e-steps", type=int, default=0, help="e2e steps (0 = --steps)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--two-phase", action="store_true", help="time the two-phase plan/execute path at N = 1")
+    ap.add_argument("--two-phase", action="store_true", help="time the two-phase plan/execute path")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"])
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     return ap.parse_args()
@@ -70,7 +84,7 @@ class Clocks:
             return self
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
-                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
                                       stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -94,31 +108,29 @@ class Clocks:
     def summary(self):
         if not self.rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
-        sm = [float(r[1]) for r in self.rows if len(r) > 8 and r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in self.rows if len(r) > 8 and r[2].replace(".", "").isdigit()]
+        ok = [r for r in self.rows if len(r) > 8 and r[1].replace(".", "").isdigit()]
+        sm = [float(r[1]) for r in ok]
+        mx = [float(r[2]) for r in ok if r[2].replace(".", "").isdigit()]
+        pw = [float(r[3]) for r in ok if r[3].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = set()
-        for r in self.rows:
-            if len(r) > 8:
-                for k, nm in enumerate(names):
-                    if r[5 + k].lower().startswith("active"):
-                        reasons.add(nm)
+        for r in ok:
+            for k, nm in enumerate(names):
+                if r[5 + k].lower().startswith("active"):
+                    reasons.add(nm)
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(self.rows)}
+                "reasons": sorted(reasons), "samples": len(self.rows),
+                "power_w_median": float(np.median(pw)) if pw else None}
 
 
-def probe_d2h(h_dsts, dev, reps=2):
-    """This box's pinned D2H rate (GB/s) for exactly this step's output, measured in this process
-    just before the timed region: plain copy-engine copies from HBM into the bench's own pinned
-    output buffers (all of them, whole), best of `reps`, CUDA events on a side stream.  The link
-    bound of the step is judged against it (a 1 GiB copy into one buffer reads up to ~10 % faster
-    than the sustained rate into all of the step's host memory on some boxes)."""
+def probe_d2h(nbytes, dev, reps=2):
+    """This box's pinned D2H rate (GB/s), measured in this process just before the timed region:
+    copy-engine copies of `nbytes` (one output chunk's size) from HBM into a pinned buffer, best of
+    `reps`, CUDA events on a side stream.  The step's link bound is judged against it."""
     import torch
-    hbs = [h.view(torch.uint8) for h in h_dsts if h.numel() > 0]
-    total = sum(h.numel() for h in hbs)
-    if total < (1 << 20):
-        return None
-    src = torch.empty(max(h.numel() for h in hbs), dtype=torch.uint8, device=dev)
+    nbytes = int(min(max(nbytes, 1 << 20), 4 << 30))
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    src = torch.empty(nbytes, dtype=torch.uint8, device=dev)
     src.fill_(7)
     s = torch.cuda.Stream(device=dev)
     best = None
@@ -127,14 +139,13 @@ def probe_d2h(h_dsts, dev, reps=2):
         e1 = torch.cuda.Event(enable_timing=True)
         with torch.cuda.stream(s):
             e0.record(s)
-            for h in hbs:
-                h.copy_(src[:h.numel()], non_blocking=True)
+            h.copy_(src, non_blocking=True)
             e1.record(s)
         s.synchronize()
         t = e0.elapsed_time(e1) / 1e3
         best = t if best is None else min(best, t)
-    del src
-    return total / best / 1e9
+    del src, h
+    return nbytes / best / 1e9
 
 
 def d2h_detail(tl, d2h_bytes):
@@ -161,39 +172,100 @@ def dist_env():
     return world, rank, local
 
 
-def load_config(args):
-    if args.config == 1:
+def load_config(args, gpu_gen=False):
+    """(A, B, budget, name, sink): sink = True when C does not fit host memory (configs 2-4)."""
+    c = args.config
+    if c == 1:
         A = W.stencil_3d27(args.n)
-        return A, A, BUDGET_C2, f"C2: 3-D 27-point stencil {args.n}^3, C=A*A, device budget 2 GiB (out-of-core)"
-    A, B, budget, name = W.config(args.config)
-    return A, B, budget or 0, name
+        return A, A, BUDGET_C2, f"C2: 3-D 27-point stencil {args.n}^3, C=A*A, device budget 2 GiB (out-of-core)", False
+    if c in (2, 3):
+        scale = args.scale or (22 if c == 2 else 24)
+        seed = 20210517 if c == 2 else 20210518
+        A = W.rmat_torch(scale, 16, seed=seed) if gpu_gen else W.rmat(scale, 16, seed=seed)
+        gen = "torch Philox on the GPU" if gpu_gen else "numpy PCG64"
+        return A, A, 0, (f"C{c + 1}: R-MAT scale {scale} ef16 (0.45,0.2,0.2,0.15), symmetric, C=A*A through the "
+                         f"sink ({gen} generator, seed {seed})"), True
+    if c == 4:
+        if gpu_gen:
+            A = W.rmat_torch(24, col_scale=22, nedges=1 << 28, seed=11, symmetric=False)
+            B = W.rmat_torch(22, col_scale=24, nedges=1 << 28, seed=12, symmetric=False)
+        else:
+            A = W.rmat_rect(24, 22, 1 << 28, seed=11)
+            B = W.rmat_rect(22, 24, 1 << 28, seed=12)
+        return A, B, 0, "C5: rect power-law A (2^24 x 2^22) x B (2^22 x 2^24), through the sink", True
+    A, B, budget, name = W.config(c)
+    return A, B, budget or 0, name, False
 
 
-def launch_bytes(A, B, rows, offs, r0, kind):
-    """Bytes of each numeric ("num") or symbolic ("sym") launch (one per analysis unit), two ways
-    (DESIGN.md §7 "Roofline"):
-      algorithmic  SURVEY §8(a) S4/S6's per-unit figures, i.e. what Gustavson's row-by-row
-                   formulation (Alg. 1) reads and writes: the A panel (row_ptr + col
-                   [+ val]), one B entry per intermediate product (col [+ val]: 4 or 12 B), the
-                   B row_ptr pair per A entry, and the unit's output (C col + val, or nnz per row);
-      compulsory   every byte touched once: the A panel, each B row the panel touches read ONCE,
-                   the output once -- the floor the L2 (126 MB) makes reachable.
-    Returns (algorithmic list, compulsory list)."""
-    bl = np.diff(B.row_ptr)
-    vb = 12.0 if kind == "num" else 4.0
-    alg, comp = [], []
-    for c in range(len(rows) - 1):
-        a0, a1 = r0 + rows[c], r0 + rows[c + 1]
-        p0, p1 = int(A.row_ptr[a0]), int(A.row_ptr[a1])
-        cols = A.col[p0:p1]
-        touched = np.unique(cols)
-        nr, na = a1 - a0, p1 - p0
-        prods = float(bl[cols].sum())
-        out = 12.0 * float(offs[c + 1] - offs[c]) if kind == "num" else 4.0 * nr
-        a_b = 8.0 * (nr + 1) + (12.0 if kind == "num" else 4.0) * na + 8.0 * nr  # + C row offsets / bounds
-        alg.append(a_b + 16.0 * na + vb * prods + out)
-        comp.append(a_b + 16.0 * len(touched) + vb * float(bl[touched].sum()) + out)
-    return alg, comp
+def tier_constants():
+    """Tier thresholds of the kernels (csrc/internal.h), for the per-launch byte accounting."""
+    txt = open(os.path.join(ROOT, "paper_conf_ipps_xia0ar21_b200", "csrc", "internal.h")).read()
+    out = {}
+    for k in ("CAPW_SYM", "CAPW_NUM", "CAPB_SYM", "CAPB_NUM", "PIECE_SYM", "PIECE_NUM", "CURSOR_MAX", "CAPM_SYM",
+              "CAPM_NUM"):
+        m = re.search(rf"\b{k}\s*=\s*(\d+)", txt)
+        if m:
+            out[k] = int(m.group(1))
+    out["CAPS_SYM"] = 32 * out["PIECE_SYM"]
+    out["CAPS_NUM"] = 32 * out["PIECE_NUM"]
+    return out
+
+
+def source_digest():
+    """Digest of the kernel sources: a committed ncu counter is reported only for the code it was
+    measured on."""
+    h = hashlib.sha256()
+    for f in ("kernels.cu", "internal.h"):
+        h.update(open(os.path.join(ROOT, "paper_conf_ipps_xia0ar21_b200", "csrc", f), "rb").read())
+    return h.hexdigest()[:16]
+
+
+def row_products_np(A, B):
+    """u_i = sum over A's row i of nnz(B_k*) (bench bookkeeping with numpy, not the oracle)."""
+    bl = np.diff(B.row_ptr).astype(np.int64)
+    deg = np.diff(A.row_ptr)
+    if A.nnz == 0:
+        return np.zeros(A.nrows, np.int64)
+    u = np.add.reduceat(bl[A.col], np.minimum(A.row_ptr[:-1], A.nnz - 1))
+    u[deg == 0] = 0
+    return u
+
+
+def tier_bytes(A, u, nnz_rows, r0, r1, info, kind):
+    """Algorithmic bytes of the step per kernel class: Gustavson's row-by-row
+    formulation (Alg. 1) reads per row its A entries (col [+ val]) and row_ptr pair, the
+    B row_ptr pair of every A entry, one B entry per intermediate product (col + val = 12 B numeric,
+    col = 4 B symbolic), and writes its output (12 B per C nonzero, or 4 B of nnz).  Rows are
+    assigned to the tier the kernels assign them (the thresholds of csrc/internal.h)."""
+    T = tier_constants()
+    deg = np.diff(A.row_ptr[r0:r1 + 1]).astype(np.float64)
+    uu = u[r0:r1].astype(np.float64)
+    maxdeg = int(deg.max()) if len(deg) else 0
+    curstride = (min(max(maxdeg, 1), T["CURSOR_MAX"]) + 31) & ~31
+    if kind == "num":
+        n = nnz_rows.astype(np.float64)
+        per = 16.0 + 28.0 * deg + 12.0 * uu + 12.0 * n
+        capw, capb, caps = T["CAPW_NUM"], T["CAPB_NUM"], T["CAPS_NUM"]
+        key = n
+    else:
+        b = np.minimum(uu, A.ncols)
+        per = 20.0 + 20.0 * deg + 4.0 * uu
+        capw, capb, caps = T["CAPW_SYM"], T["CAPB_SYM"], T["CAPS_SYM"]
+        key = b
+    w = (key > 0) & (key <= capw)
+    big = key > capw
+    blk = big & ((key <= capb) | ((key <= caps) & (deg <= curstride)))
+    g = big & ~blk
+    out = {}
+    for name, m in (("w", w), ("b", blk), ("g", g)):
+        out[f"{kind}_{name}"] = {"bytes": float(per[m].sum()), "rows": int(m.sum()), "products": float(uu[m].sum())}
+    capm = T.get("CAPM_NUM" if kind == "num" else "CAPM_SYM")
+    if capm:  # medium CTA tier (csrc/internal.h): part of the "b" rows
+        mm = blk & (key <= capm)
+        out[f"{kind}_m"] = {"bytes": float(per[mm].sum()), "rows": int(mm.sum()), "products": float(uu[mm].sum())}
+        out[f"{kind}_b"] = {"bytes": float(per[blk & ~mm].sum()), "rows": int((blk & ~mm).sum()),
+                            "products": float(uu[blk & ~mm].sum())}
+    return out
 
 
 # ---------------------------------------------------------------------------------------- reference
@@ -228,7 +300,13 @@ def run_reference(args):
     world, rank, _ = dist_env()
     if rank != 0:
         return
-    A, B, budget, name = load_config(args)
+    gpu_gen = False
+    try:
+        import torch
+        gpu_gen = torch.cuda.is_available()  # the same matrix as our arm (torch generator on the GPU)
+    except Exception:  # noqa: BLE001
+        pass
+    A, B, budget, name, _ = load_config(args, gpu_gen=gpu_gen)
     import oracle
     th = oracle.default_threads()
     per = max(2.0, min(args.cpu_seconds, 150.0 / max(1, args.steps + args.warmup)))
@@ -254,6 +332,58 @@ def run_reference(args):
 
 # ---------------------------------------------------------------------------------------- ours
 
+class SinkOut:
+    """C larger than host memory: every output chunk lands in the library's pinned staging ring and
+    is handed to this sink, which drops it (or, in the capture step, keeps per-row nnz and the
+    sampled rows for the parity check)."""
+
+    def __init__(self, r0, r1, sample_rows):
+        self.r0, self.r1 = r0, r1
+        self.sample = set(int(x) for x in sample_rows)
+        self.capture = False
+        self.nnz = 0
+        self.rownnz = None
+        self.kept = {}
+
+    def cb(self, ra, rb, rp, col, val):
+        self.nnz += int(rp[-1])
+        if self.capture:
+            self.rownnz[ra - self.r0:rb - self.r0] = np.diff(rp)
+            for r in [x for x in self.sample if ra <= x < rb]:
+                k = r - ra
+                self.kept[r] = (col[rp[k]:rp[k + 1]].copy(), val[rp[k]:rp[k + 1]].copy())
+        return 0
+
+    def run(self, P, capture=False):
+        self.nnz = 0
+        self.capture = capture
+        if capture:
+            self.rownnz = np.zeros(self.r1 - self.r0, dtype=np.int64)
+            self.kept = {}
+        P.execute_stream(self.cb)
+        return self.nnz
+
+
+class HostOut:
+    """C fits host memory (C1, C2): the rank's slice goes to pinned host arrays."""
+
+    def __init__(self, rows, nnz):
+        import torch
+        t0 = time.perf_counter()
+        self.rp = torch.empty(rows + 1, dtype=torch.int64, pin_memory=True)
+        self.col = torch.empty(nnz, dtype=torch.int32, pin_memory=True)
+        self.val = torch.empty(nnz, dtype=torch.float64, pin_memory=True)
+        self.pin_s = time.perf_counter() - t0
+        self.cap = nnz
+        self.rownnz = None
+
+    def run(self, P, capture=False):
+        z = P.execute_capacity(self.rp, self.col, self.val, self.cap)
+        if capture:
+            self.rownnz = np.diff(self.rp.numpy())
+        return z
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -276,12 +406,12 @@ def main():
             dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group(args.dist_backend)
-
     cdev = dev if (world > 1 and args.dist_backend == "nccl") else None  # collective tensors' device
-    A, B, budget, name = load_config(args)
+
+    t_gen = time.perf_counter()
+    A, B, budget, name, sink_mode = load_config(args, gpu_gen=True)
+    gen_s = time.perf_counter() - t_gen
     same = A is B
-    panels = pdist.row_panels(A.row_ptr, world)
-    r0, r1 = panels[rank]
 
     class Dev:
         pass
@@ -292,88 +422,84 @@ def main():
         d = Dev()
         d.nrows, d.ncols = M.nrows, M.ncols
         d.store = []
-        for name, x in (("row_ptr", M.row_ptr), ("col", M.col), ("val", M.val)):
+        for nm, x in (("row_ptr", M.row_ptr), ("col", M.col), ("val", M.val)):
             t = torch.from_numpy(x)
             buf = torch.zeros(pdist.padded_len(t.numel(), world), dtype=t.dtype, device=dev)
             buf[:t.numel()].copy_(t)
             d.store.append(buf)
-            setattr(d, name, buf[:t.numel()])
+            setattr(d, nm, buf[:t.numel()])
         return d
 
     dB = to_dev(B)
     dA = dB if same else to_dev(A)
-    # the budget covers every device byte of the multiply (DESIGN.md reading R15): with resident
-    # operands the arena gets the budget minus the operands' bytes
-    in_bytes = 8 * (B.nrows + 1) + 12 * B.nnz + (0 if same else 8 * (A.nrows + 1) + 12 * A.nnz)
-    ws = torch.empty((budget - in_bytes) if budget else int(torch.cuda.mem_get_info()[0] * 0.85),
-                     dtype=torch.uint8, device=dev)
-    wbytes = ws.numel()
     stream = torch.cuda.current_stream()
 
-    # Fused plans (per-chunk symbolic overlapped with the previous chunk's D2H, the call
-    # spgemm_multiply makes).  With N > 1 ranks each rank's global row_ptr base is the sum of the
-    # earlier ranks' nnz, known after execution: an 8-byte all_gather, then spgemm_rebase_host on
-    # the rank's row_ptr slice.  --two-phase: plans whose symbolic pass runs in spgemm_plan.
-    fused = not args.two_phase
-
-    def mk_opts(profile=False, base=0):
-        return capi.opts(device=local, ring=args.ring, profile=profile, row_begin=r0, row_end=r1, workspace=ws,
-                         stream=stream.cuda_stream, row_ptr_base=base, fused=fused)
-
-    ws_e2e = None
-
-    def mk_opts_e2e():
-        # host operands: the library copies them into the arena, so the arena is the whole budget
-        nonlocal ws_e2e
-        if ws_e2e is None:
-            ws_e2e = torch.empty(wbytes + in_bytes, dtype=torch.uint8, device=dev)
-        return capi.opts(device=local, ring=args.ring, row_begin=r0, row_end=r1, workspace=ws_e2e,
-                         stream=stream.cuda_stream, fused=fused)
-
-    # untimed: sizes, global base, pinned outputs (pinning is a one-time cost, reported separately)
-    with capi.Plan(dA, dB, wbytes, capi.opts(device=local, ring=args.ring, row_begin=r0, row_end=r1, workspace=ws,
-                                             stream=stream.cuda_stream)) as P:
-        info = P.info()
-    nnz_local = info["nnz"]
-    base = 0
+    # flop-balanced row panels: each rank counts the products of 1/world of the rows with the
+    # library's count kernel (spgemm_row_products), one all_gather, identical cuts everywhere
     if world > 1:
-        base, nnz_total = pdist.slice_bases(nnz_local, device=cdev)
+        s0, s1 = pdist.even_slices(A.nrows, world)[rank]
+        u_loc, _ = capi.row_products(dA, dB, capi.opts(device=local, row_begin=s0, row_end=s1,
+                                                       stream=stream.cuda_stream))
+        u_all = pdist.allgather_rows(u_loc, A.nrows, device=cdev)
+        panels = pdist.row_panels(A.row_ptr, world, weights=u_all)
     else:
-        nnz_total = nnz_local
-    t0 = time.perf_counter()
-    h_rp = torch.empty(r1 - r0 + 1, dtype=torch.int64, pin_memory=True)
-    h_col = torch.empty(nnz_local, dtype=torch.int32, pin_memory=True)
-    h_val = torch.empty(nnz_local, dtype=torch.float64, pin_memory=True)
-    pin_s = time.perf_counter() - t0
+        panels = [(0, A.nrows)]
+    r0, r1 = panels[rank]
 
-    chunk_table = {}
+    # the budget covers every device byte of the multiply (DESIGN.md reading R15): with resident
+    # operands the arena gets the budget minus the operands' bytes; without a budget the arena is
+    # 85 % of what is free (one arena for every step: cudaMalloc of ~150 GB is not part of a multiply)
+    in_bytes = 8 * (B.nrows + 1) + 12 * B.nnz + (0 if same else 8 * (A.nrows + 1) + 12 * A.nnz)
+    if budget:
+        ws = torch.empty(budget - in_bytes, dtype=torch.uint8, device=dev)
+    else:
+        ws = torch.empty(int(torch.cuda.mem_get_info()[0] * 0.85), dtype=torch.uint8, device=dev)
+    wbytes = ws.numel()
+    fused = not args.two_phase
+    chunk_nnz = args.chunk_nnz if sink_mode else 0
+
+    def mk_opts(profile=False, base=0, workspace=None):
+        return capi.opts(device=local, ring=args.ring, profile=profile, row_begin=r0, row_end=r1,
+                         workspace=ws if workspace is None else workspace, stream=stream.cuda_stream,
+                         row_ptr_base=base, fused=fused, chunk_nnz=chunk_nnz)
+
+    # untimed: sizes (and for C2 the pinned host output, a one-time cost reported separately)
+    u_np = row_products_np(A, B)
+    products_local = int(u_np[r0:r1].sum())
+    rng = np.random.default_rng(1)
+    nloc = r1 - r0
+    sample_rows = (np.unique(np.concatenate([[r0, r1 - 1], r0 + rng.integers(0, nloc, 64)])) if nloc
+                   else np.zeros(0, np.int64))
+    if sink_mode:
+        out = SinkOut(r0, r1, sample_rows)
+        pin_s = 0.0
+    else:
+        with capi.Plan(dA, dB, wbytes, capi.opts(device=local, ring=args.ring, row_begin=r0, row_end=r1,
+                                                 workspace=ws, stream=stream.cuda_stream)) as P:
+            nnz0 = P.info()["nnz"]
+        out = HostOut(r1 - r0, nnz0)
+        pin_s = out.pin_s
 
     host_ms = {"plan": [], "execute": [], "free": []}
 
-    def step(profile=False, keep=False):
+    def step(profile=False, keep=False, capture=False):
         """One multiply (plan + execute + free).  keep: return the plan unfreed, so that its
         kernel times (CUDA events recorded inside the step) are read after the timed region."""
         h0 = time.perf_counter()
         P = capi.Plan(dA, dB, wbytes, mk_opts(profile))
         h1 = time.perf_counter()
-        if fused:
-            z = P.execute_capacity(h_rp, h_col, h_val, nnz_local)
-            if world > 1:
-                b, _ = pdist.slice_bases(z, device=cdev)
-                capi.rebase_host(h_rp, b)
-        else:
-            if world > 1:
-                b, _ = pdist.slice_bases(P.info()["nnz"], device=cdev)
-                P.set_row_ptr_base(b)
-            P.execute_into(h_rp, h_col, h_val)
+        z = out.run(P, capture)
+        if world > 1 and not sink_mode:
+            b, _ = pdist.slice_bases(z, device=cdev)
+            capi.rebase_host(out.rp, b)
         h2 = time.perf_counter()
         host_ms["plan"].append(1e3 * (h1 - h0))
         host_ms["execute"].append(1e3 * (h2 - h1))
         if keep:
-            return P
+            return P, z
         P.free()
         host_ms["free"].append(1e3 * (time.perf_counter() - h2))
-        return None
+        return None, z
 
     def barrier():
         if world > 1:
@@ -385,65 +511,74 @@ def main():
     barrier()
     for v in host_ms.values():
         v.clear()
-    link_live = probe_d2h([h_col, h_val], dev)
+    d2h_est = 12 * (args.chunk_nnz if sink_mode else out.cap)
+    link_live = probe_d2h(d2h_est, dev)
     launches0 = capi.kernel_launches()
-    stats = []
     with Clocks(local) as clk:
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         w0 = time.perf_counter()
         e0.record(stream)
         for k in range(args.steps):
-            last = step(profile=True, keep=(k == args.steps - 1))
+            last = step(profile=True, keep=(k == args.steps - 1), capture=(k == args.steps - 1))
         e1.record(stream)
         barrier()
         wall = time.perf_counter() - w0
-    # kernel times of the last timed step (its events were recorded inside the timed region)
-    stats.append(last.stats())
-    tl = capi.timeline(last)  # [chunk, 6] ms: analysis, numeric and copy start/end
-    chunk_table["rows"], chunk_table["offs"] = last.chunks()
-    chunk_table["info"] = last.info()
-    last.free()
-    nstat = len(stats)
     launches = capi.kernel_launches() - launches0
+    Pl, nnz_local = last
+    stats = Pl.stats()  # kernel times of the last timed step (events recorded inside it)
+    tl = capi.timeline(Pl)  # [chunk, 6] ms: analysis, numeric and copy start/end
+    info = Pl.info()
+    Pl.free()
     ms = e0.elapsed_time(e1)
     t_max = ms
     if world > 1:
         t = torch.tensor([ms], dtype=torch.float64, device=cdev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         t_max = float(t.item())
-    products_total = info["products"]
-    if world > 1:
-        products_total = pdist.slice_bases(info["products"], device=cdev)[1]
+        products_total = pdist.slice_bases(products_local, device=cdev)[1]
+        nnz_total = pdist.slice_bases(nnz_local, device=cdev)[1]
+        copies_total = pdist.slice_bases(info["num_copies"], device=cdev)[1]
+    else:
+        products_total, nnz_total, copies_total = products_local, nnz_local, info["num_copies"]
+    assert info["products"] == products_local, (info["products"], products_local)
     value = 2.0 * products_total * args.steps / (t_max / 1e3) / 1e9
+    # bytes each step moves to the host: C values + columns, and the row offsets (sink mode: one
+    # extra offset per output chunk, which restarts at 0)
+    d2h_bytes = 12 * nnz_total + 8 * (A.nrows + (copies_total if sink_mode else 0))
 
-    # parity spot check of the last step's output (sampled rows vs the oracle)
+    # parity spot check of the last timed step's output (sampled rows vs the oracle)
     parity = None
     if rank == 0:
         import oracle
-        rng = np.random.default_rng(1)
-        nloc = r1 - r0
-        rows = np.unique(np.concatenate([[0, nloc - 1], rng.integers(0, max(nloc, 1), 64)])) if nloc else np.zeros(0, int)
-        E = oracle.spgemm(A, B, rows=rows + r0)
-        hrp, hcol, hval = h_rp.numpy(), h_col.numpy(), h_val.numpy()
-        gp = np.concatenate([[0], np.cumsum(hrp[rows + 1] - hrp[rows])])
-        idx = np.concatenate([np.arange(hrp[r] - base, hrp[r + 1] - base) for r in rows]) if len(rows) else []
-        res = oracle.compare(gp, hcol[idx], hval[idx], E)
+        rows = sample_rows
+        E = oracle.spgemm(A, B, rows=rows)
+        if sink_mode:
+            got = [out.kept.get(int(r), (np.zeros(0, np.int32), np.zeros(0))) for r in rows]
+            gp = np.concatenate([[0], np.cumsum([len(g[0]) for g in got])])
+            gc = np.concatenate([g[0] for g in got]) if got else np.zeros(0, np.int32)
+            gv = np.concatenate([g[1] for g in got]) if got else np.zeros(0)
+            res = oracle.compare(gp, gc, gv, E)
+        else:
+            hrp, hcol, hval = out.rp.numpy(), out.col.numpy(), out.val.numpy()
+            lr = rows - r0
+            base = int(hrp[0])
+            gp = np.concatenate([[0], np.cumsum(hrp[lr + 1] - hrp[lr])])
+            idx = np.concatenate([np.arange(hrp[k] - base, hrp[k + 1] - base) for k in lr])
+            res = oracle.compare(gp, hcol[idx], hval[idx], E)
         parity = {"sampled_rows": int(len(rows)), "ok": bool(res["ok"]), "worst_ratio": res["worst_ratio"],
+                  "rule": "oracle.compare: row_ptr and col bit-identical, |c - ref| <= 1e-12 sum|a*b|",
                   "nnz_c_total_matches_closed_form": None}
         if args.config == 1:
             from tests import closed_forms as CF
             p, z = CF.c2_totals(args.n)
             parity["nnz_c_total_matches_closed_form"] = bool(z == nnz_total and p == products_total)
 
-    # roofline of the dominant kernel, from the library's CUDA events on the launching stream
-    agg = {}
-    for st in stats:
-        for k, v in st.items():
-            a = agg.setdefault(k, {"launches": 0, "ms": 0.0})
-            a["launches"] += v["launches"]
-            a["ms"] += v["ms"]
-    kern = {k: v for k, v in agg.items() if k in ("count", "sym_w", "sym_b", "sym_g", "scan", "num_w", "num_b", "num_g")}
+    # roofline of the dominant kernel: algorithmic bytes of its launches in the last timed step
+    # (per-row figures of DESIGN.md §7, rows assigned to tiers exactly as the kernels do) / its
+    # CUDA-event time on the launching stream in that step
+    kern = {k: v for k, v in stats.items()
+            if k in ("count", "sym_w", "sym_m", "sym_b", "sym_g", "scan", "num_w", "num_m", "num_b", "num_g")}
     dom = max(kern, key=lambda k: kern[k]["ms"]) if kern else None
     peaks = {}
     try:
@@ -451,45 +586,51 @@ def main():
     except Exception:  # noqa: BLE001
         pass
     hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
-    peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if "hbm_gbs" in peaks else "fallback 6.65 TB/s"
+    peak_src = ("measured: MEASURED_PEAKS.json hbm_gbs (driver-written copy bandwidth)" if "hbm_gbs" in peaks
+                else "fallback 6.65 TB/s (B200_PROFILING.md)")
     roof = None
-    if dom is not None:
-        byts = byts_c = 0.0
-        if dom[:3] in ("num", "sym"):
-            alg, comp = launch_bytes(A, B, chunk_table["rows"], chunk_table["offs"], r0, dom[:3])
-            byts, byts_c = float(np.sum(alg)) * nstat, float(np.sum(comp)) * nstat
+    if dom is not None and out.rownnz is not None:
+        tb = {}
+        tb.update(tier_bytes(A, u_np, out.rownnz, r0, r1, info, "num"))
+        tb.update(tier_bytes(A, u_np, out.rownnz, r0, r1, info, "sym"))
+        per_kernel = {}
+        for k, v in kern.items():
+            b = tb.get(k, {}).get("bytes")
+            per_kernel[k] = {"ms": round(v["ms"], 3), "launches": v["launches"],
+                             "alg_bytes": b, "GBps": (b / (v["ms"] / 1e3) / 1e9) if (b and v["ms"] > 0) else None,
+                             "rows": tb.get(k, {}).get("rows"), "products": tb.get(k, {}).get("products")}
+        byts = tb.get(dom, {}).get("bytes", 0.0)
         ms_dom = kern[dom]["ms"]
         ach = byts / (ms_dom / 1e3) / 1e9 if ms_dom > 0 else 0.0
-        ach_c = byts_c / (ms_dom / 1e3) / 1e9 if ms_dom > 0 else 0.0
         nl = max(1, kern[dom]["launches"])
         roof = {"bound": "hbm", "kernel": dom, "achieved": ach, "peak": hbm_peak, "unit": "GB/s",
                 "frac": ach / hbm_peak, "traffic": None, "peak_source": peak_src,
-                "bytes_per_launch": byts / nl,
-                "bytes_rule": "algorithmic: SURVEY S6/S4 per-unit figures (A panel, 12 B (num) / 4 B (sym) of B "
-                              "per intermediate product, B row_ptr pair per A entry, C out) -- DESIGN.md §7",
-                "achieved_compulsory": ach_c, "frac_compulsory": ach_c / hbm_peak,
-                "bytes_per_launch_compulsory": byts_c / nl,
-                "avg_launch_ms": ms_dom / max(1, kern[dom]["launches"]),
-                "share_of_step": (ms_dom / nstat) / (t_max / args.steps) if t_max else None,
-                "per_kernel_ms_per_step": {k: v["ms"] / nstat for k, v in agg.items()},
-                "kernel_times_from": "CUDA events of the last timed step (read after the timed region)"}
+                "bytes_per_launch": byts / nl, "launches": nl,
+                "avg_launch_ms": ms_dom / nl,
+                "bytes_rule": "algorithmic, per row of the tier: 16 B row offsets + 28 B per A entry (col, val, "
+                              "B row_ptr pair) + 12 B per intermediate product (B col + val) + 12 B per C "
+                              "nonzero (numeric); symbolic: 20 + 20 per A entry + 4 per product (DESIGN.md §7)",
+                "share_of_step": ms_dom / (t_max / args.steps) if t_max else None,
+                "kernel_times_from": "CUDA events on the launching stream, last timed step (read after the timed "
+                                     "region); kernels of different streams overlap",
+                "per_kernel": per_kernel}
         tf = os.path.join(ROOT, "profiles", "traffic.json")
         if os.path.exists(tf):
             try:
-                tr = json.load(open(tf)).get(dom)
-                if tr:
-                    roof["traffic"] = tr["bytes_per_launch"]
+                tr = json.load(open(tf)).get(f"{dom}@config{args.config}")
+                if tr and tr.get("source_digest") == source_digest():
+                    roof["traffic"] = tr["dram_bytes_per_launch"]
+                    roof["traffic_alg_bytes_per_launch"] = tr.get("alg_bytes_per_launch")
                     roof["traffic_source"] = tr.get("source")
-                    if "lsu_pipe_frac_of_peak" in tr:  # the unit that actually binds the hash kernels
-                        roof["binding_unit"] = {"unit": "LSU data pipe (shared memory + L1)",
-                                                "frac_of_peak": tr["lsu_pipe_frac_of_peak"],
-                                                "sm_throughput_frac": tr.get("sm_throughput_frac"),
-                                                "source": tr.get("source")}
+                    roof["binding_unit"] = tr.get("binding_unit")
+                elif tr:
+                    roof["traffic_note"] = "profiles/traffic.json entry measured on other kernel sources: not reported"
             except Exception:  # noqa: BLE001
                 pass
 
     # e2e: host operands through the public API (H2D of A=B + D2H of C inside the timed region)
     e2e = None
+    e2e_steps = args.e2e_steps or args.steps
     if not args.no_e2e:
         hA = W.CSR(A.nrows, A.ncols, torch.from_numpy(A.row_ptr).pin_memory(), torch.from_numpy(A.col).pin_memory(),
                    torch.from_numpy(A.val).pin_memory())
@@ -497,13 +638,13 @@ def main():
                                    torch.from_numpy(B.col).pin_memory(), torch.from_numpy(B.val).pin_memory())
         h2d = 8 * (B.nrows + 1) + 12 * B.nnz + (0 if same else 8 * (A.nrows + 1) + 12 * A.nnz)
 
+        # host operands at N = 1: the library copies them into its arena, so the arena is the whole
+        # budget (C2: 2 GiB = operands + the arena of the device-operand runs)
+        ws_e2e = torch.empty(wbytes + in_bytes, dtype=torch.uint8, device=dev) if (budget and world == 1) else ws
+
         def e2e_step():
             if world == 1:
-                P = capi.Plan(hA, hB, wbytes + in_bytes, mk_opts_e2e())
-                if fused:
-                    P.execute_capacity(h_rp, h_col, h_val, nnz_local)
-                    P.free()
-                    return
+                P = capi.Plan(hA, hB, ws_e2e.numel(), mk_opts(workspace=ws_e2e))
             else:
                 # B from pinned host memory: every rank uploads 1/world of each array over its own
                 # host link, an all-gather over NVLink (NCCL) assembles B on every GPU
@@ -521,24 +662,19 @@ def main():
                     dA.col[p0:p1].copy_(hA.col[p0:p1], non_blocking=True)
                     dA.val[p0:p1].copy_(hA.val[p0:p1], non_blocking=True)
                 P = capi.Plan(dA, dB, wbytes, mk_opts())
-                if fused:
-                    z = P.execute_capacity(h_rp, h_col, h_val, nnz_local)
-                    b, _ = pdist.slice_bases(z, device=cdev)
-                    capi.rebase_host(h_rp, b)
-                    P.free()
-                    return
-                b, _ = pdist.slice_bases(P.info()["nnz"], device=cdev)
-                P.set_row_ptr_base(b)
-            P.execute_into(h_rp, h_col, h_val)
+            z = out.run(P)
+            if world > 1 and not sink_mode:
+                b, _ = pdist.slice_bases(z, device=cdev)
+                capi.rebase_host(out.rp, b)
             P.free()
 
-        for _ in range(max(1, args.warmup)):
+        for _ in range(max(1, min(args.warmup, 2))):
             e2e_step()
         barrier()
         f0 = torch.cuda.Event(enable_timing=True)
         f1 = torch.cuda.Event(enable_timing=True)
         f0.record(stream)
-        for _ in range(args.steps):
+        for _ in range(e2e_steps):
             e2e_step()
         f1.record(stream)
         barrier()
@@ -547,9 +683,11 @@ def main():
             t = torch.tensor([ems], dtype=torch.float64, device=cdev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ems = float(t.item())
-        e2e = {"value": 2.0 * products_total * args.steps / (ems / 1e3) / 1e9, "unit": "GFLOP/s",
+        e2e = {"value": 2.0 * products_total * e2e_steps / (ems / 1e3) / 1e9, "unit": "GFLOP/s",
                "h2d_bytes_per_step": int(h2d),  # over all ranks (each rank uploads 1/world of B)
-               "d2h_bytes_per_step": int(12 * nnz_total + 8 * (A.nrows + 1)), "ms_per_step": ems / args.steps}
+               "d2h_bytes_per_step": int(d2h_bytes), "ms_per_step": ems / e2e_steps, "steps": e2e_steps,
+               "api": "spgemm_plan(host A, B) + spgemm_execute_stream (sink) + spgemm_free" if sink_mode
+               else "spgemm_plan(host A, B) + spgemm_execute_capacity + spgemm_free"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -557,25 +695,28 @@ def main():
         cpu = {k: c[k] for k in ("value", "unit", "cores", "kind", "sample")}
 
     if rank == 0:
-        d2h_bytes = 12 * nnz_total + 8 * (A.nrows + 1)
         link = json.load(open(os.path.join(ROOT, "profiles", "hostlink.json"))) if os.path.exists(
             os.path.join(ROOT, "profiles", "hostlink.json")) else {}
         link_gbs = float(link_live) if link_live else float(link.get("d2h_GBps", 57.2))
-        link_src = ("measured live in this run: copy-engine D2H of the step's output size into the step's own "
-                    "pinned buffers, best of 2" if link_live
-                    else "profiles/hostlink.json (another box)")
+        link_src = ("measured live in this run: copy-engine D2H of one output chunk's size into pinned memory, "
+                    "best of 2" if link_live else "profiles/hostlink.json (another box)")
         bound_ms = d2h_bytes / (link_gbs * world) / 1e6
+        in_l2 = "inputs ({:.2f} GB) and output ({:.1f} GB) larger than the 126 MB L2: no flush needed".format(
+            in_bytes / 1e9, d2h_bytes / 1e9)
         line = {
             "metric": METRIC, "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": t_max / args.steps, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": name, "budget_bytes": budget, "m": A.nrows, "nnz_A": A.nnz,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (seeded generator of BASELINE.json's configuration; DESIGN.md §5)",
+            "config": {"workload": name, "config_index": args.config, "budget_bytes": budget or wbytes,
+                       "m": A.nrows, "n": B.ncols, "nnz_A": A.nnz, "nnz_B": B.nnz,
                        "products": products_total, "nnz_C": nnz_total, "C_host_bytes": d2h_bytes,
-                       "chunks": chunk_table["info"]["num_chunks"], "output_copies": chunk_table["info"]["num_copies"],
-                       "ring": args.ring,
+                       "output": "sink (pinned staging ring, chunks dropped: C exceeds host memory)" if sink_mode
+                       else "pinned host CSR", "chunks": info["num_chunks"], "output_copies": info["num_copies"],
+                       "ring": args.ring, "chunk_nnz": chunk_nnz or None,
                        "plan": "fused (per-chunk symbolic overlapped with D2H)" if fused else "two-phase",
-                       "l2": "inputs (686 MB) and output (3.07 GB) larger than L2; no flush needed",
-                       "parallelism": f"row panels x{world}"},
+                       "l2": in_l2, "parallelism": f"row panels x{world} (flop-balanced)",
+                       "generator_s": round(gen_s, 2)},
             "gpu_launches": int(launches),
             "clocks": clk.summary(),
             "roofline": roof,
@@ -584,9 +725,12 @@ def main():
             "d2h": {"bytes_per_step": d2h_bytes, "achieved_GBps": d2h_bytes / (t_max / args.steps / 1e3) / 1e9,
                     "host_link_GBps": link_gbs, "host_link_source": link_src, "host_link_bound_ms": bound_ms,
                     "frac_of_link_bound": bound_ms / (t_max / args.steps)},
-            "d2h_detail": d2h_detail(tl, d2h_bytes),
+            "d2h_detail": d2h_detail(tl, 12 * nnz_local + 8 * (r1 - r0)),
+            "tiers": {"rows_warp": info["rows_warp"], "rows_block": info["rows_block"],
+                      "rows_global": info["rows_global"], "max_row_nnz": info["max_row_nnz"]},
             "wall_s_timed": wall,
-            "host_ms_per_step": {k: round(float(np.median(v)), 3) for k, v in host_ms.items() if v}, "pinned_output_alloc_s": pin_s,
+            "host_ms_per_step": {k: round(float(np.median(v)), 3) for k, v in host_ms.items() if v},
+            "pinned_output_alloc_s": pin_s,
             "parity": parity,
         }
         print(json.dumps(line), flush=True)

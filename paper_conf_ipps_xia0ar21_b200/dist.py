@@ -37,6 +37,29 @@ def row_panels(row_ptr: np.ndarray, world: int, weights: np.ndarray | None = Non
     return [(cuts[r], cuts[r + 1]) for r in range(world)]
 
 
+def even_slices(n: int, world: int) -> List[Tuple[int, int]]:
+    """n rows split into world near-equal contiguous ranges (who counts which rows' products)."""
+    return [((n * r) // world, (n * (r + 1)) // world) for r in range(world)]
+
+
+def allgather_rows(local, n: int, group=None, device=None) -> np.ndarray:
+    """Every rank holds `local` = an int64 value per row of its even_slices(n, world) range (e.g.
+    the products per row from the library's count kernel, spgemm_row_products); returns the whole
+    length-n array on every rank (one all_gather, NCCL over NVLink on GPUs).  Used to deal
+    flop-balanced row panels (all_gather(products), then identical cuts)."""
+    import torch
+    import torch.distributed as dist
+    world = dist.get_world_size(group)
+    sl = even_slices(n, world)
+    m = max(b - a for a, b in sl) if world else 0
+    t = torch.zeros(max(m, 1), dtype=torch.int64, device=device)
+    loc = torch.as_tensor(np.asarray(local, dtype=np.int64))
+    t[:len(loc)].copy_(loc.to(t.device))
+    out = [torch.zeros_like(t) for _ in range(world)]
+    dist.all_gather(out, t, group=group)
+    return np.concatenate([out[r][:b - a].cpu().numpy() for r, (a, b) in enumerate(sl)])
+
+
 def slice_bases(local_nnz: int, group=None, device=None) -> Tuple[int, int]:
     """All-gather every rank's nnz; returns (global row_ptr base of this rank, total nnz)."""
     import torch

@@ -9,7 +9,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 def test_reference_arm_json_line():
-    out = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--n", "24", "--steps", "2",
+    out = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--config", "1", "--n", "24", "--steps", "2",
                           "--warmup", "0", "--cpu-seconds", "0.5"], cwd=ROOT, capture_output=True, text=True,
                          timeout=600)
     assert out.returncode == 0, out.stderr[-2000:]
@@ -30,7 +30,8 @@ def test_reference_arm_under_torchrun_prints_once():
     """Under torchrun (N = 2, CPU) rank 0 alone runs the reference arm and prints one line."""
     out = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
                           "--master-addr", "127.0.0.1", "--master-port", "29571", "bench.py", "--gpus", "2",
-                          "--impl", "reference", "--steps", "1", "--warmup", "0", "--cpu-seconds", "0.3"],
+                          "--impl", "reference", "--config", "2", "--scale", "12", "--steps", "1", "--warmup", "0",
+                          "--cpu-seconds", "0.3"],
                          cwd=ROOT, capture_output=True, text=True, timeout=600)
     assert out.returncode == 0, out.stderr[-2000:]
     lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
