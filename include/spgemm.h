@@ -163,6 +163,8 @@ typedef struct {
                                 /* and leave in one copy per array (0 before the first execution)  */
     int32_t col_panels;         /* column panels of B (1 = B used whole)                            */
     int32_t reserved;
+    int64_t rows_medium;        /* rows of the medium (128-thread CTA) tier in the symbolic pass;   */
+                                /* rows_block counts the large-CTA tier only                          */
 } spgemm_info;
 
 spgemm_status spgemm_plan_info(spgemm_plan_t plan, spgemm_info *info);

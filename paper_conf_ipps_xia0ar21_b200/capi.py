@@ -55,7 +55,7 @@ class spgemm_info(ctypes.Structure):
                 ("arena_bytes", ctypes.c_int64), ("arena_used", ctypes.c_int64), ("ring_bytes", ctypes.c_int64),
                 ("rows_warp", ctypes.c_int64), ("rows_block", ctypes.c_int64), ("rows_global", ctypes.c_int64),
                 ("fused", ctypes.c_int32), ("num_copies", ctypes.c_int32),
-                ("col_panels", ctypes.c_int32), ("reserved", ctypes.c_int32)]
+                ("col_panels", ctypes.c_int32), ("reserved", ctypes.c_int32), ("rows_medium", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

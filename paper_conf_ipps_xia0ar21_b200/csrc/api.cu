@@ -210,6 +210,7 @@ SymArgs sym_args(spgemm_plan_s *P, int64_t r0, int64_t r1, int tiers) {
     sa.r0 = r0;
     sa.r1 = r1;
     sa.listB = P->listB;
+    sa.listM = P->listM;
     sa.listG = P->listG;
     sa.ctl = P->ctl;
     sa.gscratch = P->gbits_sym;
@@ -475,6 +476,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
     P->listB = P->alloc<int32_t>(R, "listB");
     P->listG = P->alloc<int32_t>(R, "listG");
     P->listBn = P->alloc<int32_t>(R, "numeric listB");
+    P->listM = P->alloc<int32_t>(R, "listM");
+    P->listMn = P->alloc<int32_t>(R, "numeric listM");
     P->listGn = P->alloc<int32_t>(R, "numeric listG");
     P->ctl = P->alloc<Ctl>(2, "ctl");
     P->tmp = P->alloc<int64_t>((R + SCAN_TILE - 1) / SCAN_TILE + 64, "scan scratch");
@@ -597,7 +600,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         CKL("symbolic");
         launch_scan(P->nnzr, R, P->crp, P->tmp, s);
         CKL("scan");
-        pe.rec(8, s);
+        pe.rec(9, s);
         int64_t total = 0;
         CK(cudaMemcpyAsync(&hc, P->ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
         CK(cudaMemcpyAsync(&total, P->crp + R, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
@@ -607,6 +610,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         P->rows_w = (int64_t)hc.rows_w;
         P->rows_b = (int64_t)hc.rows_b;
         P->rows_g = (int64_t)hc.rows_g;
+        P->rows_m = (int64_t)hc.rows_m;
         int64_t cap = ring_cap(P->max_nnz);
         cap = std::max<int64_t>(std::min<int64_t>(cap, std::max<int64_t>(total, 1)), std::max<int64_t>(P->max_nnz, 1));
         P->cap = cap;
@@ -736,19 +740,20 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         }
         P->ring_bytes = size_t(P->ring) * size_t(P->cap) * 12;
     }
-    pe.rec(9, s);
+    pe.rec(10, s);
     CK(cudaStreamSynchronize(s));
     if (P->profile) {
         P->stats.clear();
-        P->add_stat("plan_device_span", elapsed(pe.ev[0], pe.ev[9]), 0);
+        P->add_stat("plan_device_span", elapsed(pe.ev[0], pe.ev[10]), 0);
         P->add_stat("plan_upload", elapsed(pe.ev[0], pe.ev[1]), 0);  // operand H2D (host operands) + setup
         P->add_stat("count", elapsed(pe.ev[1], pe.ev[2]), 0);
-        P->add_stat("plan_cut", elapsed(pe.ev[2], pe.ev[9]), 0);     // scans, cuts, round trips, ring
+        P->add_stat("plan_cut", elapsed(pe.ev[2], pe.ev[10]), 0);    // scans, cuts, round trips, ring
         if (!P->fused) {
             P->add_stat("sym_w", elapsed(pe.ev[4], pe.ev[5]), 0);
-            P->add_stat("sym_b", elapsed(pe.ev[5], pe.ev[6]), 0);
-            P->add_stat("sym_g", elapsed(pe.ev[6], pe.ev[7]), 0);
-            P->add_stat("scan", elapsed(pe.ev[7], pe.ev[8]), 0);
+            P->add_stat("sym_m", elapsed(pe.ev[5], pe.ev[6]), 0);
+            P->add_stat("sym_b", elapsed(pe.ev[6], pe.ev[7]), 0);
+            P->add_stat("sym_g", elapsed(pe.ev[7], pe.ev[8]), 0);
+            P->add_stat("scan", elapsed(pe.ev[8], pe.ev[9]), 0);
         }
     }
 }
@@ -763,6 +768,7 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t slot_off, int64
     na.out_col = P->ring_col[b] + slot_off;
     na.out_val = P->ring_val[b] + slot_off;
     na.listB = P->listBn;
+    na.listM = P->listMn;
     na.listG = P->listGn;
     na.ctl = P->ctl + 1;
     na.gbits = P->gbits;
@@ -807,7 +813,7 @@ void enqueue_analysis(spgemm_plan_s *P, int64_t j, cudaEvent_t *ev) {
     CKL("symbolic");
     launch_scan(P->nnzr + r0, r1 - r0, P->crp + r0, P->tmp, as);
     CKL("scan");
-    if (ev) CK(cudaEventRecord(ev[4], as));
+    if (ev) CK(cudaEventRecord(ev[5], as));
     launch_publish(P->crp + r1, P->ctl, P->d_small + 1 + 2 * j, as);
     CKL("publish");
     CK(cudaEventRecord(P->ev_tot[j], as));
@@ -825,27 +831,31 @@ void finalize_profile(spgemm_plan_s *P) {
     const size_t per = P->pend.per;
     const bool overflow = P->pend.overflow;
     const int64_t total = P->pend.total;
-    P->clear_stats({"num_w", "num_b", "num_g", "d2h_span", "execute_total"});
-    if (P->fused) P->clear_stats({"sym_w", "sym_b", "sym_g", "scan"});
+    P->clear_stats({"num_w", "num_m", "num_b", "num_g", "d2h_span", "execute_total"});
+    if (P->fused) P->clear_stats({"sym_w", "sym_m", "sym_b", "sym_g", "scan"});
+    // per unit: e[0..4] symbolic tier boundaries, e[5] after the scan, e[6] numeric placement,
+    // e[7..11] numeric tier boundaries, e[12..13] copy start / end (last unit of an output chunk)
     for (int64_t c = 0; c < nch; ++c) {
         cudaEvent_t *e = ev_at(size_t(c) * per);
         if (P->fused) {
             P->add_stat("sym_w", elapsed(e[0], e[1]), 0);
-            P->add_stat("sym_b", elapsed(e[1], e[2]), 0);
-            P->add_stat("sym_g", elapsed(e[2], e[3]), 0);
-            P->add_stat("scan", elapsed(e[3], e[4]), 0);
+            P->add_stat("sym_m", elapsed(e[1], e[2]), 0);
+            P->add_stat("sym_b", elapsed(e[2], e[3]), 0);
+            P->add_stat("sym_g", elapsed(e[3], e[4]), 0);
+            P->add_stat("scan", elapsed(e[4], e[5]), 0);
         }
         if (!overflow) {
-            P->add_stat("num_w", elapsed(e[6], e[7]), 0);
-            P->add_stat("num_b", elapsed(e[7], e[8]), 0);
-            P->add_stat("num_g", elapsed(e[8], e[9]), 0);
+            P->add_stat("num_w", elapsed(e[7], e[8]), 0);
+            P->add_stat("num_m", elapsed(e[8], e[9]), 0);
+            P->add_stat("num_b", elapsed(e[9], e[10]), 0);
+            P->add_stat("num_g", elapsed(e[10], e[11]), 0);
         }
     }
     const std::vector<int64_t> &gl = P->pend.group_last;
     for (size_t g = 0; g < gl.size() && !overflow; ++g) {
         const int64_t c = gl[g];
-        cudaEvent_t end = g + 1 < gl.size() ? ev[size_t(gl[g + 1]) * per + 10] : ev[size_t(nch) * per + 1];
-        P->add_stat("d2h_span", elapsed(ev[size_t(c) * per + 10], end), double(P->pend.group_nnz[g]) * 12);
+        cudaEvent_t end = g + 1 < gl.size() ? ev[size_t(gl[g + 1]) * per + 12] : ev[size_t(nch) * per + 1];
+        P->add_stat("d2h_span", elapsed(ev[size_t(c) * per + 12], end), double(P->pend.group_nnz[g]) * 12);
     }
     P->add_stat("execute_total", elapsed(ev[size_t(nch) * per], ev[size_t(nch) * per + 1]),
                 double(total) * 12 + 8.0 * (P->R + 1));
@@ -857,17 +867,17 @@ void finalize_profile(spgemm_plan_s *P) {
         double *t = &P->timeline[size_t(c) * 6];
         if (P->fused) {
             t[0] = elapsed(t0, e[0]);
-            t[1] = elapsed(t0, e[4]);
+            t[1] = elapsed(t0, e[5]);
         }
         if (!overflow) {
-            t[2] = elapsed(t0, e[6]);
-            t[3] = elapsed(t0, e[9]);
+            t[2] = elapsed(t0, e[7]);
+            t[3] = elapsed(t0, e[11]);
         }
     }
     for (size_t g = 0; g < gl.size() && !overflow; ++g) {  // copies: on each output chunk's last unit
         const size_t c = size_t(gl[g]);
-        P->timeline[c * 6 + 4] = elapsed(t0, ev[c * per + 10]);
-        P->timeline[c * 6 + 5] = elapsed(t0, ev[c * per + 11]);
+        P->timeline[c * 6 + 4] = elapsed(t0, ev[c * per + 12]);
+        P->timeline[c * 6 + 5] = elapsed(t0, ev[c * per + 13]);
     }
 }
 
@@ -906,6 +916,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         // the symbolic passes of this execution accumulate max_nnz and the per-tier row counts
         static_assert(offsetof(Ctl, rows_g) == offsetof(Ctl, max_nnz) + 3 * sizeof(unsigned long long), "Ctl layout");
         CK(cudaMemsetAsync(&P->ctl[0].max_nnz, 0, 4 * sizeof(unsigned long long), P->astream));
+        CK(cudaMemsetAsync(&P->ctl[0].rows_m, 0, sizeof(unsigned long long), P->astream));
         P->base_applied = base;
     } else {
         if (P->base_wanted != P->base_applied) {
@@ -936,7 +947,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         return reinterpret_cast<int64_t *>((char *)stage[b] + ((size_t(maxn) * 12 + 7) & ~size_t(7)));
     };
 
-    const int per = 12;
+    const int per = 14;
     EvSet pe(P->profile, P->res, 12, size_t(nch) * per + 4);
     CK(cudaEventRecord(P->ev_ready, s));
     CK(cudaStreamWaitEvent(cp, P->ev_ready, 0));
@@ -995,7 +1006,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
     auto close_group = [&](Group &G) {  // enqueue the group's copies after its numeric passes
         CK(cudaEventRecord(P->ev_num[G.b], s));
         CK(cudaStreamWaitEvent(cp, P->ev_num[G.b], 0));
-        pe.rec(size_t(G.u1 - 1) * per + 10, cp);
+        pe.rec(size_t(G.u1 - 1) * per + 12, cp);
         int32_t *dcol = sink ? st_col(G.b) : col_out + G.off;
         double *dval = sink ? st_val(G.b) : val_out + G.off;
         if (G.nnz > 0) {
@@ -1027,7 +1038,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
             if (n > h)
                 CK(cudaMemcpyAsync(drp + h, P->crp + G.r0 + 1 + h, sizeof(int64_t) * (n - h), cudaMemcpyDeviceToHost, cp));
         }
-        pe.rec(size_t(G.u1 - 1) * per + 11, cp);
+        pe.rec(size_t(G.u1 - 1) * per + 13, cp);
         CK(cudaEventRecord(P->ev_d2h[G.b], cp));
     };
 
@@ -1084,8 +1095,8 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         if (P->fused) CK(cudaStreamWaitEvent(s, P->ev_tot[j], 0));  // (already complete: host waited)
         if (!P->chunk_wait.empty() && P->chunk_wait[j] >= 0)       // host operands: value pieces
             CK(cudaStreamWaitEvent(s, P->ev_piece[P->chunk_wait[j]], 0));
-        pe.rec(size_t(j) * per + 5, s);
-        enqueue_numeric(P, j, cur.b, cur.pad + cur.nnz, mx, pe.at(size_t(j) * per + 6));
+        pe.rec(size_t(j) * per + 6, s);
+        enqueue_numeric(P, j, cur.b, cur.pad + cur.nnz, mx, pe.at(size_t(j) * per + 7));
         cur.nnz += n;
         cur.u1 = j + 1;
         cur.r1 = r1;
@@ -1124,6 +1135,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         P->rows_w = (int64_t)hc.rows_w;
         P->rows_b = (int64_t)hc.rows_b;
         P->rows_g = (int64_t)hc.rows_g;
+        P->rows_m = (int64_t)hc.rows_m;
         if (P->host_cut) {
             P->products = (int64_t)hc.sum_u;
             P->max_u = (int64_t)hc.max_u;
@@ -1241,6 +1253,7 @@ spgemm_status spgemm_plan_info(spgemm_plan_t P, spgemm_info *info) {
     info->rows_warp = P->rows_w;
     info->rows_block = P->rows_b;
     info->rows_global = P->rows_g;
+    info->rows_medium = P->rows_m;
     info->fused = P->fused ? 1 : 0;
     info->num_copies = (int32_t)P->num_groups;
     info->col_panels = P->col_panels;

@@ -135,6 +135,7 @@ struct spgemm_plan_s {
     int64_t *bnd = nullptr, *crp = nullptr, *tmp = nullptr;
     int32_t *nnzr = nullptr, *listB = nullptr, *listG = nullptr;  // symbolic long-row lists
     int32_t *listBn = nullptr, *listGn = nullptr;                  // numeric long-row lists
+    int32_t *listM = nullptr, *listMn = nullptr;                   // medium-tier lists (sym, num)
     cudaStream_t astream = nullptr;  // fused plans: symbolic passes run here, ahead of the numeric
     cudaStream_t hstream = nullptr;         // host B: value pieces H2D
     std::vector<cudaEvent_t> ev_piece;      // one per value piece, in upload order
@@ -167,7 +168,7 @@ struct spgemm_plan_s {
     std::vector<int64_t> chunk_offs;  // num_chunks + 1 offsets relative to the slice (known after
                                       // plan for two-phase plans, after an execution for fused)
     int64_t nnz = -1, products = 0, max_nnz = 0, max_u = 0, max_bound = 0, sum_bound = 0;
-    int64_t rows_w = 0, rows_b = 0, rows_g = 0;
+    int64_t rows_w = 0, rows_b = 0, rows_g = 0, rows_m = 0;
     int64_t num_groups = 0;  // output chunks (copies) of the last execution
     int64_t panel_units = 0; // column-panel plans: numeric units (chunks C[i][j]) over all panels
     std::vector<int64_t> unit_order;  // order = 1: units by decreasing flops (empty: row order)

@@ -17,6 +17,9 @@ struct DevCSR {
 
 // Accumulator tiers.  A row is handled by
 //   W: one warp, shared-memory hash table of TW_* slots   (bound <= CAPW_*)
+//   M: one 128-thread CTA, shared-memory hash table of TM_* slots (CAPW_* < bound <= CAPM_*): the
+//      rows of a few hundred to two thousand nonzeros that dominate power-law inputs (R-MAT, C3-C5)
+//      get up to 8-11 CTAs per SM instead of the B tier's 2 (medium tier)
 //   B: one CTA,  shared-memory hash table of TB_* slots.  A row with bound <= CAPB_* is one piece;
 //      a longer one (bound <= CAPS_*) is cut into column pieces [lo, hi) processed one after the
 //      other in the same table, each A entry's B row resumed from a per-entry cursor -- the paper's
@@ -31,6 +34,9 @@ constexpr int WARPS_W = 8;                 // warps per CTA in the W kernels
 // table whose bound (products) over-estimates nnz (C2: 729 products, 125 nnz per row)
 constexpr int TW_SYM = 1024, CAPW_SYM = 768;
 constexpr int TW_NUM = 512, CAPW_NUM = 256;
+constexpr int THREADS_M = 128;             // medium tier: 16 KB (symbolic) / 24 KB (numeric) tables
+constexpr int TM_SYM = 4096, CAPM_SYM = 2048;
+constexpr int TM_NUM = 2048, CAPM_NUM = 1024;
 constexpr int THREADS_B = 512;             // 2 CTAs per SM (96 KB / 64 KB of table + 13 KB)
 constexpr int TB_SYM = 16384, CAPB_SYM = 8192;
 constexpr int TB_NUM = 8192, CAPB_NUM = 4096;
@@ -45,7 +51,7 @@ struct Ctl {
     unsigned long long row_ctr;   // W kernels: next row batch                      } reset before
     unsigned int nB, nG;          // long-row list lengths                          } every pass
     unsigned long long pass_max;  // symbolic: max nnz of a row in this pass        } (32 bytes)
-    unsigned int pad1, pad0;      //                                                }
+    unsigned int nM, pad0;        // medium-tier list length                        }
     unsigned int err;             // bit 0: numeric count mismatch; bit 1: invalid input; bit 2: table overflow
     unsigned int pad;
     unsigned long long sum_u;     // count pass: sum of products
@@ -54,7 +60,8 @@ struct Ctl {
     unsigned long long max_nnz;   // symbolic pass: max nnz in a row
     unsigned long long rows_w, rows_b, rows_g;
     unsigned long long max_deg;   // count pass: longest row of A (cursor scratch of pieced rows)
-    unsigned long long pad2[5];
+    unsigned long long rows_m;    // rows of the medium tier (symbolic passes)
+    unsigned long long pad2[4];
 };
 
 // --- launchers (all asynchronous on `s`) ---------------------------------------------------
@@ -77,6 +84,7 @@ struct SymArgs {
     int32_t *nnz;        // out: nnz of every row in [r0, r1)
     int64_t r0, r1;      // rows of this pass
     int32_t *listB, *listG;
+    int32_t *listM;      // medium tier (NULL: those rows go to the B tier)
     Ctl *ctl;
     uint32_t *gscratch;  // G tier: per-CTA bitmap of ceil(ncols/32) words, zero on entry and exit
     int64_t gstride;     // words per CTA slot
@@ -90,9 +98,17 @@ struct SymArgs {
     int batch;           // rows per claim in the W kernel (set by the launcher)
 };
 
-// tier bits for a pass whose rows have bound <= maxb
-inline int sym_tiers(int64_t maxb) { return (maxb > CAPW_SYM ? 1 : 0) | (maxb > CAPS_SYM ? 2 : 0); }
-inline int num_tiers(int64_t maxnnz) { return (maxnnz > CAPW_NUM ? 1 : 0) | (maxnnz > CAPS_NUM ? 2 : 0); }
+// the medium tier is on unless SPGEMM_NO_MEDIUM=1 (A/B knob): its rows then go to the B tier
+bool medium_enabled();
+// tier bits for a pass whose rows have bound <= maxb: 1 = B (CTA), 2 = G (dense), 4 = M (medium)
+inline int sym_tiers(int64_t maxb) {
+    const bool m = medium_enabled();
+    return (maxb > (m ? CAPM_SYM : CAPW_SYM) ? 1 : 0) | (maxb > CAPS_SYM ? 2 : 0) | (m && maxb > CAPW_SYM ? 4 : 0);
+}
+inline int num_tiers(int64_t maxnnz) {
+    const bool m = medium_enabled();
+    return (maxnnz > (m ? CAPM_NUM : CAPW_NUM) ? 1 : 0) | (maxnnz > CAPS_NUM ? 2 : 0) | (m && maxnnz > CAPW_NUM ? 4 : 0);
+}
 
 // host2[0] = *end (a chunk's end offset), host2[1] = ctl->pass_max -- zero-copy stores into mapped
 // pinned memory, so no small D2H copy queues behind the big ones on the copy engine
@@ -105,8 +121,8 @@ void launch_seg_max_col(const DevCSR &A, const int64_t *rows, int64_t nseg, int6
 void launch_seg_max(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s);
 // out[k] = sum(x[rows[k] .. rows[k+1]-1])
 void launch_seg_sum(const int64_t *x, const int64_t *rows, int64_t nseg, int64_t *out, cudaStream_t s);
-// S3+S4: symbolic pass over all rows (tiering + the three tiers).  ev: NULL or 4 events recorded
-// before W, between W/B, between B/G and after G (per-kernel timing on the launching stream).
+// S3+S4: symbolic pass over all rows (tiering + the four tiers).  ev: NULL or 5 events recorded
+// before W, between W/M, M/B, B/G and after G (per-kernel timing on the launching stream).
 void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev);
 
 // S5: y[1 + t] = y[0] + x[0] + ... + x[t] for t < n, y[0] (the base) read on the device.
@@ -129,6 +145,7 @@ struct NumArgs {
     int32_t *out_col;    // ring slot: nnz of the chunk
     double *out_val;
     int32_t *listB, *listG;
+    int32_t *listM;      // as in SymArgs
     Ctl *ctl;
     uint32_t *gbits;     // G tier scratch: per CTA gstride_bits words of bitmap ...
     double *gvals;       // ... and gstride_vals doubles, all zero on entry and exit
@@ -153,7 +170,7 @@ int choose_group(const DevCSR &B, int64_t nnzB);
 
 // occupancy-derived grid sizes (queried once per device)
 struct Grids {
-    int count_blocks, symw_blocks, numw_blocks, symb_blocks, numb_blocks;
+    int count_blocks, symw_blocks, numw_blocks, symb_blocks, numb_blocks, symm_blocks, numm_blocks;
 };
 const Grids &grids(int device, int num_sms);
 
@@ -164,6 +181,8 @@ size_t symw_smem();
 size_t numw_smem(bool wide);
 size_t symb_smem();
 size_t numb_smem();
+size_t symm_smem();
+size_t numm_smem();
 
 // --- column panels of B (NEXT-1; kernels.cu "column panels") ---------------------------------
 // hist[col >> shift] += 1 over n column ids (nbins <= 4096)

@@ -228,12 +228,14 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
 // of B row k = [s0, e0) that entry e (its index within the row) contributes: the whole row, or
 // one column piece of it (PieceSeg).
 constexpr int PBATCH = 512;
-struct ProdSmem {
-    int64_t off[PBATCH + 1];
-    int64_t bs[PBATCH];
-    double a[PBATCH];
+template <int PB>
+struct ProdSmemT {
+    int64_t off[PB + 1];
+    int64_t bs[PB];
+    double a[PB];
     int64_t scan[40];
 };
+using ProdSmem = ProdSmemT<PBATCH>;
 
 struct WholeSeg {
     __device__ __forceinline__ void operator()(int, int32_t, int64_t s0, int64_t e0, int64_t &s, int64_t &en) const {
@@ -264,13 +266,14 @@ struct PieceSeg {
     }
 };
 
-template <int NT, bool VALS, typename SEG, typename F>
-__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmem &sm,
+template <int NT, bool VALS, int PB, typename SEG, typename F>
+__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
                                                    const SEG &seg, F &&f) {
-    constexpr int PER = PBATCH / NT;
+    constexpr int PER = PB / NT;
+    static_assert(PER * NT == PB, "batch must be a multiple of the CTA size");
     const int64_t as = A.rp[i], ae = A.rp[i + 1];
-    for (int64_t pb = as; pb < ae; pb += PBATCH) {
-        const int nb = (int)(ae - pb < PBATCH ? ae - pb : PBATCH);
+    for (int64_t pb = as; pb < ae; pb += PB) {
+        const int nb = (int)(ae - pb < PB ? ae - pb : PB);
         int64_t lens[PER];
         int64_t sum = 0;
 #pragma unroll
@@ -286,7 +289,7 @@ __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR
                 len = en - s;
                 if (VALS) av = __ldg(&A.val[pb + e]);
             }
-            if (e < PBATCH) {
+            if (e < PB) {
                 sm.bs[e] = bs;
                 if (VALS) sm.a[e] = av;
             }
@@ -335,8 +338,9 @@ __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR
     }
 }
 
-template <int NT, bool VALS, typename F>
-__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmem &sm, F &&f) {
+template <int NT, bool VALS, int PB, typename F>
+__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
+                                                   F &&f) {
     block_row_products<NT, VALS>(A, B, i, sm, WholeSeg{}, f);
 }
 
@@ -511,11 +515,17 @@ __global__ void k_add(int64_t *rp, int64_t n, int64_t d) {
 
 // ------------------------------------------------------------------------ tier classification
 
-// rows too long for a warp: the CTA tier (one piece up to capB; column pieces up to capS when the
-// pass has cursor scratch and the row's A entries fit it), the dense tier beyond
-__device__ __forceinline__ void push_long(int64_t i, int64_t bound, const DevCSR &A, int64_t capB, int64_t capS,
-                                          const int32_t *cursor, int64_t curstride, int32_t *listB, int32_t *listG,
-                                          Ctl *ctl) {
+// rows too long for a warp: the medium tier (bound <= capM, when enabled), the CTA tier (one piece
+// up to capB; column pieces up to capS when the pass has cursor scratch and the row's A entries
+// fit it), the dense tier beyond
+__device__ __forceinline__ void push_long(int64_t i, int64_t bound, const DevCSR &A, int64_t capM, int64_t capB,
+                                          int64_t capS, const int32_t *cursor, int64_t curstride, int32_t *listM,
+                                          int32_t *listB, int32_t *listG, Ctl *ctl) {
+    if (listM != nullptr && bound <= capM) {
+        unsigned idx = atomicAdd(&ctl->nM, 1u);
+        listM[idx] = (int32_t)i;
+        return;
+    }
     const bool pieces_ok = cursor != nullptr && bound <= capS && A.rp[i + 1] - A.rp[i] <= curstride;
     if (bound <= capB || pieces_ok) {
         unsigned idx = atomicAdd(&ctl->nB, 1u);
@@ -556,7 +566,8 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
             }
             if (bound > CAPW_SYM) {
                 if (lane == 0) {
-                    push_long(i, bound, a.A, CAPB_SYM, CAPS_SYM, a.cursor, a.curstride, a.listB, a.listG, a.ctl);
+                    push_long(i, bound, a.A, CAPM_SYM, CAPB_SYM, CAPS_SYM, a.cursor, a.curstride, a.listM, a.listB,
+                              a.listG, a.ctl);
                     nlong++;
                 }
                 continue;
@@ -729,6 +740,49 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
             atomicAdd(&a.ctl->rows_b, 1ull);
         }
         __syncthreads();
+    }
+}
+
+// ----------------------------------------------------------------------------- S4 symbolic, M
+//
+// Rows whose bound exceeds a warp's table but fits a TM_SYM table at load <= 1/2: one 128-thread CTA
+// per row with a 16 KB table, so that ~11 rows are in flight per SM instead of the B tier's 2 (on
+// R-MAT most long rows have a few hundred to two thousand products).  The same
+// flattened, load-balanced product iterator as the B tier, with a 128-entry A batch; fresh keys
+// are counted per thread (sym_insert's return) and reduced once per row.
+constexpr int PBATCH_M = THREADS_M;
+
+__global__ void __launch_bounds__(THREADS_M) k_sym_m(SymArgs a) {
+    extern __shared__ __align__(16) int32_t keys[];
+    __shared__ ProdSmemT<PBATCH_M> psm;
+    __shared__ int s_cnt;
+    constexpr int MAXLG = 12;  // log2(TM_SYM)
+    static_assert((1 << MAXLG) == TM_SYM, "table size");
+    const unsigned n = *(volatile unsigned *)&a.ctl->nM;
+    unsigned long long lmax = 0, nrow = 0;
+    for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
+        const int64_t i = a.listM[idx];
+        const int lg = table_log2(a.bnd[i], MAXLG);
+        const int T = 1 << lg;
+        for (int t = threadIdx.x; t < T; t += THREADS_M) keys[t] = EMPTY;
+        if (threadIdx.x == 0) s_cnt = 0;
+        __syncthreads();
+        int cnt = 0;
+        block_row_products<THREADS_M, false>(a.A, a.B, i, psm,
+                                             [&](int32_t c, double) { cnt += sym_insert(keys, c, lg); });
+        cnt = warp_sum(cnt);  // (block_row_products ended with a barrier: every insert is done)
+        if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(&s_cnt, cnt);
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            a.nnz[i] = s_cnt;
+            lmax = max(lmax, (unsigned long long)s_cnt);
+            nrow++;
+        }
+    }
+    if (threadIdx.x == 0 && nrow) {
+        atomicMax(&a.ctl->max_nnz, lmax);
+        atomicMax(&a.ctl->pass_max, lmax);
+        atomicAdd(&a.ctl->rows_m, nrow);
     }
 }
 
@@ -998,7 +1052,9 @@ __global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
             const int64_t n = a.crp[i + 1] - o;
             if (n == 0) continue;
             if (n > CAPW_NUM) {
-                if (lane == 0) push_long(i, n, a.A, CAPB_NUM, CAPS_NUM, a.cursor, a.curstride, a.listB, a.listG, a.ctl);
+                if (lane == 0)
+                    push_long(i, n, a.A, CAPM_NUM, CAPB_NUM, CAPS_NUM, a.cursor, a.curstride, a.listM, a.listB, a.listG,
+                              a.ctl);
                 continue;
             }
             const int lg = table_log2(a.tload == 0 ? n : a.tload == 1 ? (3 * n) / 2 : 2 * n, MAXLG);
@@ -1097,21 +1153,26 @@ __global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
 
 // ------------------------------------------------------------------------------ S6 numeric, B
 
-struct CtaSortSmem {
-    int cnt[64], cur[64], start[64], mm[3], occ[THREADS_B / 32];
+template <int NT>
+struct CtaSortSmemT {
+    int cnt[64], cur[64], start[64], mm[3], occ[NT / 32];
     int64_t scan[40];
 };
+using CtaSortSmem = CtaSortSmemT<THREADS_B>;
 
-// fine-bucket counters of the CTA sort; they alias the product iterator's ProdSmem (not in use
-// while a table is sorted)
-constexpr int SORT_PMAX = 1024;
-struct SortCnt {
-    int cnt[SORT_PMAX], cur[SORT_PMAX], start[SORT_PMAX];
+// fine-bucket counters of the CTA sort (2 per thread: the bucket scan gives each thread two); they
+// alias the product iterator's ProdSmem (not in use while a table is sorted)
+template <int NT>
+struct SortCntT {
+    int cnt[2 * NT], cur[2 * NT], start[2 * NT];
 };
-union ProdOrSort {
-    ProdSmem psm;
-    SortCnt sc;
+using SortCnt = SortCntT<THREADS_B>;
+template <int NT, int PB>
+union ProdOrSortT {
+    ProdSmemT<PB> psm;
+    SortCntT<NT> sc;
 };
+using ProdOrSort = ProdOrSortT<THREADS_B, PBATCH>;
 
 template <typename T>
 __device__ __forceinline__ T warp_incl_scan(T x) {
@@ -1130,14 +1191,16 @@ __device__ __forceinline__ T warp_incl_scan(T x) {
 // clustered columns) takes the general path: compaction + shared-memory bitonic.  Writes oc/ov
 // [0, n); returns false (nothing written) if the table does not hold exactly n keys.  All
 // threads call; ends with a barrier.
-template <int SB>
+template <int SB, int NT = THREADS_B>
 __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int32_t *oc, double *ov,
-                              CtaSortSmem &ss, SortCnt &sc) {
+                              CtaSortSmemT<NT> &ss, SortCntT<NT> &sc) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    constexpr int NW = THREADS_B / 32;
+    constexpr int NW = NT / 32;
+    constexpr int PLMAX = NT == 512 ? 10 : NT == 256 ? 9 : NT == 128 ? 8 : 7;  // 2^PLMAX = 2 NT buckets
+    static_assert((1 << PLMAX) == 2 * NT, "two fine buckets per thread");
     // fine buckets (~4 keys each): 2^pl of them, bucket of key k = (k - lo) >> sh
-    const int pl = min(10, max(5, 32 - __clz((int)max((int64_t)1, (n + 3) / 4) - 1)));
-    for (int b = threadIdx.x; b < (1 << pl); b += THREADS_B) sc.cnt[b] = 0;
+    const int pl = min(PLMAX, max(5, 32 - __clz((int)max((int64_t)1, (n + 3) / 4) - 1)));
+    for (int b = threadIdx.x; b < (1 << pl); b += NT) sc.cnt[b] = 0;
     const int P = min(64, max(1, (int)((n + 255) / 256)));
     if (threadIdx.x < 64) ss.cnt[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
@@ -1147,7 +1210,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     __syncthreads();
     {
         int lmin = INT_MAX, lmax = -1, occ = 0;
-        for (int t = threadIdx.x; t < T; t += THREADS_B) {
+        for (int t = threadIdx.x; t < T; t += NT) {
             const int32_t k = keys[t];
             if (k != EMPTY) {
                 lmin = min(lmin, k);
@@ -1182,7 +1245,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         // number of smaller keys in its bucket.  ~4 compares per key instead of a bitonic network.
         const int lspan = 64 - __clzll(span - 1);  // 2^lspan >= span
         const int sh = max(0, lspan - pl);
-        for (int t = threadIdx.x; t < T; t += THREADS_B) {
+        for (int t = threadIdx.x; t < T; t += NT) {
             const int32_t k = keys[t];
             if (k != EMPTY) atomicAdd(&sc.cnt[(int)(((int64_t)k - lo) >> sh)], 1);
         }
@@ -1191,7 +1254,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         const int b0 = 2 * threadIdx.x;
         const int c0 = b0 < nb ? sc.cnt[b0] : 0, c1 = b0 + 1 < nb ? sc.cnt[b0 + 1] : 0;
         int64_t tot;
-        const int64_t ex = block_excl_scan<THREADS_B>(c0 + c1, ss.scan, &tot);  // ends with a barrier
+        const int64_t ex = block_excl_scan<NT>(c0 + c1, ss.scan, &tot);  // ends with a barrier
         if (b0 < nb) sc.start[b0] = sc.cur[b0] = (int)ex;
         if (b0 + 1 < nb) sc.start[b0 + 1] = sc.cur[b0 + 1] = (int)ex + c0;
         int big = max(c0, c1);
@@ -1203,7 +1266,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
 #pragma unroll
         for (int w = 0; w < NW; ++w) bmax = max(bmax, ss.occ[w]);
         if (bmax <= 64) {
-            for (int t = threadIdx.x; t < T; t += THREADS_B) {  // stage; keys[t] := staged position
+            for (int t = threadIdx.x; t < T; t += NT) {  // stage; keys[t] := staged position
                 const int32_t k = keys[t];
                 if (k != EMPTY) {
                     const int pos = atomicAdd(&sc.cur[(int)(((int64_t)k - lo) >> sh)], 1);
@@ -1212,7 +1275,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
                 }
             }
             __syncthreads();
-            for (int t = threadIdx.x; t < T; t += THREADS_B) {  // rank; value out; key parked in vals[t]
+            for (int t = threadIdx.x; t < T; t += NT) {  // rank; value out; key parked in vals[t]
                 const int pos = keys[t];
                 if (pos != EMPTY) {
                     const int32_t k = oc[pos];
@@ -1230,7 +1293,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
                 }
             }
             __syncthreads();
-            for (int t = threadIdx.x; t < T; t += THREADS_B) {  // columns
+            for (int t = threadIdx.x; t < T; t += NT) {  // columns
                 const int r = keys[t];
                 if (r != EMPTY) oc[r] = reinterpret_cast<const int32_t *>(vals + t)[0];
             }
@@ -1239,7 +1302,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         }
     }
     // skewed columns (a fine bucket over 64 keys): coarse buckets sorted by warps in registers
-    for (int t = threadIdx.x; t < T; t += THREADS_B) {
+    for (int t = threadIdx.x; t < T; t += NT) {
         const int32_t k = keys[t];
         if (k != EMPTY) atomicAdd(&ss.cnt[(int)(((int64_t)k - lo) * P / span)], 1);
     }
@@ -1258,7 +1321,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     __syncthreads();
     if (ss.mm[2] <= 512) {
         unsigned long long *stage = reinterpret_cast<unsigned long long *>(ov);
-        for (int t = threadIdx.x; t < T; t += THREADS_B) {
+        for (int t = threadIdx.x; t < T; t += NT) {
             const int32_t k = keys[t];
             if (k != EMPTY) {
                 const int pos = atomicAdd(&ss.cur[(int)(((int64_t)k - lo) * P / span)], 1);
@@ -1276,13 +1339,13 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     }
     // general path: in-place compaction + shared-memory bitonic sort
     int64_t cnt = 0;
-    for (int t0 = 0; t0 < T; t0 += THREADS_B) {
+    for (int t0 = 0; t0 < T; t0 += NT) {
         const int t = t0 + threadIdx.x;
         const int32_t k = t < T ? keys[t] : EMPTY;
         const double v = t < T ? vals[t] : 0.0;
         const int occ = k != EMPTY;
         int64_t tot;
-        const int64_t ex = block_excl_scan<THREADS_B>(occ, ss.scan, &tot);  // ends with a barrier
+        const int64_t ex = block_excl_scan<NT>(occ, ss.scan, &tot);  // ends with a barrier
         if (occ) {
             keys[cnt + ex] = k;
             vals[cnt + ex] = v;
@@ -1291,10 +1354,10 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         __syncthreads();
     }
     const int N = pow2_at_least(n, 32);
-    for (int t = (int)n + threadIdx.x; t < N; t += THREADS_B) keys[t] = INT_MAX;
+    for (int t = (int)n + threadIdx.x; t < N; t += NT) keys[t] = INT_MAX;
     __syncthreads();
-    block_bitonic<THREADS_B>(keys, vals, N);
-    for (int t = threadIdx.x; t < n; t += THREADS_B) {
+    block_bitonic<NT>(keys, vals, N);
+    for (int t = threadIdx.x; t < n; t += NT) {
         oc[t] = keys[t];
         ov[t] = vals[t];
     }
@@ -1362,6 +1425,41 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
     }
 }
 
+// ------------------------------------------------------------------------------ S6 numeric, M
+// One 128-thread CTA per row of CAPW_NUM < nnz <= CAPM_NUM (24 KB table: ~8 rows in flight per SM),
+// the B tier's product iterator and bucket sort at 128 threads.
+
+__global__ void __launch_bounds__(THREADS_M) k_num_m(NumArgs a) {
+    extern __shared__ __align__(16) double smem_d[];
+    double *vals = smem_d;
+    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TM_NUM);
+    __shared__ ProdOrSortT<THREADS_M, PBATCH_M> u;
+    __shared__ CtaSortSmemT<THREADS_M> ss;
+    constexpr int MAXLG = 11;  // log2(TM_NUM)
+    static_assert((1 << MAXLG) == TM_NUM, "table size");
+    const unsigned nrows = *(volatile unsigned *)&a.ctl->nM;
+    const int64_t off0 = a.crp[a.r0];
+    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
+        const int64_t i = a.listM[idx];
+        const int64_t o = a.crp[i];
+        const int64_t n = a.crp[i + 1] - o;
+        const int lg = table_log2(n, MAXLG);
+        const int T = 1 << lg;
+        for (int t = threadIdx.x; t < T; t += THREADS_M) {
+            keys[t] = EMPTY;
+            vals[t] = 0.0;
+        }
+        __syncthreads();
+        block_row_products<THREADS_M, true>(a.A, a.B, i, u.psm, [&](int32_t c, double v) {
+            atomicAdd(&vals[find_slot(keys, c, lg)], v);
+        });  // ends with a barrier
+        const bool ok = cta_sort_emit<MAXLG, THREADS_M>(keys, vals, T, n, a.out_col + (o - off0),
+                                                        a.out_val + (o - off0), ss, u.sc);
+        if (!ok && threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
+        __syncthreads();
+    }
+}
+
 // ------------------------------------------------------------------------------ S6 numeric, G
 // Dense accumulation over all columns (§II-B): bitmap for structure (values may cancel to
 // 0.0 and must still be stored), fp64 array for values, in this CTA's arena slot.  Output is
@@ -1422,6 +1520,13 @@ size_t numw_smem(bool wide) {
 }
 size_t symb_smem() { return size_t(TB_SYM) * sizeof(int32_t); }
 size_t numb_smem() { return size_t(TB_NUM) * (sizeof(int32_t) + sizeof(double)); }
+size_t symm_smem() { return size_t(TM_SYM) * sizeof(int32_t); }
+size_t numm_smem() { return size_t(TM_NUM) * (sizeof(int32_t) + sizeof(double)); }
+
+bool medium_enabled() {  // read per pass (host side), so that a test can switch it
+    const char *v = getenv("SPGEMM_NO_MEDIUM");
+    return !(v && v[0] == '1');
+}
 
 template <int G>
 static void set_attrs_w() {
@@ -1441,6 +1546,8 @@ const Grids &grids(int device, int num_sms) {
         set_attrs_w<32>();
         cudaFuncSetAttribute(k_sym_b, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symb_smem());
         cudaFuncSetAttribute(k_num_b, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numb_smem());
+        cudaFuncSetAttribute(k_sym_m, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symm_smem());
+        cudaFuncSetAttribute(k_num_m, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numm_smem());
         Grids g;
         int occ = 0;
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_count, 256, 0);
@@ -1453,6 +1560,10 @@ const Grids &grids(int device, int num_sms) {
         g.symb_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_b, THREADS_B, numb_smem());
         g.numb_blocks = num_sms * (occ > 0 ? occ : 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_m, THREADS_M, symm_smem());
+        g.symm_blocks = num_sms * (occ > 0 ? occ : 1);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_m, THREADS_M, numm_smem());
+        g.numm_blocks = num_sms * (occ > 0 ? occ : 1);
         cache[device] = g;
         init[device] = true;
     }
@@ -1533,14 +1644,15 @@ static inline void rec(cudaEvent_t *ev, int k, cudaStream_t s) {
 void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev) {
     const int64_t rows = a.r1 - a.r0;
     if (rows <= 0) {
-        for (int k = 0; k < 4; ++k) rec(ev, k, s);
+        for (int k = 0; k < 5; ++k) rec(ev, k, s);
         return;
     }
     int dev = 0;
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
-    cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);  // row_ctr, nB, nG, pass_max, nH
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);  // row_ctr, nB, nG, pass_max, nM
     SymArgs aw = a;
+    if (!(a.tiers & 4)) aw.listM = nullptr;
     aw.batch = batch_for(rows, g.symw_blocks);
     const int wblocks = grid_for(rows, WARPS_W * aw.batch, g.symw_blocks);
     rec(ev, 0, s);
@@ -1551,11 +1663,16 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
         default: sym_w<32>(aw, wblocks, s); break;
     }
     rec(ev, 1, s);
+    if (aw.listM) {
+        k_sym_m<<<g.symm_blocks, THREADS_M, symm_smem(), s>>>(aw);
+        LAUNCHED(1);
+    }
+    rec(ev, 2, s);
     if (a.tiers & 1) {
         k_sym_b<<<a.cursor ? a.bblocks : g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
         LAUNCHED(1);
     }
-    rec(ev, 2, s);
+    rec(ev, 3, s);
     // the dense tier: rows beyond the pieced CTA tier, and rows whose A entries do not fit the
     // cursor scratch (possible whenever the pass has CTA-tier rows; the kernel exits at once
     // when its list is empty)
@@ -1563,13 +1680,13 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
         k_sym_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
         LAUNCHED(1);
     }
-    rec(ev, 3, s);
+    rec(ev, 4, s);
 }
 
 void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *ev) {
     const int64_t rows = a.r1 - a.r0;
     if (rows <= 0) {
-        for (int k = 0; k < 4; ++k) rec(ev, k, s);
+        for (int k = 0; k < 5; ++k) rec(ev, k, s);
         return;
     }
     int dev = 0;
@@ -1577,6 +1694,7 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
     const Grids &g = grids(dev, num_sms);
     cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);
     NumArgs aw = a;
+    if (!(a.tiers & 4)) aw.listM = nullptr;
     static const int tload = env_int("SPGEMM_NUMW_TLOAD", 2);  // tuning knob
     aw.tload = tload;
     aw.batch = batch_for(rows, g.numw_blocks);
@@ -1589,16 +1707,21 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
         default: num_w<32>(aw, wblocks, s); break;
     }
     rec(ev, 1, s);
+    if (aw.listM) {
+        k_num_m<<<g.numm_blocks, THREADS_M, numm_smem(), s>>>(aw);
+        LAUNCHED(1);
+    }
+    rec(ev, 2, s);
     if (a.tiers & 1) {
         k_num_b<<<a.cursor ? a.bblocks : g.numb_blocks, THREADS_B, numb_smem(), s>>>(a);
         LAUNCHED(1);
     }
-    rec(ev, 2, s);
+    rec(ev, 3, s);
     if ((a.tiers & 3) && a.gblocks > 0) {
         k_num_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
         LAUNCHED(1);
     }
-    rec(ev, 3, s);
+    rec(ev, 4, s);
 }
 
 template <typename T>

@@ -299,6 +299,8 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
     P->listB = P->alloc<int32_t>(Q.unit_rows, "listB");
     P->listG = P->alloc<int32_t>(Q.unit_rows, "listG");
     P->listBn = P->alloc<int32_t>(Q.unit_rows, "numeric listB");
+    P->listM = P->alloc<int32_t>(Q.unit_rows, "listM");
+    P->listMn = P->alloc<int32_t>(Q.unit_rows, "numeric listM");
     P->listGn = P->alloc<int32_t>(Q.unit_rows, "numeric listG");
     const int nbins_max = 4096;
     unsigned long long *dhist = P->alloc<unsigned long long>(nbins_max, "column histogram");
@@ -459,6 +461,7 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
             sa.r0 = 0;
             sa.r1 = r1 - r0;
             sa.listB = P->listB;
+            sa.listM = P->listM;
             sa.listG = P->listG;
             sa.ctl = P->ctl;
             sa.gscratch = P->gbits_sym;
@@ -468,7 +471,7 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
             sa.curstride = P->curstride;
             sa.bblocks = P->bblocks_sym;
             sa.group = Q.group[j];
-            sa.tiers = 3;
+            sa.tiers = 3 | (medium_enabled() ? 4 : 0);
             launch_symbolic(sa, P->num_sms, s, nullptr);
             CKL("symbolic");
             stage_done(P, Q);
@@ -496,6 +499,7 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
     P->rows_w = (int64_t)hc2[0].rows_w;
     P->rows_b = (int64_t)hc2[0].rows_b;
     P->rows_g = (int64_t)hc2[0].rows_g;
+    P->rows_m = (int64_t)hc2[0].rows_m;
     CK(cudaMemsetAsync(&P->ctl[1], 0, sizeof(Ctl), s));
 
     // ring from what is left; numeric units per panel from the exact piece sizes
@@ -615,6 +619,7 @@ int64_t panel_run(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double *v
             na.out_col = P->ring_col[b];
             na.out_val = P->ring_val[b];
             na.listB = P->listBn;
+            na.listM = P->listMn;
             na.listG = P->listGn;
             na.ctl = P->ctl + 1;
             na.gbits = P->gbits;

@@ -112,7 +112,8 @@ def test_struct_layouts_match_header(capi, tmp_path):
     src = tmp_path / "lay.c"
     fields = {"spgemm_opts": ["ring", "row_begin", "workspace", "stream", "chunk_nnz", "row_ptr_base", "min_chunks",
                               "fused", "col_panels", "order"],
-              "spgemm_info": ["num_chunks", "chunk_capacity", "rows_global", "fused", "num_copies", "col_panels"],
+              "spgemm_info": ["num_chunks", "chunk_capacity", "rows_global", "fused", "num_copies", "col_panels",
+                              "rows_medium"],
               "spgemm_csr": ["row_ptr", "values", "where"], "spgemm_kernel_stat": ["launches", "ms", "bytes"]}
     lines = ["#include <stdio.h>", "#include <stddef.h>", f'#include "{HEADER}"', "int main(void) {"]
     for s, fs in fields.items():

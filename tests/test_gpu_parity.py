@@ -151,6 +151,32 @@ def test_tiers_warp_block_pieced():
     assert_parity(A, B, rp, col, val)
 
 
+@pytest.mark.parametrize("fused", [False, True])
+@pytest.mark.parametrize("medium", [True, False])
+def test_medium_tier(fused, medium, monkeypatch):
+    """Rows of a few hundred to two thousand products (the R-MAT bulk) go to the 128-thread medium
+    CTA tier; SPGEMM_NO_MEDIUM=1 sends them to the 512-thread tier instead.  Same C either way."""
+    if not medium:
+        monkeypatch.setenv("SPGEMM_NO_MEDIUM", "1")
+    rng = np.random.default_rng(31)
+    ncols = 200_000
+    brows = [np.sort(rng.choice(ncols, int(rng.integers(5, 60)), replace=False)) for _ in range(4000)]
+    B = _csr_from_rows(brows, ncols, rng)
+    arows = []
+    for i in range(1500):
+        d = [3, 12, 25, 40, 70][i % 5]          # ~100 .. 2300 products per row
+        arows.append(np.sort(rng.choice(B.nrows, d, replace=False)))
+    arows[7] = np.sort(rng.choice(200, 60, replace=False))   # clustered columns (overlapping B rows)
+    A = _csr_from_rows(arows, B.nrows, rng)
+    r = run_fused(A, B) if fused else run(A, B)
+    info = r[3]
+    if medium:
+        assert info["rows_medium"] > 300, info
+    else:
+        assert info["rows_medium"] == 0 and info["rows_block"] > 300, info
+    assert_parity(A, B, r[0], r[1], r[2])
+
+
 def _csr_from_rows(rows, ncols, rng):
     rp = np.zeros(len(rows) + 1, np.int64)
     np.cumsum([len(r) for r in rows], out=rp[1:])
@@ -293,9 +319,10 @@ def test_repeat_execute_same_plan(fused):
                 got = [x.copy() for x in P.execute()]
             assert oracle.compare(*got, E)["ok"] and np.array_equal(got[2], E["val"])
             infos.append(P.info())
-    for k in ("nnz", "products", "rows_warp", "rows_block", "rows_global", "max_row_nnz"):
+    for k in ("nnz", "products", "rows_warp", "rows_medium", "rows_block", "rows_global", "max_row_nnz"):
         assert infos[0][k] == infos[1][k] == infos[2][k], k
-    assert infos[0]["rows_warp"] + infos[0]["rows_block"] + infos[0]["rows_global"] <= A.nrows
+    i0 = infos[0]
+    assert i0["rows_warp"] + i0["rows_medium"] + i0["rows_block"] + i0["rows_global"] <= A.nrows
 
 
 # ------------------------------------------------------------------------------------- device inputs
