@@ -17,6 +17,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <condition_variable>
 #include <thread>
 #include <cstdio>
 #include <cstdlib>
@@ -987,21 +988,86 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         int64_t u0, u1, r0, r1, off, nnz, pad;
     };
     std::vector<Group> groups;
-    int64_t done_cb = 0;
-    auto consume = [&](int64_t g) {  // sink: wait for group g's copy and hand it over
-        const Group &G = groups[g];
-        CK(cudaEventSynchronize(P->ev_d2h[G.b]));
-        int64_t *rp = st_rp(G.b);
-        const int64_t first = rp[0];
-        for (int64_t k = 0; k <= G.r1 - G.r0; ++k) rp[k] -= first;
-        const int rc = sink->cb(sink->user, P->row_begin + G.r0, P->row_begin + G.r1, rp, st_col(G.b), st_val(G.b),
-                                rp[G.r1 - G.r0]);
-        if (rc != 0) {
-            CK(cudaStreamSynchronize(cp));
-            CK(cudaStreamSynchronize(s));
-            fail(SPGEMM_ERR_CALLBACK, "chunk sink returned " + std::to_string(rc));
+    // Sink mode: a consumer thread hands every output chunk to the callback as soon as its copy has
+    // landed in the staging slot, while this thread keeps enqueueing later units; a staging slot is
+    // reused only after the callback of the chunk in it returned (back-pressure), so a slow sink
+    // delays the pipeline only when it is `ring` chunks behind.
+    struct Consumer {
+        std::mutex mu;
+        std::condition_variable cv;
+        std::vector<Group> q;  // closed groups, in order
+        int64_t done = 0;      // callbacks completed
+        bool stop = false;
+        int rc = 0;            // first non-zero callback return
+        std::string cuda_err;
+        std::thread th;
+        ~Consumer() {
+            {
+                std::lock_guard<std::mutex> lk(mu);
+                stop = true;
+            }
+            cv.notify_all();
+            if (th.joinable()) th.join();
         }
-        done_cb = g + 1;
+    } cons;
+    if (sink) {
+        cons.th = std::thread([&, dev = P->device] {
+            cudaSetDevice(dev);
+            for (int64_t g = 0;; ++g) {
+                Group G;
+                {
+                    std::unique_lock<std::mutex> lk(cons.mu);
+                    cons.cv.wait(lk, [&] { return int64_t(cons.q.size()) > g || cons.stop; });
+                    if (int64_t(cons.q.size()) <= g) return;
+                    G = cons.q[g];
+                }
+                const cudaError_t e = cudaEventSynchronize(P->ev_d2h[G.b]);
+                int rc = 0;
+                if (e != cudaSuccess) {
+                    std::lock_guard<std::mutex> lk(cons.mu);
+                    cons.cuda_err = cudaGetErrorString(e);
+                    rc = -1;
+                } else {
+                    int64_t *rp = st_rp(G.b);
+                    const int64_t first = rp[0];
+                    for (int64_t k = 0; k <= G.r1 - G.r0; ++k) rp[k] -= first;
+                    rc = sink->cb(sink->user, P->row_begin + G.r0, P->row_begin + G.r1, rp, st_col(G.b), st_val(G.b),
+                                  rp[G.r1 - G.r0]);
+                }
+                {
+                    std::lock_guard<std::mutex> lk(cons.mu);
+                    if (rc != 0 && cons.rc == 0) cons.rc = rc;
+                    if (rc == 0) cons.done = g + 1;
+                }
+                cons.cv.notify_all();
+                if (rc != 0) return;
+            }
+        });
+    }
+    auto sink_failed = [&]() {  // after a callback failure: drain the GPU and report
+        CK(cudaStreamSynchronize(cp));
+        CK(cudaStreamSynchronize(s));
+        if (P->astream && P->astream != s) CK(cudaStreamSynchronize(P->astream));
+        if (!cons.cuda_err.empty()) fail(SPGEMM_ERR_CUDA, "chunk copy: " + cons.cuda_err);
+        fail(SPGEMM_ERR_CALLBACK, "chunk sink returned " + std::to_string(cons.rc));
+    };
+    auto wait_consumed = [&](int64_t upto) {  // sink: callbacks of groups < upto have returned
+        std::unique_lock<std::mutex> lk(cons.mu);
+        cons.cv.wait(lk, [&] { return cons.done >= upto || cons.rc != 0; });
+        if (cons.rc != 0) {
+            lk.unlock();
+            sink_failed();
+        }
+    };
+    auto push_group = [&](const Group &G) {
+        groups.push_back(G);
+        if (sink) {
+            {
+                std::lock_guard<std::mutex> lk(cons.mu);
+                cons.q.push_back(G);
+            }
+            cons.cv.notify_all();
+        }
     };
     auto close_group = [&](Group &G) {  // enqueue the group's copies after its numeric passes
         CK(cudaEventRecord(P->ev_num[G.b], s));
@@ -1074,7 +1140,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
             if (!close && !groups.empty()) close = cudaEventQuery(P->ev_d2h[groups.back().b]) == cudaSuccess;
             if (close) {
                 close_group(cur);
-                groups.push_back(cur);
+                push_group(cur);
                 target = std::min<int64_t>(P->cap, 2 * cur.nnz);
                 cur.b = -1;
             }
@@ -1089,7 +1155,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
             }
             if (g >= ring) {
                 CK(cudaStreamWaitEvent(s, P->ev_d2h[cur.b], 0));
-                if (sink) consume(g - ring);  // frees staging slot cur.b
+                if (sink) wait_consumed(g - ring + 1);  // staging slot cur.b is free again
             }
         }
         if (P->fused) CK(cudaStreamWaitEvent(s, P->ev_tot[j], 0));  // (already complete: host waited)
@@ -1105,7 +1171,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
             // the next unit's total is known (the first group is one unit: the first copy starts
             // right after the first numeric pass)
             close_group(cur);
-            groups.push_back(cur);
+            push_group(cur);
             target = std::min<int64_t>(P->cap, 2 * cur.nnz);
             cur.b = -1;
         }
@@ -1113,10 +1179,9 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
     }
     if (cur.b >= 0) {
         close_group(cur);
-        groups.push_back(cur);
+        push_group(cur);
     }
-    if (sink)
-        for (int64_t g = done_cb; g < int64_t(groups.size()); ++g) consume(g);
+    if (sink) wait_consumed(int64_t(groups.size()));
     P->num_groups = int64_t(groups.size());
     pe.rec(size_t(nch) * per + 1, cp);
     CK(cudaStreamSynchronize(cp));
