@@ -1185,17 +1185,25 @@ __device__ __forceinline__ T warp_incl_scan(T x) {
     return x;
 }
 
-// S7 for a CTA table of T slots holding n keys (+ values): one MSD pass (bucket by column within
-// the table's column range), the packed keys (column << SB | slot) staged in the output value
-// area, then each bucket sorted by one warp in registers.  A bucket over 512 entries (very
-// clustered columns) takes the general path: compaction + shared-memory bitonic.  Writes oc/ov
-// [0, n); returns false (nothing written) if the table does not hold exactly n keys.  All
-// threads call; ends with a barrier.
+// S7 for a CTA table of T <= 2^SB slots holding n keys (+ values).  Fast path: rank inside fine
+// column buckets, entirely in shared memory -- every thread holds its SPT = 2^SB / NT slots' keys
+// in registers, so the key table itself becomes the staging array once it has been read:
+//   histogram of fine buckets (~4 keys each) -> bucket starts (block scan) -> each key staged in
+//   its bucket as (offset within the bucket << SB | slot) -> rank = bucket start + the number of
+//   smaller staged words in the bucket -> column and value written to their final position.
+// (The previous version staged the keys in the global output and ranked from there: 56 % of
+// k_num_b's instructions and 47 % of its stall samples on C3, profiles/r02/ncu_numb_c3_before.md.)
+// A bucket over 64 keys (clustered columns) takes coarse buckets sorted by warps in registers,
+// staged in the output value area; a coarse bucket over 512 keys the general path (compaction +
+// shared-memory bitonic).  Writes oc/ov [0, n); returns false (nothing written) if the table does
+// not hold exactly n keys.  All threads call; ends with a barrier; the key table is clobbered.
 template <int SB, int NT = THREADS_B>
 __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int32_t *oc, double *ov,
                               CtaSortSmemT<NT> &ss, SortCntT<NT> &sc) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     constexpr int NW = NT / 32;
+    constexpr int SPT = (1 << SB) / NT;  // table slots per thread
+    static_assert(SPT * NT == (1 << SB), "table size must be a multiple of the CTA size");
     constexpr int PLMAX = NT == 512 ? 10 : NT == 256 ? 9 : NT == 128 ? 8 : 7;  // 2^PLMAX = 2 NT buckets
     static_assert((1 << PLMAX) == 2 * NT, "two fine buckets per thread");
     // fine buckets (~4 keys each): 2^pl of them, bucket of key k = (k - lo) >> sh
@@ -1207,17 +1215,22 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         ss.mm[0] = INT_MAX;
         ss.mm[1] = -1;
     }
+    int32_t kr[SPT];  // slot j * NT + threadIdx.x
+#pragma unroll
+    for (int j = 0; j < SPT; ++j) {
+        const int t = j * NT + threadIdx.x;
+        kr[j] = t < T ? keys[t] : EMPTY;
+    }
     __syncthreads();
     {
         int lmin = INT_MAX, lmax = -1, occ = 0;
-        for (int t = threadIdx.x; t < T; t += NT) {
-            const int32_t k = keys[t];
-            if (k != EMPTY) {
-                lmin = min(lmin, k);
-                lmax = max(lmax, k);
+#pragma unroll
+        for (int j = 0; j < SPT; ++j)
+            if (kr[j] != EMPTY) {
+                lmin = min(lmin, kr[j]);
+                lmax = max(lmax, kr[j]);
                 ++occ;
             }
-        }
 #pragma unroll
         for (int d = 16; d > 0; d >>= 1) {
             lmin = min(lmin, __shfl_xor_sync(FULLMASK, lmin, d));
@@ -1240,15 +1253,11 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     }
     const int64_t lo = ss.mm[0], span = (int64_t)ss.mm[1] - lo + 1;
     {
-        // Fast path: rank inside fine buckets.  Histogram -> bucket starts -> each key staged in
-        // its bucket (in the output col area) -> each key's final position = bucket start + the
-        // number of smaller keys in its bucket.  ~4 compares per key instead of a bitonic network.
         const int lspan = 64 - __clzll(span - 1);  // 2^lspan >= span
         const int sh = max(0, lspan - pl);
-        for (int t = threadIdx.x; t < T; t += NT) {
-            const int32_t k = keys[t];
-            if (k != EMPTY) atomicAdd(&sc.cnt[(int)(((int64_t)k - lo) >> sh)], 1);
-        }
+#pragma unroll
+        for (int j = 0; j < SPT; ++j)
+            if (kr[j] != EMPTY) atomicAdd(&sc.cnt[(int)(((int64_t)kr[j] - lo) >> sh)], 1);
         __syncthreads();
         const int nb = (int)(((span - 1) >> sh) + 1);  // buckets in use (<= 2^pl)
         const int b0 = 2 * threadIdx.x;
@@ -1265,38 +1274,36 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         int bmax = 0;
 #pragma unroll
         for (int w = 0; w < NW; ++w) bmax = max(bmax, ss.occ[w]);
-        if (bmax <= 64) {
-            for (int t = threadIdx.x; t < T; t += NT) {  // stage; keys[t] := staged position
-                const int32_t k = keys[t];
-                if (k != EMPTY) {
-                    const int pos = atomicAdd(&sc.cur[(int)(((int64_t)k - lo) >> sh)], 1);
-                    oc[pos] = k;
-                    keys[t] = pos;
+        if (bmax <= 64 && sh + SB <= 31) {
+            // stage (every key is in registers: the table is free)
+            uint32_t *stg = reinterpret_cast<uint32_t *>(keys);
+            const uint32_t relmask = (1u << sh) - 1u;
+#pragma unroll
+            for (int j = 0; j < SPT; ++j)
+                if (kr[j] != EMPTY) {
+                    const uint32_t d = (uint32_t)((int64_t)kr[j] - lo);
+                    const int pos = atomicAdd(&sc.cur[d >> sh], 1);
+                    stg[pos] = ((d & relmask) << SB) | (uint32_t)(j * NT + threadIdx.x);
                 }
-            }
             __syncthreads();
-            for (int t = threadIdx.x; t < T; t += NT) {  // rank; value out; key parked in vals[t]
-                const int pos = keys[t];
-                if (pos != EMPTY) {
-                    const int32_t k = oc[pos];
-                    const int b = (int)(((int64_t)k - lo) >> sh);
+            // rank among the bucket's staged words; column and value to the final position
+#pragma unroll
+            for (int j = 0; j < SPT; ++j)
+                if (kr[j] != EMPTY) {
+                    const int t = j * NT + threadIdx.x;
+                    const uint32_t d = (uint32_t)((int64_t)kr[j] - lo);
+                    const uint32_t x = ((d & relmask) << SB) | (uint32_t)t;
+                    const int b = (int)(d >> sh);
                     const int s0 = sc.start[b], e0 = s0 + sc.cnt[b];
                     int r = s0, q = s0;
-                    for (; q + 4 <= e0; q += 4) {  // 4 independent loads in flight
-                        const int32_t x0 = oc[q], x1 = oc[q + 1], x2 = oc[q + 2], x3 = oc[q + 3];
-                        r += (x0 < k) + (x1 < k) + (x2 < k) + (x3 < k);
+                    for (; q + 4 <= e0; q += 4) {
+                        const uint32_t x0 = stg[q], x1 = stg[q + 1], x2 = stg[q + 2], x3 = stg[q + 3];
+                        r += (x0 < x) + (x1 < x) + (x2 < x) + (x3 < x);
                     }
-                    for (; q < e0; ++q) r += oc[q] < k;
+                    for (; q < e0; ++q) r += stg[q] < x;
+                    oc[r] = kr[j];
                     ov[r] = vals[t];
-                    keys[t] = r;
-                    reinterpret_cast<int32_t *>(vals + t)[0] = k;
                 }
-            }
-            __syncthreads();
-            for (int t = threadIdx.x; t < T; t += NT) {  // columns
-                const int r = keys[t];
-                if (r != EMPTY) oc[r] = reinterpret_cast<const int32_t *>(vals + t)[0];
-            }
             __syncthreads();
             return true;
         }

@@ -119,3 +119,46 @@ def test_gloo_scatter_allgather_b(world):
         p.join(timeout=60)
         assert p.exitcode == 0
     assert all(ok for _, ok in res), res
+
+
+def _worker_flops(rank, world, port, q):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        A = W.rmat(11, 8, seed=9)
+        s0, s1 = pdist.even_slices(A.nrows, world)[rank]
+        # each rank counts only its even slice (bench.py: spgemm_row_products on its GPU)
+        u_loc = oracle.products(A, A, rows=np.arange(s0, s1))
+        u_all = pdist.allgather_rows(u_loc, A.nrows)
+        panels = pdist.row_panels(A.row_ptr, world, weights=u_all)
+        q.put((rank, u_all, panels))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_gloo_flop_balanced_panels(world):
+    """every rank counts the products of 1/world of the rows, one all_gather gives
+    everybody the whole per-row count, and all ranks cut the SAME row panels, balanced by products
+    (within one row's products of the ideal share) -- bench.py's multi-GPU deal."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_flops, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=120) for _ in range(world)], key=lambda t: t[0])
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    A = W.rmat(11, 8, seed=9)
+    u = oracle.products(A, A)
+    for _, u_all, panels in res:
+        assert np.array_equal(u_all, u)
+        assert panels == res[0][2]
+    panels = res[0][2]
+    assert panels[0][0] == 0 and panels[-1][1] == A.nrows
+    loads = [int(u[a:b].sum()) for a, b in panels]
+    assert max(loads) - u.sum() / world <= u.max() + 1
