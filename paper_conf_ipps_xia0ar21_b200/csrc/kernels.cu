@@ -1160,11 +1160,13 @@ struct CtaSortSmemT {
 };
 using CtaSortSmem = CtaSortSmemT<THREADS_B>;
 
-// fine-bucket counters of the CTA sort (2 per thread: the bucket scan gives each thread two); they
-// alias the product iterator's ProdSmem (not in use while a table is sorted)
+// fine-bucket cursors of the CTA sort: 8 NT buckets, two 16-bit cursors per word (positions are
+// < 2^16); one array serves as histogram, bucket start, staging cursor and -- once staged -- bucket
+// end (= the next bucket's start).  They alias the product iterator's ProdSmem (not in use while
+// a table is sorted).
 template <int NT>
 struct SortCntT {
-    int cnt[2 * NT], cur[2 * NT], start[2 * NT];
+    uint32_t arr[4 * NT];
 };
 using SortCnt = SortCntT<THREADS_B>;
 template <int NT, int PB>
@@ -1204,11 +1206,11 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     constexpr int NW = NT / 32;
     constexpr int SPT = (1 << SB) / NT;  // table slots per thread
     static_assert(SPT * NT == (1 << SB), "table size must be a multiple of the CTA size");
-    constexpr int PLMAX = NT == 512 ? 10 : NT == 256 ? 9 : NT == 128 ? 8 : 7;  // 2^PLMAX = 2 NT buckets
-    static_assert((1 << PLMAX) == 2 * NT, "two fine buckets per thread");
-    // fine buckets (~4 keys each): 2^pl of them, bucket of key k = (k - lo) >> sh
-    const int pl = min(PLMAX, max(5, 32 - __clz((int)max((int64_t)1, (n + 3) / 4) - 1)));
-    for (int b = threadIdx.x; b < (1 << pl); b += NT) sc.cnt[b] = 0;
+    constexpr int PLMAX = NT == 512 ? 12 : NT == 256 ? 11 : NT == 128 ? 10 : 9;  // 2^PLMAX = 8 NT buckets
+    static_assert((1 << PLMAX) == 8 * NT, "eight fine buckets per thread");
+    // fine buckets (~1 key each): 2^pl of them, bucket of key k = (k - lo) >> sh
+    const int pl = min(PLMAX, max(5, 32 - __clz((int)max((int64_t)1, n) - 1)));
+    for (int w = threadIdx.x; w < (1 << (pl - 1)); w += NT) sc.arr[w] = 0u;
     const int P = min(64, max(1, (int)((n + 255) / 256)));
     if (threadIdx.x < 64) ss.cnt[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
@@ -1255,18 +1257,36 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     {
         const int lspan = 64 - __clzll(span - 1);  // 2^lspan >= span
         const int sh = max(0, lspan - pl);
+        // histogram (16-bit counters, two per word)
 #pragma unroll
         for (int j = 0; j < SPT; ++j)
-            if (kr[j] != EMPTY) atomicAdd(&sc.cnt[(int)(((int64_t)kr[j] - lo) >> sh)], 1);
+            if (kr[j] != EMPTY) {
+                const uint32_t b = (uint32_t)(((int64_t)kr[j] - lo) >> sh);
+                atomicAdd(&sc.arr[b >> 1], 1u << ((b & 1u) << 4));
+            }
         __syncthreads();
-        const int nb = (int)(((span - 1) >> sh) + 1);  // buckets in use (<= 2^pl)
-        const int b0 = 2 * threadIdx.x;
-        const int c0 = b0 < nb ? sc.cnt[b0] : 0, c1 = b0 + 1 < nb ? sc.cnt[b0 + 1] : 0;
+        // bucket starts: thread t owns words 4t .. 4t+3 (buckets 8t .. 8t+7)
+        const int w0 = 4 * threadIdx.x;
+        const bool mine = w0 < (1 << (pl - 1));
+        uint32_t wv[4];
+        int sum = 0, big = 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            wv[q] = mine ? sc.arr[w0 + q] : 0u;
+            const int c0 = (int)(wv[q] & 0xffffu), c1 = (int)(wv[q] >> 16);
+            sum += c0 + c1;
+            big = max(big, max(c0, c1));
+        }
         int64_t tot;
-        const int64_t ex = block_excl_scan<NT>(c0 + c1, ss.scan, &tot);  // ends with a barrier
-        if (b0 < nb) sc.start[b0] = sc.cur[b0] = (int)ex;
-        if (b0 + 1 < nb) sc.start[b0 + 1] = sc.cur[b0 + 1] = (int)ex + c0;
-        int big = max(c0, c1);
+        int run = (int)block_excl_scan<NT>(sum, ss.scan, &tot);  // ends with a barrier
+        if (mine) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int c0 = (int)(wv[q] & 0xffffu), c1 = (int)(wv[q] >> 16);
+                sc.arr[w0 + q] = (uint32_t)run | ((uint32_t)(run + c0) << 16);
+                run += c0 + c1;
+            }
+        }
 #pragma unroll
         for (int d = 16; d > 0; d >>= 1) big = max(big, __shfl_xor_sync(FULLMASK, big, d));
         if (lane == 0) ss.occ[wid] = big;
@@ -1275,32 +1295,32 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
 #pragma unroll
         for (int w = 0; w < NW; ++w) bmax = max(bmax, ss.occ[w]);
         if (bmax <= 64 && sh + SB <= 31) {
-            // stage (every key is in registers: the table is free)
+            // stage (every key is in registers: the key table is free) -- the word
+            // (offset within the bucket << SB | slot) at the bucket's next position
             uint32_t *stg = reinterpret_cast<uint32_t *>(keys);
             const uint32_t relmask = (1u << sh) - 1u;
 #pragma unroll
             for (int j = 0; j < SPT; ++j)
                 if (kr[j] != EMPTY) {
                     const uint32_t d = (uint32_t)((int64_t)kr[j] - lo);
-                    const int pos = atomicAdd(&sc.cur[d >> sh], 1);
+                    const uint32_t b = d >> sh, hs = (b & 1u) << 4;
+                    const int pos = (int)((atomicAdd(&sc.arr[b >> 1], 1u << hs) >> hs) & 0xffffu);
                     stg[pos] = ((d & relmask) << SB) | (uint32_t)(j * NT + threadIdx.x);
                 }
             __syncthreads();
-            // rank among the bucket's staged words; column and value to the final position
+            // rank among the bucket's staged words (bucket b = [end(b - 1), end(b))); column and
+            // value to the final position
 #pragma unroll
             for (int j = 0; j < SPT; ++j)
                 if (kr[j] != EMPTY) {
                     const int t = j * NT + threadIdx.x;
                     const uint32_t d = (uint32_t)((int64_t)kr[j] - lo);
                     const uint32_t x = ((d & relmask) << SB) | (uint32_t)t;
-                    const int b = (int)(d >> sh);
-                    const int s0 = sc.start[b], e0 = s0 + sc.cnt[b];
-                    int r = s0, q = s0;
-                    for (; q + 4 <= e0; q += 4) {
-                        const uint32_t x0 = stg[q], x1 = stg[q + 1], x2 = stg[q + 2], x3 = stg[q + 3];
-                        r += (x0 < x) + (x1 < x) + (x2 < x) + (x3 < x);
-                    }
-                    for (; q < e0; ++q) r += stg[q] < x;
+                    const uint32_t b = d >> sh;
+                    const int e0 = (int)((sc.arr[b >> 1] >> ((b & 1u) << 4)) & 0xffffu);
+                    const int s0 = b == 0 ? 0 : (int)((sc.arr[(b - 1) >> 1] >> (((b - 1) & 1u) << 4)) & 0xffffu);
+                    int r = s0;
+                    for (int q = s0; q < e0; ++q) r += stg[q] < x;
                     oc[r] = kr[j];
                     ov[r] = vals[t];
                 }
