@@ -563,7 +563,9 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         P->gstride_bits = (nwords + 63) & ~int64_t(63);
         P->gstride_vals = (P->ncols + 31) & ~int64_t(31);
         const size_t gper = size_t(P->gstride_bits) * 8 + size_t(P->gstride_vals) * 8;
-        const int64_t gwant = (P->max_bound > CAPS_NUM || P->max_deg > CURSOR_MAX) ? P->num_sms : 8;
+        // up to 4 dense-tier CTAs per SM (the kernels are latency-bound on their L2 atomics and
+        // fit 4 x 512 threads per SM; C3's 9 K hub rows: 1 CTA per SM left 3/4 of the warps idle)
+        const int64_t gwant = (P->max_bound > CAPS_NUM || P->max_deg > CURSOR_MAX) ? 4 * int64_t(P->num_sms) : 8;
         int64_t ng = std::min<int64_t>(gwant, int64_t(avail / gper));
         if (ng < 1) {
             const size_t fb = P->arena_bytes > P->used + ring_min ? P->arena_bytes - P->used - ring_min : 0;

@@ -1456,7 +1456,7 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
 // One 128-thread CTA per row of CAPW_NUM < nnz <= CAPM_NUM (24 KB table: ~8 rows in flight per SM),
 // the B tier's product iterator and bucket sort at 128 threads.
 
-__global__ void __launch_bounds__(THREADS_M) k_num_m(NumArgs a) {
+__global__ void __launch_bounds__(THREADS_M, 6) k_num_m(NumArgs a) {
     extern __shared__ __align__(16) double smem_d[];
     double *vals = smem_d;
     int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TM_NUM);
