@@ -453,7 +453,14 @@ def main():
     if budget:
         ws = torch.empty(budget - in_bytes, dtype=torch.uint8, device=dev)
     else:
-        ws = torch.empty(int(torch.cuda.mem_get_info()[0] * 0.85), dtype=torch.uint8, device=dev)
+        # ranks sharing one GPU (the gloo control-flow run) split its memory
+        share = -(-int(os.environ.get("LOCAL_WORLD_SIZE", world)) // max(1, torch.cuda.device_count()))
+        if world > 1:
+            dist.barrier()  # every rank's operands are resident before anyone sizes its arena
+        free = torch.cuda.mem_get_info()[0]
+        if world > 1:
+            dist.barrier()  # ... and every rank has read the free memory before anyone allocates
+        ws = torch.empty(int(free * 0.85 / share), dtype=torch.uint8, device=dev)
     wbytes = ws.numel()
     fused = not args.two_phase
     chunk_nnz = args.chunk_nnz if sink_mode else 0

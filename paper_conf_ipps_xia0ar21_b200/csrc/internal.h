@@ -50,8 +50,9 @@ constexpr int ROW_BATCH = 16;              // rows a warp claims per atomic in t
 struct Ctl {
     unsigned long long row_ctr;   // W kernels: next row batch                      } reset before
     unsigned int nB, nG;          // long-row list lengths                          } every pass
-    unsigned long long pass_max;  // symbolic: max nnz of a row in this pass        } (32 bytes)
-    unsigned int nM, pad0;        // medium-tier list length                        }
+    unsigned long long pass_max;  // symbolic: max nnz of a row in this pass        } (CTL_RESET
+    unsigned int nM, bctr;        // medium-tier list length; B-tier claim cursor   }  bytes)
+    unsigned int mctr, gctr;      // M / G-tier claim cursors (rows claimed one by one) }
     unsigned int err;             // bit 0: numeric count mismatch; bit 1: invalid input; bit 2: table overflow
     unsigned int pad;
     unsigned long long sum_u;     // count pass: sum of products
@@ -61,8 +62,9 @@ struct Ctl {
     unsigned long long rows_w, rows_b, rows_g;
     unsigned long long max_deg;   // count pass: longest row of A (cursor scratch of pieced rows)
     unsigned long long rows_m;    // rows of the medium tier (symbolic passes)
-    unsigned long long pad2[4];
+    unsigned long long pad2[3];
 };
+constexpr size_t CTL_RESET = 40;  // bytes of Ctl cleared before every pass (row_ctr .. gctr)
 
 // --- launchers (all asynchronous on `s`) ---------------------------------------------------
 

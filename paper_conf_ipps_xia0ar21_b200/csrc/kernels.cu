@@ -14,6 +14,7 @@
 // tiers); the G tier is a dense bitmap + fp64 array over all columns in arena scratch (the
 // "dense accumulation" of §II-B L107 / §III-B, used here for the longest rows).
 #include <climits>
+#include <cstddef>
 #include <cstdio>
 #include <cstdlib>
 
@@ -86,6 +87,17 @@ __device__ __forceinline__ T warp_sum(T v) {
 #pragma unroll
     for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(FULLMASK, v, d);
     return v;
+}
+
+// Dynamic row claim of the CTA tiers: the next index of the tier's list for the whole CTA (all
+// threads call; two barriers).  Row costs are heavy-tailed on power-law inputs (a pieced row of
+// 10^5 nonzeros next to rows of 10^3), so a static stride left CTAs idle behind the unlucky one
+// (per-unit launches of the symbolic CTA tier took 1.8x the single-launch time on C3).
+__device__ __forceinline__ unsigned cta_claim(unsigned *ctr, unsigned *s_idx) {
+    __syncthreads();  // every thread has read the previous claim
+    if (threadIdx.x == 0) *s_idx = atomicAdd(ctr, 1u);
+    __syncthreads();
+    return *s_idx;
 }
 
 // exclusive block scan of one int64 per thread; s has >= 33 entries; returns exclusive prefix,
@@ -306,33 +318,49 @@ __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR
         }
         if (threadIdx.x == 0) sm.off[nb] = tot;
         __syncthreads();
-        // Each warp takes 32 consecutive products per step (coalesced B loads).  Two lanes find
-        // the segments of the warp's first and last product; every lane then searches only that
-        // window (usually 1-3 segments) instead of all nb A entries of the batch.
+        // Each warp takes 32 consecutive products per step (coalesced B loads), two steps at a
+        // time: the B loads of both are issued before either product is consumed, so two gathers
+        // are in flight per lane while the first one's hash insert runs (long-scoreboard stalls on
+        // these loads were the top stall of the CTA kernels, profiles/r02/).  Four lanes find the
+        // segments of the first and last product of each step; every lane then searches only
+        // that window (usually 1-3 segments) instead of all nb A entries of the batch.
         const int lane = threadIdx.x & 31;
-        for (int64_t qb = threadIdx.x - lane; qb < tot; qb += NT) {  // warp-uniform trip count
-            const int64_t q = qb + lane;
+        for (int64_t qb = threadIdx.x - lane; qb < tot; qb += 2 * NT) {  // warp-uniform trip count
             int lo = 0, hi = nb;  // invariant: off[lo] <= q < off[hi]
-            if (lane < 2) {
-                const int64_t qq = lane ? min(qb + 31, tot - 1) : qb;
+            if (lane < 4) {
+                const int64_t q0 = qb + (lane >> 1) * NT;
+                const int64_t qq = (lane & 1) ? min(q0 + 31, tot - 1) : min(q0, tot - 1);
                 while (hi - lo > 1) {
                     const int mid = (lo + hi) >> 1;
                     if (sm.off[mid] <= qq) lo = mid;
                     else hi = mid;
                 }
             }
-            const int wlo = __shfl_sync(FULLMASK, lo, 0), whi = __shfl_sync(FULLMASK, lo, 1) + 1;
-            if (q < tot) {
-                lo = wlo;
-                hi = whi;
-                while (hi - lo > 1) {
-                    const int mid = (lo + hi) >> 1;
-                    if (sm.off[mid] <= q) lo = mid;
-                    else hi = mid;
+            int32_t c[2];
+            double v[2];
+            bool ok[2];
+#pragma unroll
+            for (int u = 0; u < 2; ++u) {
+                const int64_t q = qb + u * NT + lane;
+                const int wlo = __shfl_sync(FULLMASK, lo, 2 * u), whi = __shfl_sync(FULLMASK, lo, 2 * u + 1) + 1;
+                ok[u] = q < tot;
+                c[u] = 0;
+                v[u] = 0.0;
+                if (ok[u]) {
+                    int l2 = wlo, h2 = whi;
+                    while (h2 - l2 > 1) {
+                        const int mid = (l2 + h2) >> 1;
+                        if (sm.off[mid] <= q) l2 = mid;
+                        else h2 = mid;
+                    }
+                    const int64_t pos = sm.bs[l2] + (q - sm.off[l2]);
+                    c[u] = __ldg(&B.col[pos]);
+                    if (VALS) v[u] = sm.a[l2] * __ldg(&B.val[pos]);
                 }
-                const int64_t pos = sm.bs[lo] + (q - sm.off[lo]);
-                f(__ldg(&B.col[pos]), VALS ? sm.a[lo] * __ldg(&B.val[pos]) : 0.0);
             }
+#pragma unroll
+            for (int u = 0; u < 2; ++u)
+                if (ok[u]) f(c[u], v[u]);
         }
         __syncthreads();
     }
@@ -706,7 +734,8 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
     int32_t *cur = a.cursor ? a.cursor + (int64_t)blockIdx.x * 2 * a.curstride : nullptr;
     int32_t *nxt = cur ? cur + a.curstride : nullptr;
     const unsigned n = *(volatile unsigned *)&a.ctl->nB;
-    for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
+    __shared__ unsigned s_idx;
+    for (unsigned idx = cta_claim(&a.ctl->bctr, &s_idx); idx < n; idx = cta_claim(&a.ctl->bctr, &s_idx)) {
         const int64_t i = a.listB[idx];
         const int64_t bound = a.bnd[i];
         int64_t total = 0;
@@ -760,7 +789,8 @@ __global__ void __launch_bounds__(THREADS_M) k_sym_m(SymArgs a) {
     static_assert((1 << MAXLG) == TM_SYM, "table size");
     const unsigned n = *(volatile unsigned *)&a.ctl->nM;
     unsigned long long lmax = 0, nrow = 0;
-    for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
+    __shared__ unsigned s_idx;
+    for (unsigned idx = cta_claim(&a.ctl->mctr, &s_idx); idx < n; idx = cta_claim(&a.ctl->mctr, &s_idx)) {
         const int64_t i = a.listM[idx];
         const int lg = table_log2(a.bnd[i], MAXLG);
         const int T = 1 << lg;
@@ -797,7 +827,8 @@ __global__ void __launch_bounds__(THREADS_G) k_sym_g(SymArgs a) {
     uint32_t *bm = a.gscratch + (int64_t)blockIdx.x * a.gstride;
     const unsigned n = *(volatile unsigned *)&a.ctl->nG;
     const int64_t nwords = (a.B.ncols + 31) / 32;
-    for (unsigned idx = blockIdx.x; idx < n; idx += gridDim.x) {
+    __shared__ unsigned s_idx;
+    for (unsigned idx = cta_claim(&a.ctl->gctr, &s_idx); idx < n; idx = cta_claim(&a.ctl->gctr, &s_idx)) {
         const int64_t i = a.listG[idx];
         int cnt = 0;
         block_row_products<THREADS_G, false>(a.A, a.B, i, psm, [&](int32_t c, double) {
@@ -1406,7 +1437,8 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
     int32_t *nxt = cur ? cur + a.curstride : nullptr;
     const unsigned nrows = *(volatile unsigned *)&a.ctl->nB;
     const int64_t off0 = a.crp[a.r0];
-    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
+    __shared__ unsigned s_idx;
+    for (unsigned idx = cta_claim(&a.ctl->bctr, &s_idx); idx < nrows; idx = cta_claim(&a.ctl->bctr, &s_idx)) {
         const int64_t i = a.listB[idx];
         const int64_t o = a.crp[i];
         const int64_t n = a.crp[i + 1] - o;
@@ -1466,7 +1498,8 @@ __global__ void __launch_bounds__(THREADS_M, 6) k_num_m(NumArgs a) {
     static_assert((1 << MAXLG) == TM_NUM, "table size");
     const unsigned nrows = *(volatile unsigned *)&a.ctl->nM;
     const int64_t off0 = a.crp[a.r0];
-    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
+    __shared__ unsigned s_idx;
+    for (unsigned idx = cta_claim(&a.ctl->mctr, &s_idx); idx < nrows; idx = cta_claim(&a.ctl->mctr, &s_idx)) {
         const int64_t i = a.listM[idx];
         const int64_t o = a.crp[i];
         const int64_t n = a.crp[i + 1] - o;
@@ -1500,7 +1533,8 @@ __global__ void __launch_bounds__(THREADS_G) k_num_g(NumArgs a) {
     const unsigned nrows = *(volatile unsigned *)&a.ctl->nG;
     const int64_t nwords = (a.B.ncols + 31) / 32;
     const int64_t off0 = a.crp[a.r0];
-    for (unsigned idx = blockIdx.x; idx < nrows; idx += gridDim.x) {
+    __shared__ unsigned s_idx;
+    for (unsigned idx = cta_claim(&a.ctl->gctr, &s_idx); idx < nrows; idx = cta_claim(&a.ctl->gctr, &s_idx)) {
         const int64_t i = a.listG[idx];
         const int64_t o = a.crp[i];
         const int64_t n = a.crp[i + 1] - o;
@@ -1677,7 +1711,8 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
     int dev = 0;
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
-    cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);  // row_ctr, nB, nG, pass_max, nM
+    static_assert(offsetof(Ctl, err) == CTL_RESET, "Ctl layout");
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, CTL_RESET, s);  // row_ctr, list lengths, pass_max, claim cursors
     SymArgs aw = a;
     if (!(a.tiers & 4)) aw.listM = nullptr;
     aw.batch = batch_for(rows, g.symw_blocks);
@@ -1719,7 +1754,7 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
     int dev = 0;
     cudaGetDevice(&dev);
     const Grids &g = grids(dev, num_sms);
-    cudaMemsetAsync(&a.ctl->row_ctr, 0, 32, s);
+    cudaMemsetAsync(&a.ctl->row_ctr, 0, CTL_RESET, s);
     NumArgs aw = a;
     if (!(a.tiers & 4)) aw.listM = nullptr;
     static const int tload = env_int("SPGEMM_NUMW_TLOAD", 2);  // tuning knob
