@@ -215,6 +215,7 @@ SymArgs sym_args(spgemm_plan_s *P, int64_t r0, int64_t r1, int tiers) {
     sa.listG = P->listG;
     sa.ctl = P->ctl;
     sa.gscratch = P->gbits_sym;
+    sa.gcnt = P->gcnt;
     sa.gstride = P->gstride_bits;
     sa.gblocks = P->gblocks;
     sa.cursor = P->cur_sym;
@@ -567,6 +568,8 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         // fit 4 x 512 threads per SM; C3's 9 K hub rows: 1 CTA per SM left 3/4 of the warps idle)
         const int64_t gwant = (P->max_bound > CAPS_NUM || P->max_deg > CURSOR_MAX) ? 4 * int64_t(P->num_sms) : 8;
         int64_t ng = std::min<int64_t>(gwant, int64_t(avail / gper));
+        if (const char *mg = getenv("SPGEMM_MAX_GSLOTS"))  // test hook: few slots, so that dense rows
+            ng = std::min<int64_t>(ng, std::max(1, atoi(mg)));  // overflow to the one-CTA kernels
         if (ng < 1) {
             const size_t fb = P->arena_bytes > P->used + ring_min ? P->arena_bytes - P->used - ring_min : 0;
             ng = fb >= gper ? 1 : 0;
@@ -576,6 +579,9 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         P->gbits = P->alloc<uint32_t>(P->gstride_bits * ng, "dense-tier bitmap (numeric)");
         P->gbits_sym = P->alloc<uint32_t>(P->gstride_bits * ng, "dense-tier bitmap (symbolic)");
         P->gvals = P->alloc<double>(P->gstride_vals * ng, "dense-tier values");
+        // split dense rows: per slot a fresh-column counter (symbolic) / KG_SWEEP range counts (numeric)
+        P->gcnt = P->alloc<unsigned long long>(2 * ng * (KG_SWEEP + 1), "dense-tier counters");
+        CK(cudaMemsetAsync(P->gcnt, 0, sizeof(unsigned long long) * 2 * ng * (KG_SWEEP + 1), s));
         CK(cudaMemsetAsync(P->gbits, 0, size_t(P->gstride_bits) * ng * 4, s));
         CK(cudaMemsetAsync(P->gbits_sym, 0, size_t(P->gstride_bits) * ng * 4, s));
         CK(cudaMemsetAsync(P->gvals, 0, size_t(P->gstride_vals) * ng * 8, s));
@@ -697,10 +703,14 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
         CK(cudaMemsetAsync(P->crp, 0, sizeof(int64_t), s));
         const int64_t nch = P->num_chunks();
         P->ev_tot = rs->events(Res::PLAIN, ev_base, nch);
-        // the symbolic passes get their own stream so that chunk j+1's symbolic pass overlaps
-        // chunk j's numeric pass (the two passes have separate lists and arena scratch)
-        const char *ser = getenv("SPGEMM_SERIAL_ANALYSIS");  // ablation knob
-        P->astream = (ser && ser[0] == '1') ? P->stream : rs->stream(rs->astream);
+        // The symbolic passes run on the compute stream, two units ahead of the numeric passes
+        // (run_pipeline), so the GPU never waits for the host between units.  With
+        // SPGEMM_CONCURRENT_ANALYSIS=1 they get their own stream and overlap the numeric passes
+        // instead: no faster on the configured workloads (the step is host-link-bound: C3 5.72 s
+        // both ways, C2 55.5 / 55.7 ms), and the kernels' event times then include each other's
+        // contention, which makes per-kernel rates meaningless (profiles/r02/serial_analysis.md).
+        const char *conc = getenv("SPGEMM_CONCURRENT_ANALYSIS");
+        P->astream = (conc && conc[0] == '1') ? rs->stream(rs->astream) : P->stream;
     }
     // host operands: the last value piece each chunk's numeric pass reads (largest B row touched;
     // with A aliasing B also the chunk's own rows)
@@ -776,6 +786,7 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t slot_off, int64
     na.ctl = P->ctl + 1;
     na.gbits = P->gbits;
     na.gvals = P->gvals;
+    na.gcnt = P->gcnt ? P->gcnt + size_t(P->gblocks) * (KG_SWEEP + 1) : nullptr;
     na.gstride_bits = P->gstride_bits;
     na.gstride_vals = P->gstride_vals;
     na.gblocks = P->gblocks;
@@ -784,6 +795,7 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t slot_off, int64
     na.bblocks = P->bblocks_num;
     na.group = P->group;
     na.tiers = num_tiers(max_row_nnz);
+    if (P->profile && c < int64_t(P->tiers_num.size())) P->tiers_num[c] = na.tiers;
     launch_numeric(na, P->num_sms, P->stream, ev);
     CKL("numeric");
 }
@@ -812,6 +824,7 @@ void enqueue_analysis(spgemm_plan_s *P, int64_t j, cudaEvent_t *ev) {
         CKL("count");
     }
     SymArgs sa = sym_args(P, r0, r1, sym_tiers(P->chunk_maxb[j]));
+    if (P->profile && j < int64_t(P->tiers_sym.size())) P->tiers_sym[j] = sa.tiers;
     launch_symbolic(sa, P->num_sms, as, ev);
     CKL("symbolic");
     launch_scan(P->nnzr + r0, r1 - r0, P->crp + r0, P->tmp, as);
@@ -840,18 +853,22 @@ void finalize_profile(spgemm_plan_s *P) {
     // e[7..11] numeric tier boundaries, e[12..13] copy start / end (last unit of an output chunk)
     for (int64_t c = 0; c < nch; ++c) {
         cudaEvent_t *e = ev_at(size_t(c) * per);
+        // a tier's time counts only for the units that launched it
+        const int ts = c < int64_t(P->tiers_sym.size()) ? P->tiers_sym[c] : 7;
+        const int tn = c < int64_t(P->tiers_num.size()) ? P->tiers_num[c] : 7;
+        const bool g_ok = P->gblocks > 0;
         if (P->fused) {
             P->add_stat("sym_w", elapsed(e[0], e[1]), 0);
-            P->add_stat("sym_m", elapsed(e[1], e[2]), 0);
-            P->add_stat("sym_b", elapsed(e[2], e[3]), 0);
-            P->add_stat("sym_g", elapsed(e[3], e[4]), 0);
+            if (ts & 4) P->add_stat("sym_m", elapsed(e[1], e[2]), 0);
+            if (ts & 1) P->add_stat("sym_b", elapsed(e[2], e[3]), 0);
+            if ((ts & 3) && g_ok) P->add_stat("sym_g", elapsed(e[3], e[4]), 0);
             P->add_stat("scan", elapsed(e[4], e[5]), 0);
         }
         if (!overflow) {
             P->add_stat("num_w", elapsed(e[7], e[8]), 0);
-            P->add_stat("num_m", elapsed(e[8], e[9]), 0);
-            P->add_stat("num_b", elapsed(e[9], e[10]), 0);
-            P->add_stat("num_g", elapsed(e[10], e[11]), 0);
+            if (tn & 4) P->add_stat("num_m", elapsed(e[8], e[9]), 0);
+            if (tn & 1) P->add_stat("num_b", elapsed(e[9], e[10]), 0);
+            if ((tn & 3) && g_ok) P->add_stat("num_g", elapsed(e[10], e[11]), 0);
         }
     }
     const std::vector<int64_t> &gl = P->pend.group_last;
@@ -952,6 +969,10 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
 
     const int per = 14;
     EvSet pe(P->profile, P->res, 12, size_t(nch) * per + 4);
+    if (P->profile) {
+        P->tiers_sym.assign(size_t(nch), 0);
+        P->tiers_num.assign(size_t(nch), 0);
+    }
     CK(cudaEventRecord(P->ev_ready, s));
     CK(cudaStreamWaitEvent(cp, P->ev_ready, 0));
     pe.rec(size_t(nch) * per, s);
@@ -964,7 +985,11 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
             CK(cudaMemcpyAsync(rp_out, P->crp, sizeof(int64_t) * (P->R + 1), cudaMemcpyDeviceToHost, cp));
         }
     }
-    if (P->fused && nch > 0) enqueue_analysis(P, 0, pe.at(0));
+    // fused plans: the symbolic pass + scan of unit j + 2 is enqueued while unit j's numeric pass is
+    // (the host waits for unit j + 1's total in between, so the stream always holds queued work)
+    constexpr int64_t LOOKAHEAD = 2;
+    if (P->fused)
+        for (int64_t j = 0; j < std::min<int64_t>(LOOKAHEAD, nch); ++j) enqueue_analysis(P, j, pe.at(size_t(j) * per));
 
     std::vector<int64_t> offs(nch + 1, 0);  // chunk offsets relative to the slice
     if (!P->fused && nch > 0)
@@ -1125,7 +1150,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         const int64_t r0 = P->chunk_rows[j], r1 = P->chunk_rows[j + 1];
         int64_t mx = P->max_nnz;
         if (P->fused) {
-            // unit j's symbolic pass was enqueued one iteration ago; its total decides where the
+            // unit j's symbolic pass was enqueued LOOKAHEAD iterations ago; its total decides where the
             // unit lands on the host and its max row nnz which numeric tiers to launch
             CK(cudaEventSynchronize(P->ev_tot[j]));
             offs[j + 1] = P->h_small[1 + 2 * j] - base;
@@ -1134,7 +1159,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         const int64_t o = offs[j], n = offs[j + 1] - offs[j];
         if (!sink && o + n > capacity) *overflow = true;
         if (*overflow) {
-            if (P->fused && j + 1 < nch) enqueue_analysis(P, j + 1, pe.at(size_t(j + 1) * per));
+            if (P->fused && j + LOOKAHEAD < nch) enqueue_analysis(P, j + LOOKAHEAD, pe.at(size_t(j + LOOKAHEAD) * per));
             continue;
         }
         if (cur.b >= 0) {
@@ -1177,7 +1202,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
             target = std::min<int64_t>(P->cap, 2 * cur.nnz);
             cur.b = -1;
         }
-        if (P->fused && j + 1 < nch) enqueue_analysis(P, j + 1, pe.at(size_t(j + 1) * per));
+        if (P->fused && j + LOOKAHEAD < nch) enqueue_analysis(P, j + LOOKAHEAD, pe.at(size_t(j + LOOKAHEAD) * per));
     }
     if (cur.b >= 0) {
         close_group(cur);

@@ -152,6 +152,7 @@ struct spgemm_plan_s {
 
     uint32_t *gbits = nullptr, *gbits_sym = nullptr;
     double *gvals = nullptr;
+    unsigned long long *gcnt = nullptr;  // split dense rows: counters (2 x gblocks x (KG_SWEEP + 1))
     int32_t *cur_sym = nullptr, *cur_num = nullptr;  // pieced CTA tier: cursor scratch
     int64_t curstride = 0, max_deg = 0;
     int bblocks_sym = 0, bblocks_num = 0;
@@ -176,6 +177,7 @@ struct spgemm_plan_s {
     int64_t *h_small = nullptr;  // pinned + mapped: [0] base; chunk j: [1 + 2j] end offset,
     int64_t *d_small = nullptr;  //   [2 + 2j] max row nnz (fused; written by k_publish)
     std::vector<int64_t> chunk_maxb;  // fused: max row bound per chunk
+    std::vector<int> tiers_sym, tiers_num;  // per unit: tier bits launched (profile statistics)
 
     int64_t *h_rp = nullptr;
     int32_t *h_col = nullptr;

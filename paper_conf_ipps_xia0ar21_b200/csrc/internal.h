@@ -44,6 +44,9 @@ constexpr int PIECE_SYM = 8192, PIECE_NUM = 4096;   // target bound / nnz per co
 constexpr int64_t CAPS_SYM = 32 * int64_t(PIECE_SYM), CAPS_NUM = 32 * int64_t(PIECE_NUM);  // <= 32 pieces
 constexpr int CURSOR_MAX = 32768;          // longest A row a pieced row may have (cursor scratch)
 constexpr int THREADS_G = 512;
+// dense tier, split rows: a row is accumulated by KG_PARTS CTAs (1/KG_PARTS of its A entries each)
+// into its own dense slot, then swept in KG_SWEEP column ranges by as many CTAs
+constexpr int KG_PARTS = 8, KG_SWEEP = 16, THREADS_G2 = 256;
 constexpr int ROW_BATCH = 16;              // rows a warp claims per atomic in the W kernels
 
 // Per-pass control block in the arena (zeroed with cudaMemsetAsync before each pass).
@@ -88,9 +91,10 @@ struct SymArgs {
     int32_t *listB, *listG;
     int32_t *listM;      // medium tier (NULL: those rows go to the B tier)
     Ctl *ctl;
-    uint32_t *gscratch;  // G tier: per-CTA bitmap of ceil(ncols/32) words, zero on entry and exit
-    int64_t gstride;     // words per CTA slot
-    int gblocks;         // CTAs in the G kernel
+    uint32_t *gscratch;  // G tier: per-slot bitmap of ceil(ncols/32) words, zero on entry and exit
+    int64_t gstride;     // words per slot
+    int gblocks;         // dense slots (= CTAs of the one-CTA-per-row G kernel)
+    unsigned long long *gcnt;  // G tier: per slot a counter + KG_SWEEP range counts, zero on entry and exit
     int32_t *cursor;     // B tier, pieced rows: per-CTA 2 x curstride int32 cursors (NULL: none)
     int64_t curstride;
     int bblocks;         // CTAs in the B kernel (the cursor scratch holds that many slots)
@@ -149,10 +153,11 @@ struct NumArgs {
     int32_t *listB, *listG;
     int32_t *listM;      // as in SymArgs
     Ctl *ctl;
-    uint32_t *gbits;     // G tier scratch: per CTA gstride_bits words of bitmap ...
+    uint32_t *gbits;     // G tier scratch: per slot gstride_bits words of bitmap ...
     double *gvals;       // ... and gstride_vals doubles, all zero on entry and exit
     int64_t gstride_bits, gstride_vals;
     int gblocks;
+    unsigned long long *gcnt;  // as in SymArgs
     int32_t *cursor;     // as in SymArgs (a separate scratch: both passes may run concurrently)
     int64_t curstride;
     int bblocks;

@@ -279,11 +279,10 @@ struct PieceSeg {
 };
 
 template <int NT, bool VALS, int PB, typename SEG, typename F>
-__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
-                                                   const SEG &seg, F &&f) {
+__device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B, int64_t as, int64_t ae,
+                                               ProdSmemT<PB> &sm, const SEG &seg, F &&f) {
     constexpr int PER = PB / NT;
     static_assert(PER * NT == PB, "batch must be a multiple of the CTA size");
-    const int64_t as = A.rp[i], ae = A.rp[i + 1];
     for (int64_t pb = as; pb < ae; pb += PB) {
         const int nb = (int)(ae - pb < PB ? ae - pb : PB);
         int64_t lens[PER];
@@ -366,10 +365,17 @@ __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR
     }
 }
 
+// all products of row i (A entries [A.rp[i], A.rp[i+1]))
+template <int NT, bool VALS, int PB, typename SEG, typename F>
+__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
+                                                   const SEG &seg, F &&f) {
+    range_products<NT, VALS>(A, B, A.rp[i], A.rp[i + 1], sm, seg, f);
+}
+
 template <int NT, bool VALS, int PB, typename F>
 __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
                                                    F &&f) {
-    block_row_products<NT, VALS>(A, B, i, sm, WholeSeg{}, f);
+    range_products<NT, VALS>(A, B, A.rp[i], A.rp[i + 1], sm, WholeSeg{}, f);
 }
 
 // find-or-insert of a column in a warp-private table; returns the slot
@@ -828,7 +834,9 @@ __global__ void __launch_bounds__(THREADS_G) k_sym_g(SymArgs a) {
     const unsigned n = *(volatile unsigned *)&a.ctl->nG;
     const int64_t nwords = (a.B.ncols + 31) / 32;
     __shared__ unsigned s_idx;
-    for (unsigned idx = cta_claim(&a.ctl->gctr, &s_idx); idx < n; idx = cta_claim(&a.ctl->gctr, &s_idx)) {
+    // the first gblocks rows of the list were done by the split kernels (k_sym_g1 / g2)
+    for (unsigned idx = a.gblocks + cta_claim(&a.ctl->gctr, &s_idx); idx < n;
+         idx = a.gblocks + cta_claim(&a.ctl->gctr, &s_idx)) {
         const int64_t i = a.listG[idx];
         int cnt = 0;
         block_row_products<THREADS_G, false>(a.A, a.B, i, psm, [&](int32_t c, double) {
@@ -852,6 +860,152 @@ __global__ void __launch_bounds__(THREADS_G) k_sym_g(SymArgs a) {
         }
         __syncthreads();
     }
+}
+
+// ------------------------------------------------------------------- S4 / S6 dense tier, split rows
+//
+// A dense-tier row (beyond the pieced CTA tier: the hubs of C3-C5, up to 3e6 products each) is
+// shared by KG_PARTS CTAs, each taking 1/KG_PARTS of the row's A entries, all accumulating into
+// the row's own dense slot (bitmap + fp64 over all columns, L2 atomics); the slot is then swept
+// in KG_SWEEP column ranges by as many CTAs (numeric: a count kernel and a write kernel, the
+// ranges' offsets from the counts).  One CTA per row made every unit wait for its largest hub:
+// C3 has ~60 such rows per unit, so most SMs idled (ncu: 25 % warps active) and the tier took
+// 0.8 s of a 3 s step.  Row r of the tier's list uses slot r (r < gblocks); the list's rows
+// beyond the slots take the one-CTA-per-row kernels (k_sym_g / k_num_g) afterwards.
+
+__device__ __forceinline__ void part_range(const DevCSR &A, int64_t i, int64_t &p0, int64_t &p1) {
+    const int64_t as = A.rp[i], d = A.rp[i + 1] - as;
+    p0 = as + d * blockIdx.y / gridDim.y;
+    p1 = as + d * (blockIdx.y + 1) / gridDim.y;
+}
+
+__global__ void __launch_bounds__(THREADS_G) k_sym_g1(SymArgs a) {
+    const unsigned n = *(volatile unsigned *)&a.ctl->nG, r = blockIdx.x;
+    if (r >= n || r >= (unsigned)a.gblocks) return;
+    __shared__ ProdSmem psm;
+    __shared__ int s_cnt;
+    const int64_t i = a.listG[r];
+    uint32_t *bm = a.gscratch + (int64_t)r * a.gstride;
+    int64_t p0, p1;
+    part_range(a.A, i, p0, p1);
+    if (threadIdx.x == 0) s_cnt = 0;
+    __syncthreads();
+    int cnt = 0;
+    range_products<THREADS_G, false>(a.A, a.B, p0, p1, psm, WholeSeg{}, [&](int32_t c, double) {
+        const uint32_t bit = 1u << (c & 31);
+        cnt += (atomicOr(&bm[c >> 5], bit) & bit) ? 0 : 1;  // fresh column: the bit was clear
+    });
+    cnt = warp_sum(cnt);
+    if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(&s_cnt, cnt);
+    __syncthreads();
+    if (threadIdx.x == 0 && s_cnt) atomicAdd(&a.gcnt[r * (KG_SWEEP + 1)], (unsigned long long)s_cnt);
+}
+
+// the row's nnz out, the slot's bitmap range cleared
+__global__ void __launch_bounds__(THREADS_G2) k_sym_g2(SymArgs a) {
+    const unsigned n = *(volatile unsigned *)&a.ctl->nG, r = blockIdx.x;
+    if (r >= n || r >= (unsigned)a.gblocks) return;
+    const int64_t nwords = (a.B.ncols + 31) / 32;
+    uint32_t *bm = a.gscratch + (int64_t)r * a.gstride;
+    const int64_t w0 = nwords * blockIdx.y / gridDim.y, w1 = nwords * (blockIdx.y + 1) / gridDim.y;
+    for (int64_t w = w0 + threadIdx.x; w < w1; w += THREADS_G2) bm[w] = 0u;
+    if (blockIdx.y == 0 && threadIdx.x == 0) {
+        const int64_t i = a.listG[r];
+        unsigned long long *gc = &a.gcnt[r * (KG_SWEEP + 1)];
+        const unsigned long long tot = *gc;
+        *gc = 0;
+        a.nnz[i] = (int32_t)tot;
+        atomicMax(&a.ctl->max_nnz, tot);
+        atomicMax(&a.ctl->pass_max, tot);
+        atomicAdd(&a.ctl->rows_g, 1ull);
+    }
+}
+
+__global__ void __launch_bounds__(THREADS_G) k_num_g1(NumArgs a) {
+    const unsigned n = *(volatile unsigned *)&a.ctl->nG, r = blockIdx.x;
+    if (r >= n || r >= (unsigned)a.gblocks) return;
+    __shared__ ProdSmem psm;
+    const int64_t i = a.listG[r];
+    uint32_t *bm = a.gbits + (int64_t)r * a.gstride_bits;
+    double *dv = a.gvals + (int64_t)r * a.gstride_vals;
+    int64_t p0, p1;
+    part_range(a.A, i, p0, p1);
+    range_products<THREADS_G, true>(a.A, a.B, p0, p1, psm, WholeSeg{}, [&](int32_t c, double v) {
+        atomicOr(&bm[c >> 5], 1u << (c & 31));
+        atomicAdd(&dv[c], v);
+    });
+}
+
+// set bits of each column range of the slot
+__global__ void __launch_bounds__(THREADS_G2) k_num_g2(NumArgs a) {
+    const unsigned n = *(volatile unsigned *)&a.ctl->nG, r = blockIdx.x;
+    if (r >= n || r >= (unsigned)a.gblocks) return;
+    __shared__ int64_t s_scan[40];
+    const int64_t nwords = (a.B.ncols + 31) / 32;
+    const uint32_t *bm = a.gbits + (int64_t)r * a.gstride_bits;
+    const int64_t w0 = nwords * blockIdx.y / gridDim.y, w1 = nwords * (blockIdx.y + 1) / gridDim.y;
+    int64_t c = 0;
+    for (int64_t w = w0 + threadIdx.x; w < w1; w += THREADS_G2) c += __popc(__ldcg(&bm[w]));
+    int64_t tot;
+    block_excl_scan<THREADS_G2>(c, s_scan, &tot);
+    if (threadIdx.x == 0) a.gcnt[r * (KG_SWEEP + 1) + 1 + blockIdx.y] = (unsigned long long)tot;
+}
+
+// each column range written at its offset in the row (sorted: ranges and bits in column order);
+// the slot range restored to zero
+__global__ void __launch_bounds__(THREADS_G2) k_num_g3(NumArgs a) {
+    const unsigned n = *(volatile unsigned *)&a.ctl->nG, r = blockIdx.x;
+    if (r >= n || r >= (unsigned)a.gblocks) return;
+    __shared__ int64_t s_scan[40];
+    const int64_t i = a.listG[r];
+    const int64_t o = a.crp[i], len = a.crp[i + 1] - o;
+    const int64_t off0 = a.crp[a.r0];
+    int32_t *oc = a.out_col + (o - off0);
+    double *ov = a.out_val + (o - off0);
+    const int64_t nwords = (a.B.ncols + 31) / 32;
+    uint32_t *bm = a.gbits + (int64_t)r * a.gstride_bits;
+    double *dv = a.gvals + (int64_t)r * a.gstride_vals;
+    unsigned long long *gc = &a.gcnt[r * (KG_SWEEP + 1) + 1];
+    int64_t cnt = 0, all = 0;
+    for (int k = 0; k < (int)gridDim.y; ++k) {
+        const int64_t ck = (int64_t)gc[k];
+        if (k < (int)blockIdx.y) cnt += ck;
+        all += ck;
+    }
+    const int64_t w0 = nwords * blockIdx.y / gridDim.y, w1 = nwords * (blockIdx.y + 1) / gridDim.y;
+    for (int64_t wb = w0; wb < w1; wb += THREADS_G2) {
+        const int64_t w = wb + threadIdx.x;
+        uint32_t word = w < w1 ? __ldcg(&bm[w]) : 0u;
+        int64_t tot;
+        const int64_t ex = block_excl_scan<THREADS_G2>(__popc(word), s_scan, &tot);
+        if (word) {
+            int64_t pos = cnt + ex;
+            bm[w] = 0u;
+            while (word) {
+                const int b = __ffs(word) - 1;
+                word &= word - 1;
+                const int64_t c = w * 32 + b;
+                if (pos < len) {
+                    oc[pos] = (int32_t)c;
+                    ov[pos] = __ldcg(&dv[c]);
+                }
+                dv[c] = 0.0;
+                ++pos;
+            }
+        }
+        cnt += tot;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (blockIdx.y + 1 == gridDim.y && all != len) atomicOr(&a.ctl->err, 1u);
+    }
+}
+
+__global__ void k_gcnt_clear(unsigned long long *gcnt, const Ctl *ctl, int slots) {
+    // numeric range counts of the used slots back to zero (after k_num_g3 read them)
+    const unsigned n = min(*(volatile const unsigned *)&ctl->nG, (unsigned)slots);
+    for (unsigned t = blockIdx.x * blockDim.x + threadIdx.x; t < n * (KG_SWEEP + 1); t += gridDim.x * blockDim.x)
+        gcnt[t] = 0ull;
 }
 
 // ------------------------------------------------------------------------------------- S5 scan
@@ -1534,7 +1688,9 @@ __global__ void __launch_bounds__(THREADS_G) k_num_g(NumArgs a) {
     const int64_t nwords = (a.B.ncols + 31) / 32;
     const int64_t off0 = a.crp[a.r0];
     __shared__ unsigned s_idx;
-    for (unsigned idx = cta_claim(&a.ctl->gctr, &s_idx); idx < nrows; idx = cta_claim(&a.ctl->gctr, &s_idx)) {
+    // the first gblocks rows of the list were done by the split kernels (k_num_g1 .. g3)
+    for (unsigned idx = a.gblocks + cta_claim(&a.ctl->gctr, &s_idx); idx < nrows;
+         idx = a.gblocks + cta_claim(&a.ctl->gctr, &s_idx)) {
         const int64_t i = a.listG[idx];
         const int64_t o = a.crp[i];
         const int64_t n = a.crp[i + 1] - o;
@@ -1739,8 +1895,10 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
     // cursor scratch (possible whenever the pass has CTA-tier rows; the kernel exits at once
     // when its list is empty)
     if ((a.tiers & 3) && a.gblocks > 0) {
-        k_sym_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
-        LAUNCHED(1);
+        k_sym_g1<<<dim3(a.gblocks, KG_PARTS), THREADS_G, 0, s>>>(a);
+        k_sym_g2<<<dim3(a.gblocks, KG_SWEEP), THREADS_G2, 0, s>>>(a);
+        k_sym_g<<<a.gblocks, THREADS_G, 0, s>>>(a);  // rows beyond the slots (usually none)
+        LAUNCHED(3);
     }
     rec(ev, 4, s);
 }
@@ -1780,8 +1938,12 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
     }
     rec(ev, 3, s);
     if ((a.tiers & 3) && a.gblocks > 0) {
-        k_num_g<<<a.gblocks, THREADS_G, 0, s>>>(a);
-        LAUNCHED(1);
+        k_num_g1<<<dim3(a.gblocks, KG_PARTS), THREADS_G, 0, s>>>(a);
+        k_num_g2<<<dim3(a.gblocks, KG_SWEEP), THREADS_G2, 0, s>>>(a);
+        k_num_g3<<<dim3(a.gblocks, KG_SWEEP), THREADS_G2, 0, s>>>(a);
+        k_gcnt_clear<<<grid_for(int64_t(a.gblocks) * (KG_SWEEP + 1), 256, 148), 256, 0, s>>>(a.gcnt, a.ctl, a.gblocks);
+        k_num_g<<<a.gblocks, THREADS_G, 0, s>>>(a);  // rows beyond the slots (usually none)
+        LAUNCHED(5);
     }
     rec(ev, 4, s);
 }

@@ -320,6 +320,8 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
         P->gbits = P->alloc<uint32_t>(P->gstride_bits, "dense-tier bitmap (numeric)");
         P->gbits_sym = P->alloc<uint32_t>(P->gstride_bits, "dense-tier bitmap (symbolic)");
         P->gvals = P->alloc<double>(P->gstride_vals, "dense-tier values");
+        P->gcnt = P->alloc<unsigned long long>(2 * (KG_SWEEP + 1), "dense-tier counters");
+        CK(cudaMemsetAsync(P->gcnt, 0, sizeof(unsigned long long) * 2 * (KG_SWEEP + 1), s));
         CK(cudaMemsetAsync(P->gbits, 0, size_t(P->gstride_bits) * 4, s));
         CK(cudaMemsetAsync(P->gbits_sym, 0, size_t(P->gstride_bits) * 4, s));
         CK(cudaMemsetAsync(P->gvals, 0, size_t(P->gstride_vals) * 8, s));
@@ -465,6 +467,8 @@ void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const
             sa.listG = P->listG;
             sa.ctl = P->ctl;
             sa.gscratch = P->gbits_sym;
+            sa.gcnt = P->gcnt;
+    sa.gcnt = P->gcnt;
             sa.gstride = P->gstride_bits;
             sa.gblocks = P->gblocks;
             sa.cursor = P->cur_sym;
@@ -624,6 +628,8 @@ int64_t panel_run(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double *v
             na.ctl = P->ctl + 1;
             na.gbits = P->gbits;
             na.gvals = P->gvals;
+            na.gcnt = P->gcnt ? P->gcnt + size_t(P->gblocks) * (KG_SWEEP + 1) : nullptr;
+    na.gcnt = P->gcnt ? P->gcnt + size_t(P->gblocks) * (KG_SWEEP + 1) : nullptr;
             na.gstride_bits = P->gstride_bits;
             na.gstride_vals = P->gstride_vals;
             na.gblocks = P->gblocks;

@@ -206,6 +206,28 @@ def test_pieced_cta_tier_and_dense_tier(fused):
     assert_parity(A, B, r[0], r[1], r[2])
 
 
+@pytest.mark.parametrize("slots", [None, "2"])
+@pytest.mark.parametrize("fused", [False, True])
+def test_dense_tier_split_rows(fused, slots, monkeypatch):
+    """Rows beyond the pieced CTA tier (> 32 pieces: the C3 hubs) are shared by several CTAs per
+    row and swept in column ranges; with only 2 dense slots (test hook) the rows beyond the
+    slots take the one-CTA-per-row kernels.  Rows of different lengths, an empty row between."""
+    if slots:
+        monkeypatch.setenv("SPGEMM_MAX_GSLOTS", slots)
+    rng = np.random.default_rng(41)
+    ncols = 600_000
+    brows = [np.sort(rng.choice(ncols, int(rng.integers(200, 900), ), replace=False)) for _ in range(3000)]
+    B = _csr_from_rows(brows, ncols, rng)
+    arows = []
+    for i in range(9):
+        d = [600, 700, 0, 1000, 650, 3, 800, 720, 850][i]   # ~330K-550K products per row
+        arows.append(np.sort(rng.choice(B.nrows, d, replace=False)))
+    A = _csr_from_rows(arows, B.nrows, rng)
+    r = run_fused(A, B) if fused else run(A, B)
+    assert r[3]["rows_global"] >= 6, r[3]
+    assert_parity(A, B, r[0], r[1], r[2])
+
+
 @pytest.mark.parametrize("fused", [False, True])
 def test_pieced_rows_many_entries_and_dense_fallback(fused):
     """Pieced rows whose A rows hold many entries (cursor scratch per entry), one A row longer than
