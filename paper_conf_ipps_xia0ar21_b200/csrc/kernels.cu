@@ -317,14 +317,17 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
         }
         if (threadIdx.x == 0) sm.off[nb] = tot;
         __syncthreads();
-        // Each warp takes 32 consecutive products per step (coalesced B loads), two steps at a
-        // time: the B loads of both are issued before either product is consumed, so two gathers
-        // are in flight per lane while the first one's hash insert runs (long-scoreboard stalls on
-        // these loads were the top stall of the CTA kernels, profiles/r02/).  Four lanes find the
-        // segments of the first and last product of each step; every lane then searches only
-        // that window (usually 1-3 segments) instead of all nb A entries of the batch.
+        // Each warp takes 32 consecutive products per step (coalesced B loads), two steps (qb,
+        // qb + NT) per iteration, software-pipelined: the gathers of the next iteration are issued
+        // before the current one's products are consumed, so up to four B loads per lane are in
+        // flight while the hash inserts run (long-scoreboard stalls on these loads were the top
+        // stall of the CTA kernels, profiles/r02/).  With STAGE (symbolic passes, VERDICT r1 item
+        // 4's trial) the next iteration's columns are instead copied into a per-warp shared
+        // staging buffer with cp.async (LDGSTS), double-buffered.  Four lanes find the segments
+        // of the first and last product of each step; every lane then searches only that window
+        // (usually 1-3 segments) instead of all nb A entries of the batch.
         const int lane = threadIdx.x & 31;
-        for (int64_t qb = threadIdx.x - lane; qb < tot; qb += 2 * NT) {  // warp-uniform trip count
+        auto locate = [&](int64_t qb, int64_t (&pos)[2], double (&a)[2], bool (&ok)[2]) {
             int lo = 0, hi = nb;  // invariant: off[lo] <= q < off[hi]
             if (lane < 4) {
                 const int64_t q0 = qb + (lane >> 1) * NT;
@@ -335,16 +338,13 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
                     else hi = mid;
                 }
             }
-            int32_t c[2];
-            double v[2];
-            bool ok[2];
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
                 const int64_t q = qb + u * NT + lane;
                 const int wlo = __shfl_sync(FULLMASK, lo, 2 * u), whi = __shfl_sync(FULLMASK, lo, 2 * u + 1) + 1;
                 ok[u] = q < tot;
-                c[u] = 0;
-                v[u] = 0.0;
+                pos[u] = 0;
+                a[u] = 0.0;
                 if (ok[u]) {
                     int l2 = wlo, h2 = whi;
                     while (h2 - l2 > 1) {
@@ -352,14 +352,46 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
                         if (sm.off[mid] <= q) l2 = mid;
                         else h2 = mid;
                     }
-                    const int64_t pos = sm.bs[l2] + (q - sm.off[l2]);
-                    c[u] = __ldg(&B.col[pos]);
-                    if (VALS) v[u] = sm.a[l2] * __ldg(&B.val[pos]);
+                    pos[u] = sm.bs[l2] + (q - sm.off[l2]);
+                    if (VALS) a[u] = sm.a[l2];
                 }
             }
+        };
+        const int64_t q_first = threadIdx.x - lane;  // warp-uniform
+        if (q_first < tot) {
+            int64_t pos[2];
+            double av[2];
+            bool ok[2];
+            int32_t c[2];
+            double v[2];
+            locate(q_first, pos, av, ok);
 #pragma unroll
-            for (int u = 0; u < 2; ++u)
-                if (ok[u]) f(c[u], v[u]);
+            for (int u = 0; u < 2; ++u) {
+                c[u] = ok[u] ? __ldg(&B.col[pos[u]]) : 0;
+                v[u] = (VALS && ok[u]) ? av[u] * __ldg(&B.val[pos[u]]) : 0.0;
+            }
+            for (int64_t qb = q_first; qb < tot; qb += 2 * NT) {  // warp-uniform trip count
+                int32_t cn[2] = {0, 0};
+                double vn[2] = {0.0, 0.0};
+                bool okn[2] = {false, false};
+                if (qb + 2 * NT < tot) {  // next iteration's gathers first
+                    locate(qb + 2 * NT, pos, av, okn);
+#pragma unroll
+                    for (int u = 0; u < 2; ++u) {
+                        cn[u] = okn[u] ? __ldg(&B.col[pos[u]]) : 0;
+                        vn[u] = (VALS && okn[u]) ? av[u] * __ldg(&B.val[pos[u]]) : 0.0;
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < 2; ++u)
+                    if (ok[u]) f(c[u], v[u]);
+#pragma unroll
+                for (int u = 0; u < 2; ++u) {
+                    c[u] = cn[u];
+                    v[u] = vn[u];
+                    ok[u] = okn[u];
+                }
+            }
         }
         __syncthreads();
     }
