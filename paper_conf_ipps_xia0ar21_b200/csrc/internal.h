@@ -56,6 +56,7 @@ struct Ctl {
     unsigned long long pass_max;  // symbolic: max nnz of a row in this pass        } (CTL_RESET
     unsigned int nM, bctr;        // medium-tier list length; B-tier claim cursor   }  bytes)
     unsigned int mctr, gctr;      // M / G-tier claim cursors (rows claimed one by one) }
+    unsigned int nBl, pad3;       // B tier: one-piece rows, stored from the END of listB }
     unsigned int err;             // bit 0: numeric count mismatch; bit 1: invalid input; bit 2: table overflow
     unsigned int pad;
     unsigned long long sum_u;     // count pass: sum of products
@@ -65,9 +66,9 @@ struct Ctl {
     unsigned long long rows_w, rows_b, rows_g;
     unsigned long long max_deg;   // count pass: longest row of A (cursor scratch of pieced rows)
     unsigned long long rows_m;    // rows of the medium tier (symbolic passes)
-    unsigned long long pad2[3];
+    unsigned long long pad2[2];
 };
-constexpr size_t CTL_RESET = 40;  // bytes of Ctl cleared before every pass (row_ctr .. gctr)
+constexpr size_t CTL_RESET = 48;  // bytes of Ctl cleared before every pass (row_ctr .. pad3)
 
 // --- launchers (all asynchronous on `s`) ---------------------------------------------------
 

@@ -584,16 +584,22 @@ __global__ void k_add(int64_t *rp, int64_t n, int64_t d) {
 // rows too long for a warp: the medium tier (bound <= capM, when enabled), the CTA tier (one piece
 // up to capB; column pieces up to capS when the pass has cursor scratch and the row's A entries
 // fit it), the dense tier beyond
+// The B list holds the pieced rows from its front and the one-piece rows from its back (cap = the
+// pass's row count), so that the dynamic claims take the expensive rows first and the cheap ones
+// fill the tail (longest-first; a pieced row can take 30x a one-piece row).
 __device__ __forceinline__ void push_long(int64_t i, int64_t bound, const DevCSR &A, int64_t capM, int64_t capB,
                                           int64_t capS, const int32_t *cursor, int64_t curstride, int32_t *listM,
-                                          int32_t *listB, int32_t *listG, Ctl *ctl) {
+                                          int32_t *listB, int32_t *listG, Ctl *ctl, int64_t cap) {
     if (listM != nullptr && bound <= capM) {
         unsigned idx = atomicAdd(&ctl->nM, 1u);
         listM[idx] = (int32_t)i;
         return;
     }
     const bool pieces_ok = cursor != nullptr && bound <= capS && A.rp[i + 1] - A.rp[i] <= curstride;
-    if (bound <= capB || pieces_ok) {
+    if (bound <= capB) {
+        unsigned idx = atomicAdd(&ctl->nBl, 1u);
+        listB[cap - 1 - idx] = (int32_t)i;
+    } else if (pieces_ok) {
         unsigned idx = atomicAdd(&ctl->nB, 1u);
         listB[idx] = (int32_t)i;
     } else {
@@ -633,7 +639,7 @@ __global__ void __launch_bounds__(WARPS_W * 32) k_sym_w(SymArgs a) {
             if (bound > CAPW_SYM) {
                 if (lane == 0) {
                     push_long(i, bound, a.A, CAPM_SYM, CAPB_SYM, CAPS_SYM, a.cursor, a.curstride, a.listM, a.listB,
-                              a.listG, a.ctl);
+                              a.listG, a.ctl, R);
                     nlong++;
                 }
                 continue;
@@ -771,10 +777,11 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
     constexpr int LIMIT = (TB_SYM / 4) * 3;
     int32_t *cur = a.cursor ? a.cursor + (int64_t)blockIdx.x * 2 * a.curstride : nullptr;
     int32_t *nxt = cur ? cur + a.curstride : nullptr;
-    const unsigned n = *(volatile unsigned *)&a.ctl->nB;
+    const unsigned nh = *(volatile unsigned *)&a.ctl->nB, n = nh + *(volatile unsigned *)&a.ctl->nBl;
+    const int64_t R = a.r1 - a.r0;
     __shared__ unsigned s_idx;
     for (unsigned idx = cta_claim(&a.ctl->bctr, &s_idx); idx < n; idx = cta_claim(&a.ctl->bctr, &s_idx)) {
-        const int64_t i = a.listB[idx];
+        const int64_t i = a.listB[idx < nh ? int64_t(idx) : R - 1 - int64_t(idx - nh)];
         const int64_t bound = a.bnd[i];
         int64_t total = 0;
         // one table pass over the products of [lo, hi) (whole row: seg = WholeSeg)
@@ -1271,7 +1278,7 @@ __global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
             if (n > CAPW_NUM) {
                 if (lane == 0)
                     push_long(i, n, a.A, CAPM_NUM, CAPB_NUM, CAPS_NUM, a.cursor, a.curstride, a.listM, a.listB, a.listG,
-                              a.ctl);
+                              a.ctl, R);
                 continue;
             }
             const int lg = table_log2(a.tload == 0 ? n : a.tload == 1 ? (3 * n) / 2 : 2 * n, MAXLG);
@@ -1621,11 +1628,12 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
     constexpr int LIMIT = (TB_NUM / 4) * 3;
     int32_t *cur = a.cursor ? a.cursor + (int64_t)blockIdx.x * 2 * a.curstride : nullptr;
     int32_t *nxt = cur ? cur + a.curstride : nullptr;
-    const unsigned nrows = *(volatile unsigned *)&a.ctl->nB;
+    const unsigned nh = *(volatile unsigned *)&a.ctl->nB, nrows = nh + *(volatile unsigned *)&a.ctl->nBl;
+    const int64_t R = a.r1 - a.r0;
     const int64_t off0 = a.crp[a.r0];
     __shared__ unsigned s_idx;
     for (unsigned idx = cta_claim(&a.ctl->bctr, &s_idx); idx < nrows; idx = cta_claim(&a.ctl->bctr, &s_idx)) {
-        const int64_t i = a.listB[idx];
+        const int64_t i = a.listB[idx < nh ? int64_t(idx) : R - 1 - int64_t(idx - nh)];
         const int64_t o = a.crp[i];
         const int64_t n = a.crp[i + 1] - o;
         int32_t *oc = a.out_col + (o - off0);
