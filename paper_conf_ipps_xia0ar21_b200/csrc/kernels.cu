@@ -1532,22 +1532,32 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
                     stg[pos] = ((d & relmask) << SB) | (uint32_t)(j * NT + threadIdx.x);
                 }
             __syncthreads();
-            // rank among the bucket's staged words (bucket b = [end(b - 1), end(b))); column and
-            // value to the final position
-#pragma unroll
-            for (int j = 0; j < SPT; ++j)
-                if (kr[j] != EMPTY) {
-                    const int t = j * NT + threadIdx.x;
-                    const uint32_t d = (uint32_t)((int64_t)kr[j] - lo);
-                    const uint32_t x = ((d & relmask) << SB) | (uint32_t)t;
-                    const uint32_t b = d >> sh;
-                    const int e0 = (int)((sc.arr[b >> 1] >> ((b & 1u) << 4)) & 0xffffu);
-                    const int s0 = b == 0 ? 0 : (int)((sc.arr[(b - 1) >> 1] >> (((b - 1) & 1u) << 4)) & 0xffffu);
-                    int r = s0;
-                    for (int q = s0; q < e0; ++q) r += stg[q] < x;
-                    oc[r] = kr[j];
-                    ov[r] = vals[t];
+            // every bucket b = [end(b - 1), end(b)) sorted in place by its owner thread (b mod NT;
+            // ~1 key per bucket, so mostly nothing to do) and written out: consecutive lanes own
+            // consecutive buckets, so one-key buckets give coalesced stores.  (Ranking every key
+            // against its bucket-mates made each warp wait for its lane with the largest bucket:
+            // 17 % of num_b's instructions, profiles/r02/ncu_numb_c3_v4.)
+            const int nb_used = (int)(((span - 1) >> sh) + 1);
+            const uint32_t slotmask = (1u << SB) - 1u;
+            for (int b = threadIdx.x; b < nb_used; b += NT) {
+                const int e0 = (int)((sc.arr[b >> 1] >> ((b & 1) << 4)) & 0xffffu);
+                const int s0 = b == 0 ? 0 : (int)((sc.arr[(b - 1) >> 1] >> (((b - 1) & 1) << 4)) & 0xffffu);
+                for (int p = s0 + 1; p < e0; ++p) {  // insertion sort of the bucket's staged words
+                    const uint32_t v = stg[p];
+                    int q = p - 1;
+                    while (q >= s0 && stg[q] > v) {
+                        stg[q + 1] = stg[q];
+                        --q;
+                    }
+                    stg[q + 1] = v;
                 }
+                const int64_t cb = lo + ((int64_t)b << sh);
+                for (int p = s0; p < e0; ++p) {
+                    const uint32_t x = stg[p];
+                    oc[p] = (int32_t)(cb + (x >> SB));
+                    ov[p] = vals[x & slotmask];
+                }
+            }
             __syncthreads();
             return true;
         }
