@@ -1379,7 +1379,7 @@ __global__ void __launch_bounds__(WARPS_W * 32, 4) k_num_w(NumArgs a) {
 
 template <int NT>
 struct CtaSortSmemT {
-    int cnt[64], cur[64], start[64], mm[3], occ[NT / 32];
+    int mm[3], occ[NT / 32];
     int64_t scan[40];
 };
 using CtaSortSmem = CtaSortSmemT<THREADS_B>;
@@ -1390,7 +1390,12 @@ using CtaSortSmem = CtaSortSmemT<THREADS_B>;
 // a table is sorted).
 template <int NT>
 struct SortCntT {
-    uint32_t arr[4 * NT];
+    union {
+        uint32_t arr[4 * NT];
+        struct {
+            int cnt[64], cur[64], start[64];  // coarse buckets of the clustered-column fallback
+        } co;
+    };
 };
 using SortCnt = SortCntT<THREADS_B>;
 template <int NT, int PB>
@@ -1430,13 +1435,12 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     constexpr int NW = NT / 32;
     constexpr int SPT = (1 << SB) / NT;  // table slots per thread
     static_assert(SPT * NT == (1 << SB), "table size must be a multiple of the CTA size");
-    constexpr int PLMAX = NT == 512 ? 12 : NT == 256 ? 11 : NT == 128 ? 10 : 9;  // 2^PLMAX = 8 NT buckets
+    constexpr int PLMAX = NT == 1024 ? 13 : NT == 512 ? 12 : NT == 256 ? 11 : NT == 128 ? 10 : 9;  // 2^PLMAX = 8 NT
     static_assert((1 << PLMAX) == 8 * NT, "eight fine buckets per thread");
     // fine buckets (~1 key each): 2^pl of them, bucket of key k = (k - lo) >> sh
     const int pl = min(PLMAX, max(5, 32 - __clz((int)max((int64_t)1, n) - 1)));
     for (int w = threadIdx.x; w < (1 << (pl - 1)); w += NT) sc.arr[w] = 0u;
     const int P = min(64, max(1, (int)((n + 255) / 256)));
-    if (threadIdx.x < 64) ss.cnt[threadIdx.x] = 0;
     if (threadIdx.x == 0) {
         ss.mm[0] = INT_MAX;
         ss.mm[1] = -1;
@@ -1563,17 +1567,20 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         }
     }
     // skewed columns (a fine bucket over 64 keys): coarse buckets sorted by warps in registers
+    // (their counters alias the fine-bucket cursors, no longer read past the last barrier)
+    if (threadIdx.x < 64) sc.co.cnt[threadIdx.x] = 0;
+    __syncthreads();
     for (int t = threadIdx.x; t < T; t += NT) {
         const int32_t k = keys[t];
-        if (k != EMPTY) atomicAdd(&ss.cnt[(int)(((int64_t)k - lo) * P / span)], 1);
+        if (k != EMPTY) atomicAdd(&sc.co.cnt[(int)(((int64_t)k - lo) * P / span)], 1);
     }
     __syncthreads();
     if (wid == 0) {  // bucket starts (lane l owns buckets l and l + 32) and the largest bucket
-        const int c0 = lane < P ? ss.cnt[lane] : 0, c1 = lane + 32 < P ? ss.cnt[lane + 32] : 0;
+        const int c0 = lane < P ? sc.co.cnt[lane] : 0, c1 = lane + 32 < P ? sc.co.cnt[lane + 32] : 0;
         const int i0 = warp_incl_scan(c0), i1 = warp_incl_scan(c1);
         const int tot0 = __shfl_sync(FULLMASK, i0, 31);
-        if (lane < P) ss.start[lane] = ss.cur[lane] = i0 - c0;
-        if (lane + 32 < P) ss.start[lane + 32] = ss.cur[lane + 32] = tot0 + i1 - c1;
+        if (lane < P) sc.co.start[lane] = sc.co.cur[lane] = i0 - c0;
+        if (lane + 32 < P) sc.co.start[lane + 32] = sc.co.cur[lane + 32] = tot0 + i1 - c1;
         int big = max(c0, c1);
 #pragma unroll
         for (int d = 16; d > 0; d >>= 1) big = max(big, __shfl_xor_sync(FULLMASK, big, d));
@@ -1585,13 +1592,13 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         for (int t = threadIdx.x; t < T; t += NT) {
             const int32_t k = keys[t];
             if (k != EMPTY) {
-                const int pos = atomicAdd(&ss.cur[(int)(((int64_t)k - lo) * P / span)], 1);
+                const int pos = atomicAdd(&sc.co.cur[(int)(((int64_t)k - lo) * P / span)], 1);
                 stage[pos] = ((unsigned long long)(uint32_t)k << SB) | (unsigned)t;
             }
         }
         __syncthreads();  // staged keys (global) visible to the block
         for (int b = wid; b < P; b += NW) {
-            const int st = ss.start[b], m = ss.cnt[b];
+            const int st = sc.co.start[b], m = sc.co.cnt[b];
             if (m == 0) continue;
             sort_emit_any<SB, true, false>(stage + st, m, vals, oc + st, ov + st);
         }
@@ -1626,15 +1633,16 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     return true;
 }
 
-__global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
+__global__ void __launch_bounds__(THREADS_BN, 1024 / THREADS_BN) k_num_b(NumArgs a) {
     extern __shared__ __align__(16) double smem_d[];
     double *vals = smem_d;
     int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);
-    __shared__ ProdOrSort u;
-    ProdSmem &psm = u.psm;
-    __shared__ CtaSortSmem ss;
+    __shared__ ProdOrSortT<THREADS_BN, PBATCH_BN> u;
+    ProdSmemT<PBATCH_BN> &psm = u.psm;
+    __shared__ CtaSortSmemT<THREADS_BN> ss;
     __shared__ int s_ins, s_ovf, s_span[2];
-    constexpr int MAXLG = 13;  // log2(TB_NUM)
+    constexpr int MAXLG = TB_NUM == 16384 ? 14 : TB_NUM == 8192 ? 13 : TB_NUM == 4096 ? 12 : 11;  // log2(TB_NUM)
+    static_assert((1 << MAXLG) == TB_NUM, "table size");
     constexpr int LIMIT = (TB_NUM / 4) * 3;
     int32_t *cur = a.cursor ? a.cursor + (int64_t)blockIdx.x * 2 * a.curstride : nullptr;
     int32_t *nxt = cur ? cur + a.curstride : nullptr;
@@ -1650,7 +1658,7 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
         double *ov = a.out_val + (o - off0);
         auto pass = [&](int lg, const auto &seg, int limit) {
             const int T = 1 << lg;
-            for (int t = threadIdx.x; t < T; t += THREADS_B) {
+            for (int t = threadIdx.x; t < T; t += THREADS_BN) {
                 keys[t] = EMPTY;
                 vals[t] = 0.0;
             }
@@ -1659,7 +1667,7 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
                 s_ovf = 0;
             }
             __syncthreads();
-            block_row_products<THREADS_B, true>(a.A, a.B, i, psm, seg, [&](int32_t c, double v) {
+            block_row_products<THREADS_BN, true>(a.A, a.B, i, psm, seg, [&](int32_t c, double v) {
                 const int h = insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
                 if (h >= 0) atomicAdd(&vals[h], v);
             });  // ends with a barrier
@@ -1669,15 +1677,15 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_num_b(NumArgs a) {
         if (n <= CAPB_NUM) {
             const int lg = table_log2(n, MAXLG);
             pass(lg, WholeSeg{}, INT_MAX);
-            ok = cta_sort_emit<MAXLG>(keys, vals, 1 << lg, n, oc, ov, ss, u.sc);
+            ok = cta_sort_emit<MAXLG, THREADS_BN>(keys, vals, 1 << lg, n, oc, ov, ss, u.sc);
         } else {
             int64_t written = 0;
-            row_pieces<THREADS_B>(
+            row_pieces<THREADS_BN>(
                 a.A, a.B, i, n, PIECE_NUM, cur, nxt, s_span,
                 [&](int32_t lo, int32_t hi) { return pass(MAXLG, PieceSeg{a.B.col, cur, nxt, hi}, LIMIT); },
                 [&]() {
                     const int m = s_ins;
-                    if (written + m <= n) ok &= cta_sort_emit<MAXLG>(keys, vals, TB_NUM, m, oc + written, ov + written, ss, u.sc);
+                    if (written + m <= n) ok &= cta_sort_emit<MAXLG, THREADS_BN>(keys, vals, TB_NUM, m, oc + written, ov + written, ss, u.sc);
                     else ok = false;
                     written += m;
                 });
@@ -1825,7 +1833,7 @@ const Grids &grids(int device, int num_sms) {
         g.numw_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b, THREADS_B, symb_smem());
         g.symb_blocks = num_sms * (occ > 0 ? occ : 1);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_b, THREADS_B, numb_smem());
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_b, THREADS_BN, numb_smem());
         g.numb_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_m, THREADS_M, symm_smem());
         g.symm_blocks = num_sms * (occ > 0 ? occ : 1);
@@ -1983,7 +1991,7 @@ void launch_numeric(const NumArgs &a, int num_sms, cudaStream_t s, cudaEvent_t *
     }
     rec(ev, 2, s);
     if (a.tiers & 1) {
-        k_num_b<<<a.cursor ? a.bblocks : g.numb_blocks, THREADS_B, numb_smem(), s>>>(a);
+        k_num_b<<<a.cursor ? a.bblocks : g.numb_blocks, THREADS_BN, numb_smem(), s>>>(a);
         LAUNCHED(1);
     }
     rec(ev, 3, s);
