@@ -39,11 +39,13 @@ constexpr int TM_SYM = 4096, CAPM_SYM = 2048;
 constexpr int TM_NUM = 2048, CAPM_NUM = 1024;
 constexpr int THREADS_B = 512;             // 2 CTAs per SM (96 KB / 64 KB of table + 13 KB)
 constexpr int TB_SYM = 16384, CAPB_SYM = 8192;
-// numeric CTA tier: 1024 threads, one CTA per SM with a 16 K-slot table (192 KB + 26 KB)
-constexpr int THREADS_BN = 1024, PBATCH_BN = 1024;
-constexpr int TB_NUM = 16384, CAPB_NUM = 8192;
-constexpr int PIECE_SYM = 8192, PIECE_NUM = 8192;   // target bound / nnz per column piece
-constexpr int64_t CAPS_SYM = 32 * int64_t(PIECE_SYM), CAPS_NUM = 16 * int64_t(PIECE_NUM);  // <= 32 / 16 pieces
+// numeric CTA tier: 512 threads, 2 CTAs per SM (96 KB table + 13 KB each).  Measured on C3
+// (tools/tier_times.py): 256 threads / 4 K slots / pieces of 2048 took 1180 ms, 1024 threads /
+// 16 K slots / pieces of 8192 took 1061 ms, this configuration 997 ms.
+constexpr int THREADS_BN = 512, PBATCH_BN = 512;
+constexpr int TB_NUM = 8192, CAPB_NUM = 4096;
+constexpr int PIECE_SYM = 8192, PIECE_NUM = 4096;   // target bound / nnz per column piece
+constexpr int64_t CAPS_SYM = 32 * int64_t(PIECE_SYM), CAPS_NUM = 32 * int64_t(PIECE_NUM);  // <= 32 pieces
 constexpr int CURSOR_MAX = 32768;          // longest A row a pieced row may have (cursor scratch)
 constexpr int THREADS_G = 512;
 // dense tier, split rows: a row is accumulated by KG_PARTS CTAs (1/KG_PARTS of its A entries each)
