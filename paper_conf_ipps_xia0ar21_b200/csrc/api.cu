@@ -227,6 +227,7 @@ SymArgs sym_args(spgemm_plan_s *P, int64_t r0, int64_t r1, int tiers) {
 }
 
 void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const spgemm_opts *o, spgemm_plan_s *P) {
+    NvtxRange nv("spgemm_plan");
     check_csr(Ah, "A");
     check_csr(Bh, "B");
     if (Ah->ncols != Bh->nrows)
@@ -772,6 +773,7 @@ void do_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const sp
 }
 
 void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t slot_off, int64_t max_row_nnz, cudaEvent_t *ev) {
+    NvtxRange nv("enqueue numeric");
     NumArgs na{};
     na.A = P->A;
     na.B = P->B;
@@ -803,6 +805,7 @@ void enqueue_numeric(spgemm_plan_s *P, int64_t c, int b, int64_t slot_off, int64
 // fused plans: symbolic + scan of chunk j; its end offset and max row nnz land in
 // h_small[1 + 2j], h_small[2 + 2j] through zero-copy stores (no D2H on the copy engine)
 void enqueue_analysis(spgemm_plan_s *P, int64_t j, cudaEvent_t *ev) {
+    NvtxRange nv("enqueue symbolic + scan");
     const int64_t r0 = P->chunk_rows[j], r1 = P->chunk_rows[j + 1];
     cudaStream_t as = P->astream;
     if (P->host_cut) {
@@ -910,6 +913,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
 
 int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double *val_out, int64_t capacity,
                      const Sink *sink, bool *overflow) {
+    NvtxRange nv("spgemm_execute");
     if (P->pan) return run_panels(P, rp_out, col_out, val_out, capacity, sink, overflow);
     if (P->failed) fail(SPGEMM_ERR_STATE, "plan is in a failed state");
     DeviceGuard g(P->device);
@@ -1058,6 +1062,7 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
                     int64_t *rp = st_rp(G.b);
                     const int64_t first = rp[0];
                     for (int64_t k = 0; k <= G.r1 - G.r0; ++k) rp[k] -= first;
+                    NvtxRange cbr("sink callback");
                     rc = sink->cb(sink->user, P->row_begin + G.r0, P->row_begin + G.r1, rp, st_col(G.b), st_val(G.b),
                                   rp[G.r1 - G.r0]);
                 }
@@ -1152,7 +1157,10 @@ int64_t run_pipeline(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double
         if (P->fused) {
             // unit j's symbolic pass was enqueued LOOKAHEAD iterations ago; its total decides where the
             // unit lands on the host and its max row nnz which numeric tiers to launch
-            CK(cudaEventSynchronize(P->ev_tot[j]));
+            {
+                NvtxRange w("wait unit total");
+                CK(cudaEventSynchronize(P->ev_tot[j]));
+            }
             offs[j + 1] = P->h_small[1 + 2 * j] - base;
             mx = P->h_small[2 + 2 * j];
         }

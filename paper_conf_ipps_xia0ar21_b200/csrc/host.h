@@ -3,6 +3,7 @@
 // Not part of the public ABI (include/spgemm.h).
 #pragma once
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <mutex>
 #include <string>
@@ -10,6 +11,17 @@
 
 #include "../../include/spgemm.h"
 #include "internal.h"
+
+// NVTX range for the host side of the pipeline (plan, execute, each unit's enqueue, the wait for a
+// unit's total, every sink callback), so that an Nsight Systems timeline shows the host thread next
+// to the compute / analysis / copy streams.  nvtx3 is header-only: without an attached tool each
+// push/pop is a no-op call.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
 
 namespace spgh {
 using namespace spg;

@@ -166,6 +166,7 @@ DevCSR build_panel(spgemm_plan_s *P, Panels &Q, int j) {
 
 void panel_plan(const spgemm_csr *Ah, const spgemm_csr *Bh, size_t budget, const spgemm_opts *o,
                 spgemm_plan_s *P) {
+    NvtxRange nv("spgemm_plan (column panels)");
     check_csr(Ah, "A");
     check_csr(Bh, "B");
     if (Ah->ncols != Bh->nrows)
@@ -571,6 +572,7 @@ struct HostMap {
 
 int64_t panel_run(spgemm_plan_s *P, int64_t *rp_out, int32_t *col_out, double *val_out, int64_t capacity,
                   const Sink *sink, bool *overflow) {
+    NvtxRange nv("spgemm_execute (column panels)");
     if (P->failed) fail(SPGEMM_ERR_STATE, "plan is in a failed state");
     if (sink) fail(SPGEMM_ERR_INVALID_ARGUMENT, "sink mode is not available with column panels of B (a row of C is "
                                                 "complete only after the last panel)");
