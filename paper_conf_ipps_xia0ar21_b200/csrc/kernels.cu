@@ -136,9 +136,11 @@ __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t *s, int64_
 // Visits every intermediate product A_ik * B_kj of row i with one warp (Alg. 1 lines 3-5).
 //  * A entries are fetched 32 at a time (one per lane) together with their B row bounds and staged
 //    in the warp's shared-memory slot `st`, so the A.col -> B.rp dependency is paid once per 32
-//    entries; a round then reads its entry's bounds with one broadcast LDS.128 (+ one LDS.64 for
-//    the A value) -- shuffles would cost six LSU wavefronts per round, and the LSU data pipe
-//    (shared memory, shuffles, L1) is what bounds these kernels.
+//    entries; a round then reads its entry with ONE broadcast LDS.128: the B row's start and length
+//    packed in one word (start < 2^40, length < 2^24) next to the A value.  (Separate arrays of
+//    column / value pointers, lengths and A values cost four LDS per round: 11 % of num_w's shared
+//    wavefronts on C2, profiles/r02/; the LSU data pipe -- shared memory, shuffles, L1 -- is what
+//    bounds these kernels.)
 //  * Lanes form 32/G subgroups; subgroup g takes one B row per round and its lanes take G
 //    consecutive entries of it (coalesced).  U rounds are loaded before any is consumed, so U
 //    independent B-row loads are in flight per warp (latency, not bandwidth, bounds this loop).
@@ -147,12 +149,21 @@ __device__ __forceinline__ int64_t block_excl_scan(int64_t v, int64_t *s, int64_
 //    pass only inserts keys with atomicCAS and needs no ordering between rounds).  With
 //    G == 32 all active lanes of a round hold entries of ONE B row, i.e. distinct columns
 //    (rows are sorted and unique), which lets the numeric pass update values without atomics.
-struct AStage {
-    const int32_t *pc[32];  // &B.col[first entry of B row A.col[e]] for the 32 staged A entries
-    const double *pv[32];   // &B.val[...] (numeric pass)
-    int32_t len[32];        // length of that B row
-    double a[32];           // A values (numeric pass)
+constexpr int AST_LSH = 40;  // packed staged entry (numeric pass): B row start | length << 40
+struct __align__(16) AStage {
+    union {
+        ulonglong2 e[32];  // numeric: .x = start of B row A.col[entry] | its length << 40, .y = A value
+        struct {           // symbolic (issue-bound, not LSU-bound: no unpacking, two broadcast LDS)
+            const int32_t *pc[32];
+            int32_t len[32];
+        } s;
+    };
 };
+__device__ __forceinline__ void ast_unpack(const ulonglong2 &x, int64_t &bs, int32_t &len, double &a) {
+    bs = (int64_t)(x.x & ((1ull << AST_LSH) - 1));
+    len = (int32_t)(x.x >> AST_LSH);
+    a = __longlong_as_double((long long)x.y);
+}
 
 template <int G, int U, bool VALS, bool SYNC, typename F>
 __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR &B, int64_t i, AStage *st, F &&f) {
@@ -162,28 +173,24 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
     const int64_t as = A.rp[i], ae = A.rp[i + 1];
     for (int64_t pb = as; pb < ae; pb += 32) {
         const int64_t e = pb + lane;
-        int32_t len = 0;
-        const int32_t *pc = B.col;
-        const double *pv = B.val;
+        int64_t len = 0, bs = 0;
         double av = 0.0;
         if (e < ae) {
             const int32_t k = __ldg(&A.col[e]);
-            const int64_t bs = __ldg(&B.rp[k]);
-            len = (int32_t)(__ldg(&B.rp[k + 1]) - bs);
-            pc += bs;
-            if (VALS) {
-                pv += bs;
-                av = __ldg(&A.val[e]);
-            }
+            bs = __ldg(&B.rp[k]);
+            len = __ldg(&B.rp[k + 1]) - bs;
+            if (VALS) av = __ldg(&A.val[e]);
         }
         // rows longer than a group need the remainder loop below (never on the stencils)
         const bool any_long = __any_sync(FULLMASK, len > G);
         __syncwarp();  // the previous batch's rounds have read their entries
-        st->pc[lane] = pc;  // lanes past the row's end stage empty rows
-        st->len[lane] = len;
+        // lanes past the row's end stage empty rows
         if (VALS) {
-            st->pv[lane] = pv;
-            st->a[lane] = av;
+            st->e[lane] = make_ulonglong2((unsigned long long)bs | ((unsigned long long)len << AST_LSH),
+                                          (unsigned long long)__double_as_longlong(av));
+        } else {
+            st->s.pc[lane] = B.col + bs;
+            st->s.len[lane] = (int32_t)len;
         }
         __syncwarp();
         const int nb = (int)(ae - pb < 32 ? ae - pb : 32);
@@ -194,11 +201,16 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 const int src = t + u * R + sub;
-                ok[u] = sl < st->len[src];
-                c[u] = ok[u] ? __ldg(st->pc[src] + sl) : 0;
                 if (VALS) {
-                    a[u] = st->a[src];
-                    v[u] = ok[u] ? __ldg(st->pv[src] + sl) : 0.0;
+                    int64_t s0;
+                    int32_t ln;
+                    ast_unpack(st->e[src], s0, ln, a[u]);
+                    ok[u] = sl < ln;
+                    c[u] = ok[u] ? __ldg(B.col + s0 + sl) : 0;
+                    v[u] = ok[u] ? __ldg(B.val + s0 + sl) : 0.0;
+                } else {
+                    ok[u] = sl < st->s.len[src];
+                    c[u] = ok[u] ? __ldg(st->s.pc[src] + sl) : 0;
                 }
             }
 #pragma unroll
@@ -211,16 +223,21 @@ __device__ __forceinline__ void warp_row_products(const DevCSR &A, const DevCSR 
                 for (int u = 0; u < U; ++u) {
                     // remainder of B rows longer than G (uniform trip count across the warp)
                     const int src = t + u * R + sub;
-                    const int32_t *pc2 = st->pc[src];
-                    const double *pv2 = VALS ? st->pv[src] : nullptr;
-                    const int32_t ln2 = st->len[src];
-                    const double a2 = VALS ? st->a[src] : 0.0;
+                    int64_t s2 = 0;
+                    int32_t ln2;
+                    double a2 = 0.0;
+                    if (VALS) {
+                        ast_unpack(st->e[src], s2, ln2, a2);
+                    } else {
+                        s2 = st->s.pc[src] - B.col;
+                        ln2 = st->s.len[src];
+                    }
                     for (int o = G;; o += G) {
                         if (!__any_sync(FULLMASK, o < ln2)) break;
                         const int q = o + sl;
                         const bool okk = q < ln2;
-                        const int32_t cc = okk ? __ldg(pc2 + q) : 0;
-                        const double vv = (VALS && okk) ? __ldg(pv2 + q) : 0.0;
+                        const int32_t cc = okk ? __ldg(B.col + s2 + q) : 0;
+                        const double vv = (VALS && okk) ? __ldg(B.val + s2 + q) : 0.0;
                         f(okk, cc, VALS ? a2 * vv : 0.0);
                         if (SYNC) __syncwarp();
                     }
@@ -278,9 +295,22 @@ struct PieceSeg {
     }
 };
 
-template <int NT, bool VALS, int PB, typename SEG, typename F>
+// cp.async (LDGSTS) staging of the symbolic pass's column gathers (VERDICT r1 item 4 trial):
+// per warp two buffers of 64 columns; every lane copies and later reads only its own elements,
+// so completion of its own copies (cp.async.wait_group) is the only ordering needed.
+__device__ __forceinline__ void cp_async4(int32_t *dst, const int32_t *src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+
+template <int NT, bool VALS, int PB, bool STAGE = false, typename SEG, typename F>
 __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B, int64_t as, int64_t ae,
-                                               ProdSmemT<PB> &sm, const SEG &seg, F &&f) {
+                                               ProdSmemT<PB> &sm, const SEG &seg, F &&f,
+                                               int32_t *stg = nullptr) {
+    static_assert(!(STAGE && VALS), "cp.async staging: symbolic pass only");
     constexpr int PER = PB / NT;
     static_assert(PER * NT == PB, "batch must be a multiple of the CTA size");
     for (int64_t pb = as; pb < ae; pb += PB) {
@@ -358,7 +388,38 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
             }
         };
         const int64_t q_first = threadIdx.x - lane;  // warp-uniform
-        if (q_first < tot) {
+        if (STAGE && q_first < tot) {
+            int32_t *wb = stg + (threadIdx.x >> 5) * 128;  // this warp's two buffers of 64
+            int64_t pos[2];
+            double av[2];
+            bool ok[2], okn[2];
+            locate(q_first, pos, av, ok);
+#pragma unroll
+            for (int u = 0; u < 2; ++u)
+                if (ok[u]) cp_async4(wb + u * 32 + lane, &B.col[pos[u]]);
+            cp_async_commit();
+            int b = 0;
+            for (int64_t qb = q_first; qb < tot; qb += 2 * NT) {  // warp-uniform trip count
+                const bool more = qb + 2 * NT < tot;
+                okn[0] = okn[1] = false;
+                if (more) {
+                    locate(qb + 2 * NT, pos, av, okn);
+#pragma unroll
+                    for (int u = 0; u < 2; ++u)
+                        if (okn[u]) cp_async4(wb + (b ^ 1) * 64 + u * 32 + lane, &B.col[pos[u]]);
+                    cp_async_commit();
+                    cp_async_wait<1>();
+                } else {
+                    cp_async_wait<0>();
+                }
+#pragma unroll
+                for (int u = 0; u < 2; ++u)
+                    if (ok[u]) f(wb[b * 64 + u * 32 + lane], 0.0);
+                ok[0] = okn[0];
+                ok[1] = okn[1];
+                b ^= 1;
+            }
+        } else if (q_first < tot) {
             int64_t pos[2];
             double av[2];
             bool ok[2];
@@ -402,6 +463,11 @@ template <int NT, bool VALS, int PB, typename SEG, typename F>
 __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
                                                    const SEG &seg, F &&f) {
     range_products<NT, VALS>(A, B, A.rp[i], A.rp[i + 1], sm, seg, f);
+}
+template <int NT, bool STAGE, int PB, typename SEG, typename F>
+__device__ __forceinline__ void block_row_products_sym(const DevCSR &A, const DevCSR &B, int64_t i,
+                                                       ProdSmemT<PB> &sm, const SEG &seg, F &&f, int32_t *stg) {
+    range_products<NT, false, PB, STAGE>(A, B, A.rp[i], A.rp[i + 1], sm, seg, f, stg);
 }
 
 template <int NT, bool VALS, int PB, typename F>
@@ -769,9 +835,11 @@ __device__ __forceinline__ void row_pieces(const DevCSR &A, const DevCSR &B, int
     }
 }
 
+template <bool STAGE>
 __global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
     extern __shared__ __align__(16) int32_t keys[];
     __shared__ ProdSmem psm;
+    __shared__ __align__(16) int32_t s_stg[STAGE ? THREADS_B / 32 * 128 : 1];
     __shared__ int s_ins, s_ovf, s_span[2];
     constexpr int MAXLG = 14;  // log2(TB_SYM)
     constexpr int LIMIT = (TB_SYM / 4) * 3;
@@ -793,9 +861,9 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
                 s_ovf = 0;
             }
             __syncthreads();
-            block_row_products<THREADS_B, false>(a.A, a.B, i, psm, seg, [&](int32_t c, double) {
+            block_row_products_sym<THREADS_B, STAGE>(a.A, a.B, i, psm, seg, [&](int32_t c, double) {
                 insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
-            });  // ends with a barrier
+            }, s_stg);  // ends with a barrier
             return s_ovf == 0;
         };
         if (bound <= CAPB_SYM) {
@@ -1819,7 +1887,8 @@ const Grids &grids(int device, int num_sms) {
         set_attrs_w<8>();
         set_attrs_w<16>();
         set_attrs_w<32>();
-        cudaFuncSetAttribute(k_sym_b, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symb_smem());
+        cudaFuncSetAttribute(k_sym_b<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symb_smem());
+        cudaFuncSetAttribute(k_sym_b<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symb_smem());
         cudaFuncSetAttribute(k_num_b, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numb_smem());
         cudaFuncSetAttribute(k_sym_m, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symm_smem());
         cudaFuncSetAttribute(k_num_m, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numm_smem());
@@ -1831,7 +1900,7 @@ const Grids &grids(int device, int num_sms) {
         g.symw_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false>, WARPS_W * 32, numw_smem(false));
         g.numw_blocks = num_sms * (occ > 0 ? occ : 1);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b, THREADS_B, symb_smem());
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b<false>, THREADS_B, symb_smem());
         g.symb_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_b, THREADS_BN, numb_smem());
         g.numb_blocks = num_sms * (occ > 0 ? occ : 1);
@@ -1945,7 +2014,9 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
     }
     rec(ev, 2, s);
     if (a.tiers & 1) {
-        k_sym_b<<<a.cursor ? a.bblocks : g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
+        static const bool stage = env_int("SPGEMM_SYMB_CPASYNC", 0) == 1;  // A/B knob (cp.async trial)
+        if (stage) k_sym_b<true><<<a.cursor ? a.bblocks : g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
+        else k_sym_b<false><<<a.cursor ? a.bblocks : g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
         LAUNCHED(1);
     }
     rec(ev, 3, s);

@@ -31,7 +31,7 @@ s = torch.cuda.current_stream()
 for r in range(reps):
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    P = capi.Plan(d, d, ws.numel(), capi.opts(workspace=ws, ring=3, chunk_nnz=200_000_000, stream=s.cuda_stream))
+    P = capi.Plan(d, d, ws.numel(), capi.opts(workspace=ws, fused=True, ring=3, chunk_nnz=200_000_000, stream=s.cuda_stream))
     P.execute_stream(lambda *a: 0)
     P.free()
     torch.cuda.synchronize()

@@ -5,7 +5,7 @@ TAG=${1:-x}; shift
 KS=${@:-num_b sym_b}
 mkdir -p gpurun_out
 for K in $KS; do
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_${K}\b" --launch-skip 70 --launch-count 1 \
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:"k_${K}$" --launch-skip 70 --launch-count 1 \
      -o gpurun_out/prof_${K}_$TAG python tools/c3_once.py > gpurun_out/ncu_${K}_$TAG.log 2>&1
   python tools/ncu_summary.py gpurun_out/prof_${K}_$TAG.ncu-rep > gpurun_out/ncu_${K}_$TAG.md 2>&1
 
