@@ -358,20 +358,25 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
         // (usually 1-3 segments) instead of all nb A entries of the batch.
         const int lane = threadIdx.x & 31;
         auto locate = [&](int64_t qb, int64_t (&pos)[2], double (&a)[2], bool (&ok)[2]) {
-            int lo = 0, hi = nb;  // invariant: off[lo] <= q < off[hi]
-            if (lane < 4) {
-                const int64_t q0 = qb + (lane >> 1) * NT;
-                const int64_t qq = (lane & 1) ? min(q0 + 31, tot - 1) : min(q0, tot - 1);
-                while (hi - lo > 1) {
-                    const int mid = (lo + hi) >> 1;
-                    if (sm.off[mid] <= qq) lo = mid;
-                    else hi = mid;
-                }
+            // the four window ends (first / last product of each step) are found by four groups of
+            // 8 lanes in parallel, an 8-ary search over off[0, nb) (3 levels for PB = 512) -- the
+            // whole warp busy, instead of 4 lanes walking a 9-level binary search while 28 idle
+            const int grp = lane >> 3, k = lane & 7;
+            const int64_t q0 = qb + (grp >> 1) * NT;
+            const int64_t qq = (grp & 1) ? min(q0 + 31, tot - 1) : min(q0, tot - 1);
+            int lo = 0;  // invariant: off[lo] <= qq, answer in [lo, lo + S * 8)
+#pragma unroll
+            for (int S = PB / 8;; S = S >= 8 ? S / 8 : 1) {
+                const int idx = lo + k * S;
+                const bool le = idx < nb && sm.off[idx] <= qq;
+                const unsigned m = (__ballot_sync(FULLMASK, le) >> (grp * 8)) & 0xffu;
+                lo += (__popc(m) - 1) * S;
+                if (S == 1) break;
             }
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
                 const int64_t q = qb + u * NT + lane;
-                const int wlo = __shfl_sync(FULLMASK, lo, 2 * u), whi = __shfl_sync(FULLMASK, lo, 2 * u + 1) + 1;
+                const int wlo = __shfl_sync(FULLMASK, lo, 16 * u), whi = __shfl_sync(FULLMASK, lo, 16 * u + 8) + 1;
                 ok[u] = q < tot;
                 pos[u] = 0;
                 a[u] = 0.0;
