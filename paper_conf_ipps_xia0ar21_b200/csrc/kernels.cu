@@ -295,22 +295,9 @@ struct PieceSeg {
     }
 };
 
-// cp.async (LDGSTS) staging of the symbolic pass's column gathers (VERDICT r1 item 4 trial):
-// per warp two buffers of 64 columns; every lane copies and later reads only its own elements,
-// so completion of its own copies (cp.async.wait_group) is the only ordering needed.
-__device__ __forceinline__ void cp_async4(int32_t *dst, const int32_t *src) {
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(d), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
-
-template <int NT, bool VALS, int PB, bool STAGE = false, typename SEG, typename F>
+template <int NT, bool VALS, int PB, typename SEG, typename F>
 __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B, int64_t as, int64_t ae,
-                                               ProdSmemT<PB> &sm, const SEG &seg, F &&f,
-                                               int32_t *stg = nullptr) {
-    static_assert(!(STAGE && VALS), "cp.async staging: symbolic pass only");
+                                               ProdSmemT<PB> &sm, const SEG &seg, F &&f) {
     constexpr int PER = PB / NT;
     static_assert(PER * NT == PB, "batch must be a multiple of the CTA size");
     for (int64_t pb = as; pb < ae; pb += PB) {
@@ -351,11 +338,10 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
         // qb + NT) per iteration, software-pipelined: the gathers of the next iteration are issued
         // before the current one's products are consumed, so up to four B loads per lane are in
         // flight while the hash inserts run (long-scoreboard stalls on these loads were the top
-        // stall of the CTA kernels, profiles/r02/).  With STAGE (symbolic passes, VERDICT r1 item
-        // 4's trial) the next iteration's columns are instead copied into a per-warp shared
-        // staging buffer with cp.async (LDGSTS), double-buffered.  Four lanes find the segments
-        // of the first and last product of each step; every lane then searches only that window
-        // (usually 1-3 segments) instead of all nb A entries of the batch.
+        // stall of the CTA kernels, profiles/r02/; a cp.async double buffer of the same gathers was
+        // slower, profiles/r02/NOTES.md).  Four groups of 8 lanes find the segments of the first
+        // and last product of each step; every lane then searches only that window (usually 1-3
+        // segments) instead of all nb A entries of the batch.
         const int lane = threadIdx.x & 31;
         auto locate = [&](int64_t qb, int64_t (&pos)[2], double (&a)[2], bool (&ok)[2]) {
             // the four window ends (first / last product of each step) are found by four groups of
@@ -393,38 +379,7 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
             }
         };
         const int64_t q_first = threadIdx.x - lane;  // warp-uniform
-        if (STAGE && q_first < tot) {
-            int32_t *wb = stg + (threadIdx.x >> 5) * 128;  // this warp's two buffers of 64
-            int64_t pos[2];
-            double av[2];
-            bool ok[2], okn[2];
-            locate(q_first, pos, av, ok);
-#pragma unroll
-            for (int u = 0; u < 2; ++u)
-                if (ok[u]) cp_async4(wb + u * 32 + lane, &B.col[pos[u]]);
-            cp_async_commit();
-            int b = 0;
-            for (int64_t qb = q_first; qb < tot; qb += 2 * NT) {  // warp-uniform trip count
-                const bool more = qb + 2 * NT < tot;
-                okn[0] = okn[1] = false;
-                if (more) {
-                    locate(qb + 2 * NT, pos, av, okn);
-#pragma unroll
-                    for (int u = 0; u < 2; ++u)
-                        if (okn[u]) cp_async4(wb + (b ^ 1) * 64 + u * 32 + lane, &B.col[pos[u]]);
-                    cp_async_commit();
-                    cp_async_wait<1>();
-                } else {
-                    cp_async_wait<0>();
-                }
-#pragma unroll
-                for (int u = 0; u < 2; ++u)
-                    if (ok[u]) f(wb[b * 64 + u * 32 + lane], 0.0);
-                ok[0] = okn[0];
-                ok[1] = okn[1];
-                b ^= 1;
-            }
-        } else if (q_first < tot) {
+        if (q_first < tot) {
             int64_t pos[2];
             double av[2];
             bool ok[2];
@@ -468,11 +423,6 @@ template <int NT, bool VALS, int PB, typename SEG, typename F>
 __device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
                                                    const SEG &seg, F &&f) {
     range_products<NT, VALS>(A, B, A.rp[i], A.rp[i + 1], sm, seg, f);
-}
-template <int NT, bool STAGE, int PB, typename SEG, typename F>
-__device__ __forceinline__ void block_row_products_sym(const DevCSR &A, const DevCSR &B, int64_t i,
-                                                       ProdSmemT<PB> &sm, const SEG &seg, F &&f, int32_t *stg) {
-    range_products<NT, false, PB, STAGE>(A, B, A.rp[i], A.rp[i + 1], sm, seg, f, stg);
 }
 
 template <int NT, bool VALS, int PB, typename F>
@@ -840,11 +790,9 @@ __device__ __forceinline__ void row_pieces(const DevCSR &A, const DevCSR &B, int
     }
 }
 
-template <bool STAGE>
 __global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
     extern __shared__ __align__(16) int32_t keys[];
     __shared__ ProdSmem psm;
-    __shared__ __align__(16) int32_t s_stg[STAGE ? THREADS_B / 32 * 128 : 1];
     __shared__ int s_ins, s_ovf, s_span[2];
     constexpr int MAXLG = 14;  // log2(TB_SYM)
     constexpr int LIMIT = (TB_SYM / 4) * 3;
@@ -866,9 +814,9 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
                 s_ovf = 0;
             }
             __syncthreads();
-            block_row_products_sym<THREADS_B, STAGE>(a.A, a.B, i, psm, seg, [&](int32_t c, double) {
+            block_row_products<THREADS_B, false>(a.A, a.B, i, psm, seg, [&](int32_t c, double) {
                 insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
-            }, s_stg);  // ends with a barrier
+            });  // ends with a barrier
             return s_ovf == 0;
         };
         if (bound <= CAPB_SYM) {
@@ -1892,8 +1840,7 @@ const Grids &grids(int device, int num_sms) {
         set_attrs_w<8>();
         set_attrs_w<16>();
         set_attrs_w<32>();
-        cudaFuncSetAttribute(k_sym_b<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symb_smem());
-        cudaFuncSetAttribute(k_sym_b<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symb_smem());
+        cudaFuncSetAttribute(k_sym_b, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symb_smem());
         cudaFuncSetAttribute(k_num_b, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numb_smem());
         cudaFuncSetAttribute(k_sym_m, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)symm_smem());
         cudaFuncSetAttribute(k_num_m, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)numm_smem());
@@ -1905,7 +1852,7 @@ const Grids &grids(int device, int num_sms) {
         g.symw_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_w<32, false>, WARPS_W * 32, numw_smem(false));
         g.numw_blocks = num_sms * (occ > 0 ? occ : 1);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b<false>, THREADS_B, symb_smem());
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sym_b, THREADS_B, symb_smem());
         g.symb_blocks = num_sms * (occ > 0 ? occ : 1);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_num_b, THREADS_BN, numb_smem());
         g.numb_blocks = num_sms * (occ > 0 ? occ : 1);
@@ -2019,9 +1966,7 @@ void launch_symbolic(const SymArgs &a, int num_sms, cudaStream_t s, cudaEvent_t 
     }
     rec(ev, 2, s);
     if (a.tiers & 1) {
-        static const bool stage = env_int("SPGEMM_SYMB_CPASYNC", 0) == 1;  // A/B knob (cp.async trial)
-        if (stage) k_sym_b<true><<<a.cursor ? a.bblocks : g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
-        else k_sym_b<false><<<a.cursor ? a.bblocks : g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
+        k_sym_b<<<a.cursor ? a.bblocks : g.symb_blocks, THREADS_B, symb_smem(), s>>>(a);
         LAUNCHED(1);
     }
     rec(ev, 3, s);
