@@ -1449,7 +1449,14 @@ __device__ __forceinline__ T warp_incl_scan(T x) {
 // staged in the output value area; a coarse bucket over 512 keys the general path (compaction +
 // shared-memory bitonic).  Writes oc/ov [0, n); returns false (nothing written) if the table does
 // not hold exactly n keys.  All threads call; ends with a barrier; the key table is clobbered.
-template <int SB, int NT = THREADS_B>
+// ZV: the value table is left all zero (each value is cleared where it is read; the rare paths
+// clear the whole table), so that the next pass need not refill it.
+__device__ __forceinline__ void cswap_u32(uint32_t &a, uint32_t &b) {
+    const uint32_t x = min(a, b), y = max(a, b);
+    a = x;
+    b = y;
+}
+template <int SB, int NT = THREADS_B, bool ZV = false>
 __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int32_t *oc, double *ov,
                               CtaSortSmemT<NT> &ss, SortCntT<NT> &sc) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -1499,6 +1506,8 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
 #pragma unroll
     for (int w = 0; w < NW; ++w) occ_total += ss.occ[w];
     if (occ_total != n || n == 0) {
+        if (ZV && occ_total != n)
+            for (int t = threadIdx.x; t < T; t += NT) vals[t] = 0.0;
         __syncthreads();
         return occ_total == n;
     }
@@ -1562,25 +1571,51 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
             // consecutive buckets, so one-key buckets give coalesced stores.  (Ranking every key
             // against its bucket-mates made each warp wait for its lane with the largest bucket:
             // 17 % of num_b's instructions, profiles/r02/ncu_numb_c3_v4.)
+            // A bucket of <= 4 keys (99.6 % at ~1 key per bucket) is sorted by a 5-comparator network
+            // on predicated loads -- every lane the same instructions; a larger bucket by insertion
+            // sort.  (The per-bucket loops alone made each warp wait for its lane with the largest
+            // bucket: the owner loop was 25 % of num_b's instructions at 3.8 active lanes per
+            // instruction, profiles/r02/NOTES.md.)
             const int nb_used = (int)(((span - 1) >> sh) + 1);
             const uint32_t slotmask = (1u << SB) - 1u;
             for (int b = threadIdx.x; b < nb_used; b += NT) {
                 const int e0 = (int)((sc.arr[b >> 1] >> ((b & 1) << 4)) & 0xffffu);
                 const int s0 = b == 0 ? 0 : (int)((sc.arr[(b - 1) >> 1] >> (((b - 1) & 1) << 4)) & 0xffffu);
-                for (int p = s0 + 1; p < e0; ++p) {  // insertion sort of the bucket's staged words
-                    const uint32_t v = stg[p];
-                    int q = p - 1;
-                    while (q >= s0 && stg[q] > v) {
-                        stg[q + 1] = stg[q];
-                        --q;
-                    }
-                    stg[q + 1] = v;
-                }
+                const int m = e0 - s0;
                 const int64_t cb = lo + ((int64_t)b << sh);
-                for (int p = s0; p < e0; ++p) {
-                    const uint32_t x = stg[p];
-                    oc[p] = (int32_t)(cb + (x >> SB));
-                    ov[p] = vals[x & slotmask];
+                if (m <= 4) {
+                    uint32_t w[4];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) w[q] = q < m ? stg[s0 + q] : 0xffffffffu;
+                    cswap_u32(w[0], w[1]);
+                    cswap_u32(w[2], w[3]);
+                    cswap_u32(w[0], w[2]);
+                    cswap_u32(w[1], w[3]);
+                    cswap_u32(w[1], w[2]);
+#pragma unroll
+                    for (int q = 0; q < 4; ++q)
+                        if (q < m) {
+                            const uint32_t sl = w[q] & slotmask;
+                            oc[s0 + q] = (int32_t)(cb + (w[q] >> SB));
+                            ov[s0 + q] = vals[sl];
+                            if (ZV) vals[sl] = 0.0;
+                        }
+                } else {
+                    for (int p = s0 + 1; p < e0; ++p) {  // insertion sort of the bucket's staged words
+                        const uint32_t v = stg[p];
+                        int q = p - 1;
+                        while (q >= s0 && stg[q] > v) {
+                            stg[q + 1] = stg[q];
+                            --q;
+                        }
+                        stg[q + 1] = v;
+                    }
+                    for (int p = s0; p < e0; ++p) {
+                        const uint32_t x = stg[p];
+                        oc[p] = (int32_t)(cb + (x >> SB));
+                        ov[p] = vals[x & slotmask];
+                        if (ZV) vals[x & slotmask] = 0.0;
+                    }
                 }
             }
             __syncthreads();
@@ -1624,6 +1659,11 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
             sort_emit_any<SB, true, false>(stage + st, m, vals, oc + st, ov + st);
         }
         __syncthreads();
+        if (ZV) {
+            for (int t = threadIdx.x; t < T; t += NT)
+                if (keys[t] != EMPTY) vals[t] = 0.0;
+            __syncthreads();
+        }
         return true;
     }
     // general path: in-place compaction + shared-memory bitonic sort
@@ -1651,6 +1691,10 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
         ov[t] = vals[t];
     }
     __syncthreads();
+    if (ZV) {
+        for (int t = threadIdx.x; t < T; t += NT) vals[t] = 0.0;
+        __syncthreads();
+    }
     return true;
 }
 
@@ -1671,6 +1715,14 @@ __global__ void __launch_bounds__(THREADS_BN, 1024 / THREADS_BN) k_num_b(NumArgs
     const int64_t R = a.r1 - a.r0;
     const int64_t off0 = a.crp[a.r0];
     __shared__ unsigned s_idx;
+    // the value table is zeroed once here and kept zero by cta_sort_emit<.., ZV> (each value cleared
+    // where the sort reads it); only a piece abandoned on overflow leaves it dirty
+    auto zero_vals = [&]() {
+        double2 *v2 = reinterpret_cast<double2 *>(vals);
+        for (int t = threadIdx.x; t < TB_NUM / 2; t += THREADS_BN) v2[t] = make_double2(0.0, 0.0);
+    };
+    zero_vals();  // (cta_claim's barrier follows)
+    bool dirty = false;
     for (unsigned idx = cta_claim(&a.ctl->bctr, &s_idx); idx < nrows; idx = cta_claim(&a.ctl->bctr, &s_idx)) {
         const int64_t i = a.listB[idx < nh ? int64_t(idx) : R - 1 - int64_t(idx - nh)];
         const int64_t o = a.crp[i];
@@ -1679,10 +1731,10 @@ __global__ void __launch_bounds__(THREADS_BN, 1024 / THREADS_BN) k_num_b(NumArgs
         double *ov = a.out_val + (o - off0);
         auto pass = [&](int lg, const auto &seg, int limit) {
             const int T = 1 << lg;
-            for (int t = threadIdx.x; t < T; t += THREADS_BN) {
-                keys[t] = EMPTY;
-                vals[t] = 0.0;
-            }
+            if (dirty) zero_vals();
+            dirty = false;
+            int4 *k4 = reinterpret_cast<int4 *>(keys);
+            for (int t = threadIdx.x; t < T / 4; t += THREADS_BN) k4[t] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
             if (threadIdx.x == 0) {
                 s_ins = 0;
                 s_ovf = 0;
@@ -1692,13 +1744,14 @@ __global__ void __launch_bounds__(THREADS_BN, 1024 / THREADS_BN) k_num_b(NumArgs
                 const int h = insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
                 if (h >= 0) atomicAdd(&vals[h], v);
             });  // ends with a barrier
-            return s_ovf == 0;
+            dirty = s_ovf != 0;
+            return !dirty;
         };
         bool ok = true;
         if (n <= CAPB_NUM) {
             const int lg = table_log2(n, MAXLG);
             pass(lg, WholeSeg{}, INT_MAX);
-            ok = cta_sort_emit<MAXLG, THREADS_BN>(keys, vals, 1 << lg, n, oc, ov, ss, u.sc);
+            ok = cta_sort_emit<MAXLG, THREADS_BN, true>(keys, vals, 1 << lg, n, oc, ov, ss, u.sc);
         } else {
             int64_t written = 0;
             row_pieces<THREADS_BN>(
@@ -1706,8 +1759,13 @@ __global__ void __launch_bounds__(THREADS_BN, 1024 / THREADS_BN) k_num_b(NumArgs
                 [&](int32_t lo, int32_t hi) { return pass(MAXLG, PieceSeg{a.B.col, cur, nxt, hi}, LIMIT); },
                 [&]() {
                     const int m = s_ins;
-                    if (written + m <= n) ok &= cta_sort_emit<MAXLG, THREADS_BN>(keys, vals, TB_NUM, m, oc + written, ov + written, ss, u.sc);
-                    else ok = false;
+                    if (written + m <= n) {
+                        ok &= cta_sort_emit<MAXLG, THREADS_BN, true>(keys, vals, TB_NUM, m, oc + written, ov + written,
+                                                                     ss, u.sc);
+                    } else {
+                        ok = false;
+                        dirty = true;
+                    }
                     written += m;
                 });
             ok &= written == n;
@@ -1732,21 +1790,23 @@ __global__ void __launch_bounds__(THREADS_M, 6) k_num_m(NumArgs a) {
     const unsigned nrows = *(volatile unsigned *)&a.ctl->nM;
     const int64_t off0 = a.crp[a.r0];
     __shared__ unsigned s_idx;
+    {  // zero once; cta_sort_emit<.., ZV> keeps the value table zero (cta_claim's barrier follows)
+        double2 *v2 = reinterpret_cast<double2 *>(vals);
+        for (int t = threadIdx.x; t < TM_NUM / 2; t += THREADS_M) v2[t] = make_double2(0.0, 0.0);
+    }
     for (unsigned idx = cta_claim(&a.ctl->mctr, &s_idx); idx < nrows; idx = cta_claim(&a.ctl->mctr, &s_idx)) {
         const int64_t i = a.listM[idx];
         const int64_t o = a.crp[i];
         const int64_t n = a.crp[i + 1] - o;
         const int lg = table_log2(n, MAXLG);
         const int T = 1 << lg;
-        for (int t = threadIdx.x; t < T; t += THREADS_M) {
-            keys[t] = EMPTY;
-            vals[t] = 0.0;
-        }
+        int4 *k4 = reinterpret_cast<int4 *>(keys);
+        for (int t = threadIdx.x; t < T / 4; t += THREADS_M) k4[t] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
         __syncthreads();
         block_row_products<THREADS_M, true>(a.A, a.B, i, u.psm, [&](int32_t c, double v) {
             atomicAdd(&vals[find_slot(keys, c, lg)], v);
         });  // ends with a barrier
-        const bool ok = cta_sort_emit<MAXLG, THREADS_M>(keys, vals, T, n, a.out_col + (o - off0),
+        const bool ok = cta_sort_emit<MAXLG, THREADS_M, true>(keys, vals, T, n, a.out_col + (o - off0),
                                                         a.out_val + (o - off0), ss, u.sc);
         if (!ok && threadIdx.x == 0) atomicOr(&a.ctl->err, 1u);
         __syncthreads();
