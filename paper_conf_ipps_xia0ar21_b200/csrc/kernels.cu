@@ -19,6 +19,7 @@
 #include <cstdlib>
 
 #include <atomic>
+#include <type_traits>
 
 #include "internal.h"
 
@@ -263,6 +264,7 @@ struct ProdSmemT {
     int64_t bs[PB];
     double a[PB];
     int64_t scan[40];
+    unsigned next;  // next claim of 64 products (dynamic distribution over the warps)
 };
 using ProdSmem = ProdSmemT<PBATCH>;
 
@@ -332,23 +334,29 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
             if (e < nb) sm.off[e] = run;
             run += lens[r];
         }
-        if (threadIdx.x == 0) sm.off[nb] = tot;
+        constexpr int NW = NT / 32;
+        if (threadIdx.x == 0) {
+            sm.off[nb] = tot;
+            sm.next = NW;  // claims 0 .. NW-1 are the warps' first ones
+        }
         __syncthreads();
-        // Each warp takes 32 consecutive products per step (coalesced B loads), two steps (qb,
-        // qb + NT) per iteration, software-pipelined: the gathers of the next iteration are issued
-        // before the current one's products are consumed, so up to four B loads per lane are in
-        // flight while the hash inserts run (long-scoreboard stalls on these loads were the top
-        // stall of the CTA kernels, profiles/r02/; a cp.async double buffer of the same gathers was
-        // slower, profiles/r02/NOTES.md).  Four groups of 8 lanes find the segments of the first
-        // and last product of each step; every lane then searches only that window (usually 1-3
-        // segments) instead of all nb A entries of the batch.
+        // Each warp claims 64 consecutive products at a time (two steps of 32: coalesced B loads)
+        // from a shared counter, so a warp whose inserts probed longer takes fewer claims -- with a
+        // static stride the warps left the batch up to a step apart and the barrier after it was
+        // the top stall of the CTA kernels (14 % of num_b's and 24 % of sym_b's stall samples,
+        // profiles/r02/NOTES.md).  Software-pipelined: the next claim and its gathers are issued
+        // before the current products are consumed, so up to four B loads per lane are in flight
+        // while the hash inserts run (a cp.async double buffer of the same gathers was slower).
+        // Four groups of 8 lanes find the segments of the first and last product of each step;
+        // every lane then searches only that window (usually 1-3 segments) instead of all nb A
+        // entries of the batch.
         const int lane = threadIdx.x & 31;
         auto locate = [&](int64_t qb, int64_t (&pos)[2], double (&a)[2], bool (&ok)[2]) {
             // the four window ends (first / last product of each step) are found by four groups of
             // 8 lanes in parallel, an 8-ary search over off[0, nb) (3 levels for PB = 512) -- the
             // whole warp busy, instead of 4 lanes walking a 9-level binary search while 28 idle
             const int grp = lane >> 3, k = lane & 7;
-            const int64_t q0 = qb + (grp >> 1) * NT;
+            const int64_t q0 = qb + (grp >> 1) * 32;
             const int64_t qq = (grp & 1) ? min(q0 + 31, tot - 1) : min(q0, tot - 1);
             int lo = 0;  // invariant: off[lo] <= qq, answer in [lo, lo + S * 8)
 #pragma unroll
@@ -361,7 +369,7 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
             }
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
-                const int64_t q = qb + u * NT + lane;
+                const int64_t q = qb + u * 32 + lane;
                 const int wlo = __shfl_sync(FULLMASK, lo, 16 * u), whi = __shfl_sync(FULLMASK, lo, 16 * u + 8) + 1;
                 ok[u] = q < tot;
                 pos[u] = 0;
@@ -378,25 +386,28 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
                 }
             }
         };
-        const int64_t q_first = threadIdx.x - lane;  // warp-uniform
-        if (q_first < tot) {
+        int64_t qb = (int64_t)(threadIdx.x >> 5) * 64;  // warp-uniform
+        if (qb < tot) {
             int64_t pos[2];
             double av[2];
             bool ok[2];
             int32_t c[2];
             double v[2];
-            locate(q_first, pos, av, ok);
+            locate(qb, pos, av, ok);
 #pragma unroll
             for (int u = 0; u < 2; ++u) {
                 c[u] = ok[u] ? __ldg(&B.col[pos[u]]) : 0;
                 v[u] = (VALS && ok[u]) ? av[u] * __ldg(&B.val[pos[u]]) : 0.0;
             }
-            for (int64_t qb = q_first; qb < tot; qb += 2 * NT) {  // warp-uniform trip count
+            while (true) {
+                unsigned nc = 0;
+                if (lane == 0) nc = atomicAdd(&sm.next, 1u);
+                const int64_t qn = (int64_t)__shfl_sync(FULLMASK, nc, 0) * 64;
                 int32_t cn[2] = {0, 0};
                 double vn[2] = {0.0, 0.0};
                 bool okn[2] = {false, false};
-                if (qb + 2 * NT < tot) {  // next iteration's gathers first
-                    locate(qb + 2 * NT, pos, av, okn);
+                if (qn < tot) {  // next claim's gathers first
+                    locate(qn, pos, av, okn);
 #pragma unroll
                     for (int u = 0; u < 2; ++u) {
                         cn[u] = okn[u] ? __ldg(&B.col[pos[u]]) : 0;
@@ -406,6 +417,7 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
 #pragma unroll
                 for (int u = 0; u < 2; ++u)
                     if (ok[u]) f(c[u], v[u]);
+                if (qn >= tot) break;
 #pragma unroll
                 for (int u = 0; u < 2; ++u) {
                     c[u] = cn[u];
@@ -1740,9 +1752,15 @@ __global__ void __launch_bounds__(THREADS_BN, 1024 / THREADS_BN) k_num_b(NumArgs
                 s_ovf = 0;
             }
             __syncthreads();
+            // a whole row's key count is known (n) and its table cannot overflow: no counting
+            constexpr bool whole = std::is_same<std::decay_t<decltype(seg)>, WholeSeg>::value;
             block_row_products<THREADS_BN, true>(a.A, a.B, i, psm, seg, [&](int32_t c, double v) {
-                const int h = insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
-                if (h >= 0) atomicAdd(&vals[h], v);
+                if (whole) {
+                    atomicAdd(&vals[find_slot(keys, c, lg)], v);
+                } else {
+                    const int h = insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
+                    if (h >= 0) atomicAdd(&vals[h], v);
+                }
             });  // ends with a barrier
             dirty = s_ovf != 0;
             return !dirty;
