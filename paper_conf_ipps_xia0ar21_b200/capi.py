@@ -15,7 +15,9 @@ from typing import Callable, Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libspgemm_b200.so")
+# SPGEMM_CHECKED=1 loads the checked build (device-side bounds checks that trap; build.py), for tests
+LIB_PATH = os.path.join(_HERE, "libspgemm_b200_checked.so" if os.environ.get("SPGEMM_CHECKED") == "1"
+                        else "libspgemm_b200.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

@@ -30,6 +30,24 @@ long long kernel_launches() { return g_launches.load(); }
 #define LAUNCHED(n) g_launches.fetch_add((n), std::memory_order_relaxed)
 
 #define FULLMASK 0xffffffffu
+
+// Device-side bounds checks of the checked build (libspgemm_b200_checked.so, -DSPGEMM_CHECKS;
+// compute-sanitizer is not available on the GPU pool): a failed check prints its site and traps.
+// In the product build they compile to nothing.
+#ifdef SPGEMM_CHECKS
+#define SPG_CHECK(cond)                                                                                   \
+    do {                                                                                                  \
+        if (!(cond)) {                                                                                    \
+            printf("SPG_CHECK failed: %s (%s:%d) block %d thread %d\n", #cond, __FILE__, __LINE__,       \
+                   (int)blockIdx.x, (int)threadIdx.x);                                                    \
+            __trap();                                                                                     \
+        }                                                                                                 \
+    } while (0)
+#else
+#define SPG_CHECK(cond) \
+    do {                \
+    } while (0)
+#endif
 constexpr int32_t EMPTY = -1;
 
 // Home slot of column c in a table of 2^lg slots: multiplicative (Fibonacci) hashing.  (A variant
@@ -285,6 +303,7 @@ struct PieceSeg {
     int32_t *nxt;
     int32_t hi;
     __device__ __forceinline__ void operator()(int e, int32_t, int64_t s0, int64_t e0, int64_t &s, int64_t &en) const {
+        SPG_CHECK(cur[e] >= 0 && s0 + cur[e] <= e0);
         s = s0 + cur[e];
         int64_t lo = s, h = e0;
         while (lo < h) {
@@ -382,6 +401,8 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
                         else h2 = mid;
                     }
                     pos[u] = sm.bs[l2] + (q - sm.off[l2]);
+                    SPG_CHECK(l2 >= 0 && l2 < nb && q >= sm.off[l2] && q < sm.off[l2 + 1]);
+                    SPG_CHECK(pos[u] >= B.rp[0] && pos[u] < B.rp[B.nrows]);
                     if (VALS) a[u] = sm.a[l2];
                 }
             }
@@ -625,18 +646,22 @@ __device__ __forceinline__ void push_long(int64_t i, int64_t bound, const DevCSR
                                           int32_t *listB, int32_t *listG, Ctl *ctl, int64_t cap) {
     if (listM != nullptr && bound <= capM) {
         unsigned idx = atomicAdd(&ctl->nM, 1u);
+        SPG_CHECK(idx < cap);
         listM[idx] = (int32_t)i;
         return;
     }
     const bool pieces_ok = cursor != nullptr && bound <= capS && A.rp[i + 1] - A.rp[i] <= curstride;
     if (bound <= capB) {
         unsigned idx = atomicAdd(&ctl->nBl, 1u);
+        SPG_CHECK(idx < cap);
         listB[cap - 1 - idx] = (int32_t)i;
     } else if (pieces_ok) {
         unsigned idx = atomicAdd(&ctl->nB, 1u);
+        SPG_CHECK(idx < cap);
         listB[idx] = (int32_t)i;
     } else {
         unsigned idx = atomicAdd(&ctl->nG, 1u);
+        SPG_CHECK(idx < cap);
         listG[idx] = (int32_t)i;
     }
 }
@@ -820,15 +845,26 @@ __global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
         // one table pass over the products of [lo, hi) (whole row: seg = WholeSeg)
         auto pass = [&](int lg, const auto &seg, int limit) {
             const int T = 1 << lg;
-            for (int t = threadIdx.x; t < T; t += THREADS_B) keys[t] = EMPTY;
+            int4 *k4 = reinterpret_cast<int4 *>(keys);
+            for (int t = threadIdx.x; t < T / 4; t += THREADS_B) k4[t] = make_int4(EMPTY, EMPTY, EMPTY, EMPTY);
             if (threadIdx.x == 0) {
                 s_ins = 0;
                 s_ovf = 0;
             }
             __syncthreads();
+            // a whole row's table cannot overflow (>= 2 x bound slots): fresh keys are counted per
+            // thread and reduced once, instead of a ballot + shared atomic per insert
+            constexpr bool whole = std::is_same<std::decay_t<decltype(seg)>, WholeSeg>::value;
+            int mine = 0;
             block_row_products<THREADS_B, false>(a.A, a.B, i, psm, seg, [&](int32_t c, double) {
-                insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
+                if (whole) mine += sym_insert(keys, c, lg);
+                else insert_counted(keys, c, lg, &s_ins, limit, &s_ovf);
             });  // ends with a barrier
+            if (whole) {
+                mine = warp_sum(mine);
+                if ((threadIdx.x & 31) == 0 && mine) atomicAdd(&s_ins, mine);
+                __syncthreads();
+            }
             return s_ovf == 0;
         };
         if (bound <= CAPB_SYM) {
@@ -1003,6 +1039,7 @@ __global__ void __launch_bounds__(THREADS_G) k_num_g1(NumArgs a) {
     int64_t p0, p1;
     part_range(a.A, i, p0, p1);
     range_products<THREADS_G, true>(a.A, a.B, p0, p1, psm, WholeSeg{}, [&](int32_t c, double v) {
+        SPG_CHECK(c >= 0 && c < a.B.ncols);
         atomicOr(&bm[c >> 5], 1u << (c & 31));
         atomicAdd(&dv[c], v);
     });
@@ -1260,6 +1297,7 @@ __device__ __forceinline__ void sort_emit(const K *pk, int n, const double *vals
     for (int r = 0; r < E; ++r) {
         const int e = (r << 5) | lane;
         if (e < n) {
+            SPG_CHECK((int)(x[r] & ((K(1) << SB) - 1u)) < (1 << SB));
             oc[e] = (int32_t)(x[r] >> SB);
             const int slot = (int)(x[r] & ((K(1) << SB) - 1u));
             ov[e] = V_G ? __ldcg(vals + slot) : vals[slot];
@@ -1575,6 +1613,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
                     const uint32_t d = (uint32_t)((int64_t)kr[j] - lo);
                     const uint32_t b = d >> sh, hs = (b & 1u) << 4;
                     const int pos = (int)((atomicAdd(&sc.arr[b >> 1], 1u << hs) >> hs) & 0xffffu);
+                    SPG_CHECK(b < (1u << pl) && pos >= 0 && pos < n);
                     stg[pos] = ((d & relmask) << SB) | (uint32_t)(j * NT + threadIdx.x);
                 }
             __syncthreads();
@@ -1608,6 +1647,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
                     for (int q = 0; q < 4; ++q)
                         if (q < m) {
                             const uint32_t sl = w[q] & slotmask;
+                            SPG_CHECK(s0 + q < n && (int)sl < T);
                             oc[s0 + q] = (int32_t)(cb + (w[q] >> SB));
                             ov[s0 + q] = vals[sl];
                             if (ZV) vals[sl] = 0.0;
@@ -1624,6 +1664,7 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
                     }
                     for (int p = s0; p < e0; ++p) {
                         const uint32_t x = stg[p];
+                        SPG_CHECK(p < n && (int)(x & slotmask) < T);
                         oc[p] = (int32_t)(cb + (x >> SB));
                         ov[p] = vals[x & slotmask];
                         if (ZV) vals[x & slotmask] = 0.0;

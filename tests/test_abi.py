@@ -145,3 +145,20 @@ def test_order_needs_two_phase_plan(capi):
     o = capi.opts(order=2)
     assert capi._lib.spgemm_plan(ctypes.byref(ca), ctypes.byref(ca), 0, ctypes.byref(o), ctypes.byref(h)) == \
         capi.ERR_INVALID_ARGUMENT
+
+
+def test_checked_library_exports_the_same_abi_and_product_has_no_checks():
+    """libspgemm_b200_checked.so (SPG_CHECK bounds checks, tests only) exports exactly the product
+    library's C ABI; the product library carries none of the checks."""
+    pkg = os.path.join(ROOT, "paper_conf_ipps_xia0ar21_b200")
+
+    def syms(name):
+        out = subprocess.run(["nm", "-D", "--defined-only", os.path.join(pkg, name)], capture_output=True,
+                             text=True).stdout
+        return {ln.split()[-1] for ln in out.splitlines() if " T spgemm_" in ln}
+
+    prod, chk = syms("libspgemm_b200.so"), syms("libspgemm_b200_checked.so")
+    assert prod and prod == chk
+    blob = open(os.path.join(pkg, "libspgemm_b200.so"), "rb").read()
+    assert b"SPG_CHECK failed" not in blob
+    assert b"SPG_CHECK failed" in open(os.path.join(pkg, "libspgemm_b200_checked.so"), "rb").read()

@@ -1,5 +1,6 @@
 """Small multiplies through every path for compute-sanitizer (memcheck / racecheck / synccheck):
-in-core two-phase and fused plans (host cut included), forced chunking, long-row tiers, column panels, sink mode."""
+in-core two-phase and fused plans (host cut included), forced chunking, long-row tiers (medium, CTA whole / pieced,
+dense), column panels.  Run under every compute-sanitizer tool (memcheck, racecheck, synccheck, initcheck)."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
@@ -40,4 +41,9 @@ for kw in ({"fused": True}, {"fused": True, "chunk_nnz": 3000, "ring": 1}):
     run(S, S, **kw)
     run(R, R, **kw)
 del os.environ["SPGEMM_PIECE_NNZ"]
+# power-law rows through the medium, CTA (whole and pieced) and dense tiers: R-MAT s12 with a small
+# dense-slot count and pieces forced by a wide column span
+R2 = W.rmat(12, 16, seed=7)
+run(R2, R2, fused=True)
+run(R2, R2, chunk_nnz=200_000, ring=2)
 print("sanitize cases ok")
