@@ -37,7 +37,10 @@ constexpr int TW_NUM = 512, CAPW_NUM = 256;
 constexpr int THREADS_M = 128;             // medium tier: 16 KB (symbolic) / 24 KB (numeric) tables
 constexpr int TM_SYM = 4096, CAPM_SYM = 2048;
 constexpr int TM_NUM = 2048, CAPM_NUM = 1024;
-constexpr int THREADS_B = 512;             // 2 CTAs per SM (96 KB / 64 KB of table + 13 KB)
+// symbolic CTA tier: 512 threads, 16 K-slot tables, 2 CTAs per SM.  Measured on C3 (round 2): 256
+// threads / 8 K slots / pieces of 4096 at 4 CTAs per SM gave the same sym_b time (383 ms) but sent
+// 6x more rows to the dense tier (sym_g 30 -> 89 ms)
+constexpr int THREADS_B = 512;
 constexpr int TB_SYM = 16384, CAPB_SYM = 8192;
 // numeric CTA tier: 512 threads, 2 CTAs per SM (96 KB table + 13 KB each).  Measured on C3
 // (tools/tier_times.py): 256 threads / 4 K slots / pieces of 2048 took 1180 ms, 1024 threads /

@@ -827,11 +827,12 @@ __device__ __forceinline__ void row_pieces(const DevCSR &A, const DevCSR &B, int
     }
 }
 
-__global__ void __launch_bounds__(THREADS_B, 2) k_sym_b(SymArgs a) {
+__global__ void __launch_bounds__(THREADS_B, 1024 / THREADS_B) k_sym_b(SymArgs a) {
     extern __shared__ __align__(16) int32_t keys[];
     __shared__ ProdSmem psm;
     __shared__ int s_ins, s_ovf, s_span[2];
-    constexpr int MAXLG = 14;  // log2(TB_SYM)
+    constexpr int MAXLG = TB_SYM == 16384 ? 14 : TB_SYM == 8192 ? 13 : 12;  // log2(TB_SYM)
+    static_assert((1 << MAXLG) == TB_SYM, "table size");
     constexpr int LIMIT = (TB_SYM / 4) * 3;
     int32_t *cur = a.cursor ? a.cursor + (int64_t)blockIdx.x * 2 * a.curstride : nullptr;
     int32_t *nxt = cur ? cur + a.curstride : nullptr;
@@ -1453,7 +1454,6 @@ struct CtaSortSmemT {
     int mm[3], occ[NT / 32];
     int64_t scan[40];
 };
-using CtaSortSmem = CtaSortSmemT<THREADS_B>;
 
 // fine-bucket cursors of the CTA sort: 8 NT buckets, two 16-bit cursors per word (positions are
 // < 2^16); one array serves as histogram, bucket start, staging cursor and -- once staged -- bucket
@@ -1468,13 +1468,11 @@ struct SortCntT {
         } co;
     };
 };
-using SortCnt = SortCntT<THREADS_B>;
 template <int NT, int PB>
 union ProdOrSortT {
     ProdSmemT<PB> psm;
     SortCntT<NT> sc;
 };
-using ProdOrSort = ProdOrSortT<THREADS_B, PBATCH>;
 
 template <typename T>
 __device__ __forceinline__ T warp_incl_scan(T x) {
