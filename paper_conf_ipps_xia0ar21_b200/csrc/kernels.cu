@@ -316,11 +316,15 @@ struct PieceSeg {
     }
 };
 
+// f(col, value) or f(col, value, q) with q the product's index in the flattened sequence of the
+// range (0 .. total-1, batch after batch).  Returns the total number of products (every thread).
 template <int NT, bool VALS, int PB, typename SEG, typename F>
-__device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B, int64_t as, int64_t ae,
-                                               ProdSmemT<PB> &sm, const SEG &seg, F &&f) {
+__device__ __forceinline__ int64_t range_products(const DevCSR &A, const DevCSR &B, int64_t as, int64_t ae,
+                                                  ProdSmemT<PB> &sm, const SEG &seg, F &&f) {
     constexpr int PER = PB / NT;
     static_assert(PER * NT == PB, "batch must be a multiple of the CTA size");
+    constexpr bool WITH_Q = std::is_invocable<F, int32_t, double, int64_t>::value;
+    int64_t qbase = 0;
     for (int64_t pb = as; pb < ae; pb += PB) {
         const int nb = (int)(ae - pb < PB ? ae - pb : PB);
         int64_t lens[PER];
@@ -420,6 +424,7 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
                 c[u] = ok[u] ? __ldg(&B.col[pos[u]]) : 0;
                 v[u] = (VALS && ok[u]) ? av[u] * __ldg(&B.val[pos[u]]) : 0.0;
             }
+            int64_t qc = qb;  // first product of the claim being consumed
             while (true) {
                 unsigned nc = 0;
                 if (lane == 0) nc = atomicAdd(&sm.next, 1u);
@@ -437,8 +442,12 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
                 }
 #pragma unroll
                 for (int u = 0; u < 2; ++u)
-                    if (ok[u]) f(c[u], v[u]);
+                    if (ok[u]) {
+                        if constexpr (WITH_Q) f(c[u], v[u], qbase + qc + u * 32 + lane);
+                        else f(c[u], v[u]);
+                    }
                 if (qn >= tot) break;
+                qc = qn;
 #pragma unroll
                 for (int u = 0; u < 2; ++u) {
                     c[u] = cn[u];
@@ -447,21 +456,23 @@ __device__ __forceinline__ void range_products(const DevCSR &A, const DevCSR &B,
                 }
             }
         }
+        qbase += tot;
         __syncthreads();
     }
+    return qbase;
 }
 
 // all products of row i (A entries [A.rp[i], A.rp[i+1]))
 template <int NT, bool VALS, int PB, typename SEG, typename F>
-__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
-                                                   const SEG &seg, F &&f) {
-    range_products<NT, VALS>(A, B, A.rp[i], A.rp[i + 1], sm, seg, f);
+__device__ __forceinline__ int64_t block_row_products(const DevCSR &A, const DevCSR &B, int64_t i,
+                                                      ProdSmemT<PB> &sm, const SEG &seg, F &&f) {
+    return range_products<NT, VALS>(A, B, A.rp[i], A.rp[i + 1], sm, seg, f);
 }
 
 template <int NT, bool VALS, int PB, typename F>
-__device__ __forceinline__ void block_row_products(const DevCSR &A, const DevCSR &B, int64_t i, ProdSmemT<PB> &sm,
-                                                   F &&f) {
-    range_products<NT, VALS>(A, B, A.rp[i], A.rp[i + 1], sm, WholeSeg{}, f);
+__device__ __forceinline__ int64_t block_row_products(const DevCSR &A, const DevCSR &B, int64_t i,
+                                                      ProdSmemT<PB> &sm, F &&f) {
+    return range_products<NT, VALS>(A, B, A.rp[i], A.rp[i + 1], sm, WholeSeg{}, f);
 }
 
 // find-or-insert of a column in a warp-private table; returns the slot
@@ -1467,6 +1478,7 @@ struct SortCntT {
             int cnt[64], cur[64], start[64];  // coarse buckets of the clustered-column fallback
         } co;
     };
+    int esc_w[8][NT / 32];  // esc_sort_emit: per owner round and warp, the distinct count
 };
 template <int NT, int PB>
 union ProdOrSortT {
@@ -1749,10 +1761,216 @@ __device__ bool cta_sort_emit(int32_t *keys, double *vals, int T, int64_t n, int
     return true;
 }
 
+// ------------------------------------------------------------ S6+S7 by sorting the products (ESC)
+//
+// The numeric CTA tier's rows and pieces are nearly all-distinct on power-law inputs (C3: 1.06
+// products per nonzero), so accumulating them in a hash table and then sorting the table does the
+// work twice: every product is an unsuccessful hash search with a CAS, and then every key is
+// bucket-sorted.  Here the products themselves are sorted (expand - sort - compress): the product
+// iterator stores product q's column and value at index q (no atomics, no probing; consecutive
+// lanes, consecutive q), the products are bucketed by column (~1 per fine bucket, a histogram, a
+// scan and a staging pass as in cta_sort_emit), each bucket is sorted by (column, q) and equal
+// columns merged -- values summed in product order -- and a prefix over the buckets' distinct
+// counts places every bucket's output.  Up to ESC_CAP products per pass (16 B each: value, column,
+// staged word, in the 96 KB of the hash table).
+constexpr int ESC_CAP = TB_NUM * 12 / 16;  // 6144
+
+// u products in pc / pv [0, u) with columns in [lo, hi]; writes the distinct columns in order and
+// their summed values to oc / ov.  Returns the number of distinct columns, -1 if some fine bucket
+// holds more than 64 products (clustered or heavily repeated columns: the caller uses the hash
+// path), -2 if there are more than nmax distinct columns (nothing written).  All threads call;
+// ends with a barrier; stg and the sort counters are clobbered.
+template <int NT>
+__device__ int esc_sort_emit(const int32_t *pc, const double *pv, uint32_t *stg, int u, int32_t lo, int32_t hi,
+                             int64_t nmax, int32_t *oc, double *ov, CtaSortSmemT<NT> &ss, SortCntT<NT> &sc) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    constexpr int NW = NT / 32;
+    constexpr int PLMAX = NT == 1024 ? 13 : NT == 512 ? 12 : NT == 256 ? 11 : NT == 128 ? 10 : 9;  // 2^PLMAX = 8 NT
+    if (u == 0) return 0;
+    const int QB = 32 - __clz(max(u, 2) - 1);  // bits of a product index (2^QB >= u)
+    const int pl = min(PLMAX, max(5, QB));     // 2^pl fine buckets, ~1 product each
+    const int64_t span = (int64_t)hi - lo + 1;
+    const int lspan = span <= 1 ? 0 : 64 - __clzll(span - 1);
+    const int sh = max(0, lspan - pl);         // sh + QB <= lspan + 1 <= 32
+    const uint32_t relmask = (1u << sh) - 1u, qmask = (1u << QB) - 1u;
+    for (int w = threadIdx.x; w < (1 << (pl - 1)); w += NT) sc.arr[w] = 0u;
+    __syncthreads();
+    for (int q = threadIdx.x; q < u; q += NT) {  // histogram (16-bit counters, two per word)
+        const uint32_t b = (uint32_t)(pc[q] - lo) >> sh;
+        atomicAdd(&sc.arr[b >> 1], 1u << ((b & 1u) << 4));
+    }
+    __syncthreads();
+    {  // bucket starts: thread t owns words 4t .. 4t+3 (buckets 8t .. 8t+7)
+        const int w0 = 4 * threadIdx.x;
+        const bool mine = w0 < (1 << (pl - 1));
+        uint32_t wv[4];
+        int sum = 0, big = 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            wv[q] = mine ? sc.arr[w0 + q] : 0u;
+            const int c0 = (int)(wv[q] & 0xffffu), c1 = (int)(wv[q] >> 16);
+            sum += c0 + c1;
+            big = max(big, max(c0, c1));
+        }
+        int64_t tot;
+        int run = (int)block_excl_scan<NT>(sum, ss.scan, &tot);  // ends with a barrier
+        if (mine) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int c0 = (int)(wv[q] & 0xffffu), c1 = (int)(wv[q] >> 16);
+                sc.arr[w0 + q] = (uint32_t)run | ((uint32_t)(run + c0) << 16);
+                run += c0 + c1;
+            }
+        }
+#pragma unroll
+        for (int d = 16; d > 0; d >>= 1) big = max(big, __shfl_xor_sync(FULLMASK, big, d));
+        if (lane == 0) ss.occ[wid] = big;
+        __syncthreads();
+        int bmax = 0;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) bmax = max(bmax, ss.occ[w]);
+        if (bmax > 64) {
+            __syncthreads();
+            return -1;
+        }
+    }
+    for (int q = threadIdx.x; q < u; q += NT) {  // stage (offset in the bucket << QB | q) in its bucket
+        const uint32_t d = (uint32_t)(pc[q] - lo);
+        const uint32_t b = d >> sh, hs = (b & 1u) << 4;
+        const int pos = (int)((atomicAdd(&sc.arr[b >> 1], 1u << hs) >> hs) & 0xffffu);
+        SPG_CHECK(b < (1u << pl) && pos >= 0 && pos < u);
+        stg[pos] = ((d & relmask) << QB) | (uint32_t)q;
+    }
+    __syncthreads();
+    // owner pass 1 (bucket b = k NT + thread): sort in place by (column, q), count distinct columns
+    const int nb_used = (int)(((span - 1) >> sh) + 1);
+    auto bucket = [&](int b, int &s0, int &e0) {
+        e0 = (int)((sc.arr[b >> 1] >> ((b & 1) << 4)) & 0xffffu);
+        s0 = b == 0 ? 0 : (int)((sc.arr[(b - 1) >> 1] >> (((b - 1) & 1) << 4)) & 0xffffu);
+    };
+    int pos0[8];  // per round: the exclusive prefix of the distinct counts (-> first output position)
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+        const int b = k * NT + threadIdx.x;
+        int dd = 0;
+        if (b < nb_used) {
+            int s0, e0;
+            bucket(b, s0, e0);
+            const int m = e0 - s0;
+            if (m <= 4) {
+                uint32_t w[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) w[q] = q < m ? stg[s0 + q] : 0xffffffffu;
+                cswap_u32(w[0], w[1]);
+                cswap_u32(w[2], w[3]);
+                cswap_u32(w[0], w[2]);
+                cswap_u32(w[1], w[3]);
+                cswap_u32(w[1], w[2]);
+                dd = m > 0;
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    if (q < m) {
+                        stg[s0 + q] = w[q];
+                        if (q > 0) dd += (w[q] >> QB) != (w[q - 1] >> QB);
+                    }
+            } else {
+                // insertion sort by column only: a large bucket is mostly repeats of a few (hub)
+                // columns, already in order among themselves (their values are summed in any order,
+                // as by the hash path's atomics)
+                for (int p = s0 + 1; p < e0; ++p) {
+                    const uint32_t v = stg[p];
+                    int q = p - 1;
+                    while (q >= s0 && (stg[q] >> QB) > (v >> QB)) {
+                        stg[q + 1] = stg[q];
+                        --q;
+                    }
+                    stg[q + 1] = v;
+                }
+                dd = 1;
+                for (int p = s0 + 1; p < e0; ++p) dd += (stg[p] >> QB) != (stg[p - 1] >> QB);
+            }
+        }
+        const int inc = warp_incl_scan(dd);
+        pos0[k] = inc - dd;
+        if (lane == 31) sc.esc_w[k][wid] = inc;
+    }
+    __syncthreads();
+    // every warp scans the per-warp totals of each round itself (one barrier instead of two)
+    int total = 0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+        const int x = lane < NW ? sc.esc_w[k][lane] : 0;
+        const int y = warp_incl_scan(x);
+        pos0[k] += total + __shfl_sync(FULLMASK, y - x, wid);
+        total += __shfl_sync(FULLMASK, y, 31);
+    }
+    if (total > nmax) {
+        __syncthreads();
+        return -2;
+    }
+    // owner pass 2: merge equal columns (values summed in product order) and write the bucket
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+        const int b = k * NT + threadIdx.x;
+        int s0 = 0, e0 = 0;
+        if (b < nb_used) bucket(b, s0, e0);
+        const int m = e0 - s0;
+        if (m > 0) {
+            const int64_t cb = lo + ((int64_t)b << sh);
+            int pos = pos0[k];
+            uint32_t prev = stg[s0];
+            double acc = pv[prev & qmask];
+            prev >>= QB;
+            if (m <= 4) {
+#pragma unroll
+                for (int q = 1; q < 4; ++q)
+                    if (q < m) {
+                        const uint32_t x = stg[s0 + q];
+                        const double v = pv[x & qmask];
+                        if ((x >> QB) != prev) {
+                            SPG_CHECK(pos < total);
+                            oc[pos] = (int32_t)(cb + prev);
+                            ov[pos] = acc;
+                            ++pos;
+                            prev = x >> QB;
+                            acc = v;
+                        } else {
+                            acc += v;
+                        }
+                    }
+            } else {
+                for (int p = s0 + 1; p < e0; ++p) {
+                    const uint32_t x = stg[p];
+                    const double v = pv[x & qmask];
+                    if ((x >> QB) != prev) {
+                        SPG_CHECK(pos < total);
+                        oc[pos] = (int32_t)(cb + prev);
+                        ov[pos] = acc;
+                        ++pos;
+                        prev = x >> QB;
+                        acc = v;
+                    } else {
+                        acc += v;
+                    }
+                }
+            }
+            SPG_CHECK(pos < total);
+            oc[pos] = (int32_t)(cb + prev);
+            ov[pos] = acc;
+        }
+    }
+    __syncthreads();
+    return total;
+}
+
 __global__ void __launch_bounds__(THREADS_BN, 1024 / THREADS_BN) k_num_b(NumArgs a) {
     extern __shared__ __align__(16) double smem_d[];
-    double *vals = smem_d;
-    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);
+    double *vals = smem_d;                                          // hash path: TB_NUM values
+    int32_t *keys = reinterpret_cast<int32_t *>(smem_d + TB_NUM);   // ... and TB_NUM keys
+    double *pv = smem_d;                                            // ESC path (same 96 KB): values,
+    int32_t *pc = reinterpret_cast<int32_t *>(smem_d + ESC_CAP);    // columns and staged words of
+    uint32_t *stg = reinterpret_cast<uint32_t *>(pc + ESC_CAP);     // up to ESC_CAP products
+    static_assert(ESC_CAP * 16 <= TB_NUM * 12, "ESC staging fits the table");
     __shared__ ProdOrSortT<THREADS_BN, PBATCH_BN> u;
     ProdSmemT<PBATCH_BN> &psm = u.psm;
     __shared__ CtaSortSmemT<THREADS_BN> ss;
@@ -1804,17 +2022,82 @@ __global__ void __launch_bounds__(THREADS_BN, 1024 / THREADS_BN) k_num_b(NumArgs
             dirty = s_ovf != 0;
             return !dirty;
         };
+        // ESC pass over the products of seg: 1 = done (*m distinct columns written to ocw / ovw),
+        // 0 = more than ESC_CAP products, -1 = a fine bucket over 64 products, -2 = more than nmax
+        // distinct columns.  It overwrites the hash tables (dirty).
+        auto esc_pass = [&](const auto &seg, int64_t nmax, int32_t *ocw, double *ovw, int &m) {
+            if (threadIdx.x == 0) {
+                ss.mm[0] = INT_MAX;
+                ss.mm[1] = -1;
+            }
+            dirty = true;
+            __syncthreads();
+            int lmin = INT_MAX, lmax = -1;
+            const int64_t nprod = block_row_products<THREADS_BN, true>(
+                a.A, a.B, i, psm, seg, [&](int32_t c, double v, int64_t q) {
+                    if (q < ESC_CAP) {
+                        pc[q] = c;
+                        pv[q] = v;
+                        lmin = min(lmin, (int)c);
+                        lmax = max(lmax, (int)c);
+                    }
+                });  // ends with a barrier
+            if (nprod > ESC_CAP) return 0;
+#pragma unroll
+            for (int d = 16; d > 0; d >>= 1) {
+                lmin = min(lmin, __shfl_xor_sync(FULLMASK, lmin, d));
+                lmax = max(lmax, __shfl_xor_sync(FULLMASK, lmax, d));
+            }
+            if ((threadIdx.x & 31) == 0 && lmax >= 0) {
+                atomicMin(&ss.mm[0], lmin);
+                atomicMax(&ss.mm[1], lmax);
+            }
+            __syncthreads();
+            const int r = esc_sort_emit<THREADS_BN>(pc, pv, stg, (int)nprod, ss.mm[0], ss.mm[1], nmax, ocw, ovw, ss,
+                                                    u.sc);
+            m = r;
+            return r >= 0 ? 1 : r;
+        };
         bool ok = true;
         if (n <= CAPB_NUM) {
-            const int lg = table_log2(n, MAXLG);
-            pass(lg, WholeSeg{}, INT_MAX);
-            ok = cta_sort_emit<MAXLG, THREADS_BN, true>(keys, vals, 1 << lg, n, oc, ov, ss, u.sc);
+            int m = 0;
+            const int r = esc_pass(WholeSeg{}, n, oc, ov, m);
+            if (r == 1) {
+                ok = m == n;
+            } else if (r == -2) {
+                ok = false;
+            } else {  // too many products or clustered columns: hash table + table sort
+                const int lg = table_log2(n, MAXLG);
+                pass(lg, WholeSeg{}, INT_MAX);
+                ok = cta_sort_emit<MAXLG, THREADS_BN, true>(keys, vals, 1 << lg, n, oc, ov, ss, u.sc);
+            }
         } else {
             int64_t written = 0;
+            int esc_m = 0;  // >= 0: the piece was written by the ESC pass; -1: by the hash path
             row_pieces<THREADS_BN>(
                 a.A, a.B, i, n, PIECE_NUM, cur, nxt, s_span,
-                [&](int32_t lo, int32_t hi) { return pass(MAXLG, PieceSeg{a.B.col, cur, nxt, hi}, LIMIT); },
+                [&](int32_t lo, int32_t hi) {
+                    const PieceSeg sg{a.B.col, cur, nxt, hi};
+                    int m = 0;
+                    const int r = esc_pass(sg, n - written, oc + written, ov + written, m);
+                    if (r == 0) return false;  // too many products: the piece is halved
+                    if (r == 1) {
+                        esc_m = m;
+                        return true;
+                    }
+                    if (r == -2) {
+                        esc_m = 0;
+                        ok = false;
+                        return true;
+                    }
+                    esc_m = -1;  // clustered columns: this piece through the hash table
+                    return pass(MAXLG, sg, LIMIT);
+                },
                 [&]() {
+                    if (esc_m >= 0) {
+                        written += esc_m;
+                        return;
+                    }
                     const int m = s_ins;
                     if (written + m <= n) {
                         ok &= cta_sort_emit<MAXLG, THREADS_BN, true>(keys, vals, TB_NUM, m, oc + written, ov + written,
