@@ -306,10 +306,24 @@ struct PieceSeg {
         SPG_CHECK(cur[e] >= 0 && s0 + cur[e] <= e0);
         s = s0 + cur[e];
         int64_t lo = s, h = e0;
-        while (lo < h) {
+        if (lo < h) {
+            // the row's last column is loaded next to the first midpoint (independent loads): in
+            // the row's last piece -- and for every B row that ends before hi -- the search ends
+            // there, instead of after log2(length) dependent loads
             const int64_t m = (lo + h) >> 1;
-            if (__ldg(&bcol[m]) < hi) lo = m + 1;
-            else h = m;
+            const int32_t cl = __ldg(&bcol[h - 1]), cm = __ldg(&bcol[m]);
+            if (cl < hi) {
+                lo = h;
+            } else {
+                if (cm < hi) lo = m + 1;
+                else h = m;
+                h = min(h, e0 - 1);  // bcol[e0 - 1] >= hi
+                while (lo < h) {
+                    const int64_t m2 = (lo + h) >> 1;
+                    if (__ldg(&bcol[m2]) < hi) lo = m2 + 1;
+                    else h = m2;
+                }
+            }
         }
         en = lo;
         nxt[e] = (int32_t)(lo - s0);
