@@ -202,12 +202,10 @@ def tier_constants():
     txt = open(os.path.join(ROOT, "paper_conf_ipps_xia0ar21_b200", "csrc", "internal.h")).read()
     out = {}
     for k in ("CAPW_SYM", "CAPW_NUM", "CAPB_SYM", "CAPB_NUM", "PIECE_SYM", "PIECE_NUM", "CURSOR_MAX", "CAPM_SYM",
-              "CAPM_NUM"):
+              "CAPM_NUM", "CAPS_SYM", "CAPS_NUM"):
         m = re.search(rf"\b{k}\s*=\s*(\d+)", txt)
         if m:
             out[k] = int(m.group(1))
-    out["CAPS_SYM"] = 32 * out["PIECE_SYM"]
-    out["CAPS_NUM"] = 32 * out["PIECE_NUM"]
     return out
 
 

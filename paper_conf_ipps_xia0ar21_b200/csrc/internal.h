@@ -47,8 +47,11 @@ constexpr int TB_SYM = 16384, CAPB_SYM = 8192;
 // 16 K slots / pieces of 8192 took 1061 ms, this configuration 997 ms.
 constexpr int THREADS_BN = 512, PBATCH_BN = 512;
 constexpr int TB_NUM = 8192, CAPB_NUM = 4096;
-constexpr int PIECE_SYM = 8192, PIECE_NUM = 4096;   // target bound / nnz per column piece
-constexpr int64_t CAPS_SYM = 32 * int64_t(PIECE_SYM), CAPS_NUM = 32 * int64_t(PIECE_NUM);  // <= 32 pieces
+// target bound / nnz per column piece, measured on C3 (profiles/r02/NOTES.md): numeric 3584 / 4096 /
+// 4608 / 5120 / 5632 -> 915 / 878 / 853 / 838 / 960 ms (an ESC pass holds <= 6144 products);
+// symbolic 10240 / 8192 / 6144 / 4096 -> 426 / 380 / 349 / 350 ms
+constexpr int PIECE_SYM = 6144, PIECE_NUM = 5120;
+constexpr int64_t CAPS_SYM = 262144, CAPS_NUM = 131072;  // longest pieced row (bound / nnz); beyond: dense tier
 constexpr int CURSOR_MAX = 32768;          // longest A row a pieced row may have (cursor scratch)
 constexpr int THREADS_G = 512;
 // dense tier, split rows: a row is accumulated by KG_PARTS CTAs (1/KG_PARTS of its A entries each)
