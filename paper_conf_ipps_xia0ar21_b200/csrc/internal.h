@@ -46,7 +46,9 @@ constexpr int TB_SYM = 16384, CAPB_SYM = 8192;
 // (tools/tier_times.py): 256 threads / 4 K slots / pieces of 2048 took 1180 ms, 1024 threads /
 // 16 K slots / pieces of 8192 took 1061 ms, this configuration 997 ms.
 constexpr int THREADS_BN = 512, PBATCH_BN = 512;
-constexpr int TB_NUM = 8192, CAPB_NUM = 4096;
+// whole rows up to 5120 nonzeros (the ESC pass holds 6144 products; the hash fallback's 8 K table is
+// then up to 5/8 full): 4096 -> 5120 took C3's num_b from 831 to 815 ms
+constexpr int TB_NUM = 8192, CAPB_NUM = 5120;
 // target bound / nnz per column piece, measured on C3 (profiles/r02/NOTES.md): numeric 3584 / 4096 /
 // 4608 / 5120 / 5632 -> 915 / 878 / 853 / 838 / 960 ms (an ESC pass holds <= 6144 products);
 // symbolic 10240 / 8192 / 6144 / 4096 -> 426 / 380 / 349 / 350 ms
